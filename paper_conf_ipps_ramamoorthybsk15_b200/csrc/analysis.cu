@@ -1,0 +1,302 @@
+// analysis.cu — Phase I of the method: per-row intermediate-product
+// counts, classification of rows into light/heavy classes (the paper's Boolean H/L array,
+// generalised to a few classes), log2 flop histogram, and the scans/split points the
+// symbolic phase and the multi-GPU partitioner need.
+#include "kernels.cuh"
+
+namespace spg {
+
+// f_i = sum over stored A(i,k) of len_B(k); nz_i = #entries with len_B(k) > 0 (capped at 2).
+// One block owns ROWS consecutive rows; its threads stride over the rows' A entries
+// (coalesced colA loads), find the owning row by binary search in the cached row_ptr
+// tile, and accumulate with shared-memory atomics.  Hub rows (thousands of entries) are
+// thereby spread over the whole block instead of one thread.
+template <int ROWS>
+__global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict__ rpA, const int* __restrict__ colA,
+                                                    int K, const int* __restrict__ rpB, int* __restrict__ f_out,
+                                                    uint8_t* __restrict__ nz_out, unsigned long long* __restrict__ hist,
+                                                    int* __restrict__ err) {
+  __shared__ int s_rp[ROWS + 1];
+  __shared__ unsigned long long s_f[ROWS];
+  __shared__ int s_nz[ROWS];
+  __shared__ unsigned s_hist[65];
+  const int t = threadIdx.x;
+  const int r0 = blockIdx.x * ROWS;
+  const int nr = min(ROWS, M - r0);
+  if (t <= nr) s_rp[t] = rpA[r0 + t];
+  if (t == 0 && nr == ROWS) s_rp[ROWS] = rpA[r0 + ROWS];
+  s_f[t] = 0;
+  s_nz[t] = 0;
+  if (t < 65) s_hist[t] = 0;
+  __syncthreads();
+  const int e0 = s_rp[0], e1 = s_rp[nr];
+  int bad = 0;
+  for (int e = e0 + t; e < e1; e += ROWS) {
+    int k = colA[e];
+    if ((unsigned)k >= (unsigned)K) { bad = 1; continue; }
+    int L = rpB[k + 1] - rpB[k];
+    int r = upper_idx(s_rp, nr, e);
+    atomicAdd(&s_f[r], (unsigned long long)L);
+    if (L > 0) atomicAdd(&s_nz[r], 1);
+  }
+  __syncthreads();
+  if (t < nr) {
+    unsigned long long f = s_f[t];
+    if (f > (unsigned long long)INT_MAX) { bad |= 2; f = INT_MAX; }
+    f_out[r0 + t] = (int)f;
+    nz_out[r0 + t] = (uint8_t)min(s_nz[t], 2);
+    int b = f == 0 ? 0 : 1 + (f == 1 ? 0 : 32 - __clz((int)f - 1));
+    atomicAdd(&s_hist[b], 1u);
+  }
+  if (bad) atomicOr(err, bad);
+  __syncthreads();
+  if (t < 65 && s_hist[t]) atomicAdd(&hist[t], (unsigned long long)s_hist[t]);
+}
+
+__device__ __forceinline__ int classify(int f, int nz, const ClassParams& p) {
+  if (f == 0) return CLS_EMPTY;
+  if (p.force < 0 && nz == 1 && p.single_ok) return CLS_SINGLE;
+  int c;
+  if (f <= TINY_MAX) c = CLS_TINY;
+  else if (f <= p.light_max) c = CLS_LIGHT;
+  else if (f <= p.medium_max) c = CLS_MEDIUM;
+  else if (f <= p.heavy_max) c = CLS_HEAVY;
+  else c = CLS_HUGE;
+  if (p.force > c) c = p.force;
+  return c;
+}
+
+// Classify this rank's rows [rb, re): append each row to its class list (warp-aggregated
+// atomics), write c_i for rows whose nnz(C) is known without work (EMPTY: 0; SINGLE: f_i,
+// B canonical), and accumulate per-class row/flop statistics.
+__global__ void __launch_bounds__(256) k_classify(const int* __restrict__ f, const uint8_t* __restrict__ nz,
+                                                  int rb_h, int re_h, const int* __restrict__ range_d,
+                                                  ClassParams prm, ClassLists lists, int* __restrict__ counts,
+                                                  unsigned long long* __restrict__ cstats /* [2*NUM_CLS + 2] */,
+                                                  long long* __restrict__ crow) {
+  const int rb = range_d ? range_d[0] : rb_h;
+  const int re = range_d ? range_d[1] : re_h;
+  const int lane = lane_id();
+  __shared__ unsigned long long s_rows[NUM_CLS], s_flops[NUM_CLS], s_fmax, s_ftot;
+  if (threadIdx.x < NUM_CLS) { s_rows[threadIdx.x] = 0; s_flops[threadIdx.x] = 0; }
+  if (threadIdx.x == 0) { s_fmax = 0; s_ftot = 0; }
+  __syncthreads();
+  unsigned long long fmax = 0, ftot = 0;
+  // every warp runs the same number of iterations so the warp collectives are uniform
+  const long long n = (long long)re - rb;
+  const long long stride = (long long)gridDim.x * blockDim.x;
+  for (long long base = (long long)blockIdx.x * blockDim.x; base < n; base += stride) {
+    const long long li = base + threadIdx.x;
+    const bool act = li < n;
+    int cls = -1, fi = 0;
+    if (act) {
+      const int i = rb + (int)li;
+      fi = f[i];
+      cls = classify(fi, nz[i], prm);
+      if (cls == CLS_EMPTY) crow[li + 1] = 0;
+      else if (cls == CLS_SINGLE) crow[li + 1] = fi;
+      fmax = max(fmax, (unsigned long long)fi);
+      ftot += fi;
+    }
+    const bool listed = act && cls >= CLS_TINY;
+    const unsigned grp = __match_any_sync(FULL, listed ? cls : -1);
+    const int leader = __ffs(grp) - 1;
+    int pos = 0;
+    if (listed && lane == leader) pos = atomicAdd(&counts[cls], __popc(grp));
+    pos = __shfl_sync(FULL, pos, leader);
+    if (listed) lists.rows[cls][pos + __popc(grp & lanemask_lt())] = rb + (int)li;
+    if (act) {
+      atomicAdd(&s_rows[cls], 1ull);
+      atomicAdd(&s_flops[cls], (unsigned long long)fi);
+    }
+  }
+  atomicMax(&s_fmax, fmax);
+  atomicAdd(&s_ftot, ftot);
+  __syncthreads();
+  if (threadIdx.x < NUM_CLS) {
+    if (s_rows[threadIdx.x]) atomicAdd(&cstats[threadIdx.x], s_rows[threadIdx.x]);
+    if (s_flops[threadIdx.x]) atomicAdd(&cstats[NUM_CLS + threadIdx.x], s_flops[threadIdx.x]);
+  }
+  if (threadIdx.x == 0) {
+    atomicMax(&cstats[2 * NUM_CLS], s_fmax);
+    atomicAdd(&cstats[2 * NUM_CLS + 1], s_ftot);
+  }
+}
+
+// ---- inclusive scan to int64 (three passes: tile scan, tile-sum scan, add) -------------------
+constexpr int SCAN_NT = 256, SCAN_IPT = 8, SCAN_TILE = SCAN_NT * SCAN_IPT;
+
+template <typename Tin>
+__global__ void __launch_bounds__(SCAN_NT) k_scan_tiles(const Tin* __restrict__ in, long long* __restrict__ out,
+                                                        long long n, long long* __restrict__ tile_sums) {
+  __shared__ long long s_w[SCAN_NT / 32];
+  const long long base = (long long)blockIdx.x * SCAN_TILE + (long long)threadIdx.x * SCAN_IPT;
+  long long v[SCAN_IPT];
+  long long run = 0;
+#pragma unroll
+  for (int k = 0; k < SCAN_IPT; ++k) {
+    long long x = base + k < n ? (long long)in[base + k] : 0;
+    run += x;
+    v[k] = run;
+  }
+  // block exclusive scan of per-thread totals
+  long long incl = warp_incl_scan(run);
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 31) s_w[w] = incl;
+  __syncthreads();
+  if (w == 0) {
+    long long x = lane < SCAN_NT / 32 ? s_w[lane] : 0;
+    long long xi = warp_incl_scan(x);
+    if (lane < SCAN_NT / 32) s_w[lane] = xi - x;
+    if (lane == SCAN_NT / 32 - 1) tile_sums[blockIdx.x] = xi;
+  }
+  __syncthreads();
+  const long long off = incl - run + s_w[w];
+#pragma unroll
+  for (int k = 0; k < SCAN_IPT; ++k)
+    if (base + k < n) out[base + k] = v[k] + off;
+}
+
+// Exclusive scan of tile sums in place (one block, sequential over chunks).
+__global__ void __launch_bounds__(1024) k_scan_tile_sums(long long* __restrict__ s, int ntiles) {
+  __shared__ long long s_w[32];
+  __shared__ long long s_carry;
+  if (threadIdx.x == 0) s_carry = 0;
+  __syncthreads();
+  for (int c0 = 0; c0 < ntiles; c0 += 1024) {
+    const int i = c0 + threadIdx.x;
+    long long x = i < ntiles ? s[i] : 0;
+    long long incl = warp_incl_scan(x);
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (lane == 31) s_w[w] = incl;
+    __syncthreads();
+    if (w == 0) {
+      long long y = s_w[lane];
+      long long yi = warp_incl_scan(y);
+      s_w[lane] = yi - y;
+    }
+    __syncthreads();
+    long long excl = incl - x + s_w[w] + s_carry;
+    __syncthreads();
+    if (i < ntiles) s[i] = excl;
+    if (threadIdx.x == 1023) s_carry = excl + x;
+    __syncthreads();
+  }
+}
+
+__global__ void __launch_bounds__(SCAN_NT) k_scan_add(long long* __restrict__ out, long long n,
+                                                      const long long* __restrict__ tile_off) {
+  const long long base = (long long)blockIdx.x * SCAN_TILE;
+  const long long add = tile_off[blockIdx.x];
+  if (add == 0) return;
+  for (int k = threadIdx.x; k < SCAN_TILE; k += SCAN_NT)
+    if (base + k < n) out[base + k] += add;
+}
+
+// s_0 = 0, s_P = M, s_r = min{ i : Pf[i]*P >= r*F }.  Pf = int64[M+1].
+__global__ void k_split_points(const long long* __restrict__ Pf, int M, int P, int* __restrict__ s) {
+  const int r = threadIdx.x + blockIdx.x * blockDim.x;
+  if (r > P) return;
+  if (r == 0) { s[0] = 0; return; }
+  if (r == P) { s[P] = M; return; }
+  const __int128 F = Pf[M];
+  const __int128 target = (__int128)r * F;
+  int lo = 0, hi = M;  // smallest i in [0, M] with Pf[i]*P >= target (Pf[M]*P >= target holds)
+  while (lo < hi) {
+    int mid = lo + ((hi - lo) >> 1);
+    if ((__int128)Pf[mid] * P >= target) hi = mid; else lo = mid + 1;
+  }
+  s[r] = lo;
+}
+
+// SPG_OPT_VALIDATE: err |= 4 malformed row_ptr, 8 column out of range, 16 row not strictly ascending.
+__global__ void k_validate(int M, const int* __restrict__ rp, const int* __restrict__ ci, int ncols, long long nnz,
+                           int check_sorted, int* __restrict__ err) {
+  int bad = 0;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < M; i += (long long)gridDim.x * blockDim.x) {
+    const int s = rp[i], e = rp[i + 1];
+    if (s > e || s < 0 || (long long)e > nnz) { bad |= 4; continue; }
+    if (i == 0 && s != 0) bad |= 4;
+    if (i == M - 1 && (long long)e != nnz) bad |= 4;
+    int prev = -1;
+    for (int p = s; p < e; ++p) {
+      const int c = ci[p];
+      if (c < 0 || c >= ncols) bad |= 8;
+      if (check_sorted && c <= prev) bad |= 16;
+      prev = c;
+    }
+  }
+  if (M == 0 && nnz != 0 && blockIdx.x == 0 && threadIdx.x == 0) bad |= 4;
+  if (bad) atomicOr(err, bad);
+}
+
+// row_ptr_full[i] += off[r] for the rank r owning row i; row_ptr_full[M] = off[P].
+__global__ void k_rebase(long long* __restrict__ rp, int M, int P, const int* __restrict__ sp,
+                         const long long* __restrict__ off) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i <= M; i += (long long)gridDim.x * blockDim.x) {
+    if (i == M) { rp[M] = off[P]; continue; }
+    int lo = 0, hi = P - 1;  // largest r with sp[r] <= i
+    while (lo < hi) { int mid = (lo + hi + 1) >> 1; if (sp[mid] <= i) lo = mid; else hi = mid - 1; }
+    rp[i] += off[lo];
+  }
+}
+
+// ---- host launchers ------------------------------------------------------------------------
+cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB,
+                             int* f, uint8_t* nz, unsigned long long* hist, int* err) {
+  if (M <= 0) return cudaSuccess;
+  constexpr int ROWS = 256;
+  k_row_flops<ROWS><<<(M + ROWS - 1) / ROWS, ROWS, 0, st>>>(M, rpA, colA, K, rpB, f, nz, hist, err);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
+                            const int* range_d, const ClassParams& prm, const ClassLists& lists, int* counts,
+                            unsigned long long* cstats, long long* crow) {
+  long long n = range_d ? (long long)re : (long long)re - rb;  // range_d: re is an upper bound on the count
+  if (n <= 0) return cudaSuccess;
+  long long blocks = (n + 255) / 256;
+  if (blocks > (long long)sms * 8) blocks = (long long)sms * 8;
+  k_classify<<<(int)blocks, 256, 0, st>>>(f, nz, rb, re, range_d, prm, lists, counts, cstats, crow);
+  return cudaGetLastError();
+}
+
+size_t scan_tmp_elems(long long n) { return (size_t)((n + SCAN_TILE - 1) / SCAN_TILE) + 1; }
+int scan_launches(long long n) { return n <= 0 ? 0 : (n > SCAN_TILE ? 3 : 1); }
+
+template <typename Tin>
+cudaError_t launch_incl_scan(cudaStream_t st, const Tin* in, long long* out, long long n, long long* tmp) {
+  if (n <= 0) return cudaSuccess;
+  const int ntiles = (int)((n + SCAN_TILE - 1) / SCAN_TILE);
+  k_scan_tiles<Tin><<<ntiles, SCAN_NT, 0, st>>>(in, out, n, tmp);
+  if (ntiles > 1) {
+    k_scan_tile_sums<<<1, 1024, 0, st>>>(tmp, ntiles);
+    k_scan_add<<<ntiles, SCAN_NT, 0, st>>>(out, n, tmp);
+  }
+  return cudaGetLastError();
+}
+template cudaError_t launch_incl_scan<int>(cudaStream_t, const int*, long long*, long long, long long*);
+template cudaError_t launch_incl_scan<long long>(cudaStream_t, const long long*, long long*, long long, long long*);
+
+cudaError_t launch_validate(cudaStream_t st, int sms, int M, const int* rp, const int* ci, int ncols, long long nnz,
+                            int check_sorted, int* err) {
+  int grid = (M + 255) / 256;
+  if (grid > sms * 8) grid = sms * 8;
+  if (grid < 1) grid = 1;
+  k_validate<<<grid, 256, 0, st>>>(M, rp, ci, ncols, nnz, check_sorted, err);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_rebase(cudaStream_t st, long long* rp_full, int M, int P, const int* splits, const long long* off) {
+  int grid = (M + 1 + 255) / 256;
+  if (grid > 4096) grid = 4096;
+  k_rebase<<<grid, 256, 0, st>>>(rp_full, M, P, splits, off);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_split_points(cudaStream_t st, const long long* Pf, int M, int P, int* s) {
+  k_split_points<<<(P + 1 + 127) / 128, 128, 0, st>>>(Pf, M, P, s);
+  return cudaGetLastError();
+}
+
+}  // namespace spg

@@ -1,0 +1,815 @@
+// capi.cu — the C ABI of include/spg.h: handle, options, workspace, orchestration of the
+// analysis -> symbolic -> numeric pipeline on the handle's stream (class kernels forked onto
+// concurrent streams), the host-buffer end-to-end path and the NCCL multi-GPU pieces.
+#include <nccl.h>
+
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "kernels.cuh"
+#include "spg.h"
+
+using namespace spg;
+
+namespace {
+
+struct DevBuf {
+  void* p = nullptr;
+  size_t cap = 0;
+  cudaError_t ensure(size_t bytes) {
+    if (bytes <= cap && p) return cudaSuccess;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    size_t b = bytes < 256 ? 256 : bytes;
+    cudaError_t e = cudaMalloc(&p, b);
+    if (e == cudaSuccess) cap = b;
+    return e;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+  }
+  template <typename T>
+  T* as() const { return reinterpret_cast<T*>(p); }
+};
+
+// Small per-call device scratch (zeroed at the start of every symbolic call).
+struct Small {
+  int counts[8];
+  int err;
+  int range[2];
+  int pad;
+  unsigned long long hist[65];
+  unsigned long long cstats[2 * NUM_CLS + 2];
+};
+
+struct HostRead {  // pinned readback area
+  Small small;
+  long long nnz;
+  int splits[1025];
+};
+
+struct SymKey {
+  int32_t Am, An, Bm, Bn;
+  int64_t Annz, Bnnz;
+  const void *Arp, *Aci, *Brp, *Bci;
+  bool operator==(const SymKey& o) const { return std::memcmp(this, &o, sizeof(SymKey)) == 0; }
+};
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int d) {
+    cudaGetDevice(&prev);
+    if (prev != d) cudaSetDevice(d);
+  }
+  ~DeviceGuard() {
+    int cur;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+const char* class_name(int c) {
+  static const char* n[] = {"empty", "single", "tiny", "light", "medium", "heavy", "huge"};
+  return (c >= 0 && c < NUM_CLS) ? n[c] : "?";
+}
+
+}  // namespace
+
+struct spg_ctx {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  spg_dtype dtype = SPG_FP64;
+  int sms = 148;
+  int rank = 0, nranks = 1;
+  ncclComm_t comm = nullptr;
+  // options
+  int light_max = 256, medium_max = MEDIUM_CAP, heavy_max = HEAVY_CAP, force = -1;
+  int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
+  // workspace
+  DevBuf f, nz, lists, small, scan_tmp, Pf, splits, huge_bm, huge_acc, canonB[3], iota, ones, crow_tmp;
+  long long huge_bm_slots = 0, huge_acc_slots = 0, huge_N = -1;
+  HostRead* hr = nullptr;
+  cudaStream_t aux[NUM_CLS] = {};
+  cudaEvent_t ev_fork = nullptr, ev_join[NUM_CLS] = {};
+  cudaEvent_t ev_t[8] = {};
+  cudaEvent_t ev_c0[NUM_CLS] = {}, ev_c1[NUM_CLS] = {};
+  bool class_timed[NUM_CLS] = {};
+  int max_bpsm[2][NUM_CLS] = {};
+  // cached symbolic state
+  bool sym_ok = false;
+  SymKey key{};
+  int32_t rb = 0, re = 0;
+  int64_t nnzC = 0;
+  int counts[NUM_CLS] = {};
+  spg_stats stats{};
+  bool num_timed = false;
+  int launches = 0;  // kernels launched by the current phase
+  // host (end-to-end) path buffers
+  DevBuf hbuf[9];
+  spg_csr hA{}, hB{};
+  bool host_sym_ok = false;
+  std::string err;
+};
+
+namespace {
+
+spg_status setf(spg_handle h, spg_status s, const char* fmt, ...) {
+  if (h) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    h->err = buf;
+  }
+  return s;
+}
+
+#define CK(call)                                                                                 \
+  do {                                                                                           \
+    cudaError_t e_ = (call);                                                                     \
+    if (e_ != cudaSuccess) {                                                                     \
+      spg_status s_ = e_ == cudaErrorMemoryAllocation ? SPG_ERR_OUT_OF_MEMORY : SPG_ERR_CUDA;    \
+      return setf(h, s_, "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    }                                                                                            \
+  } while (0)
+
+#define NK(call)                                                                                    \
+  do {                                                                                              \
+    ncclResult_t r_ = (call);                                                                       \
+    if (r_ != ncclSuccess)                                                                          \
+      return setf(h, SPG_ERR_NCCL, "%s failed: %s (%s:%d)", #call, ncclGetErrorString(r_), __FILE__, __LINE__); \
+  } while (0)
+
+spg_status check_csr(spg_handle h, const spg_csr* m, const char* name, bool need_vals) {
+  if (!m) return setf(h, SPG_ERR_INVALID_ARGUMENT, "%s is NULL", name);
+  if (m->nrows < 0 || m->ncols < 0 || m->nnz < 0)
+    return setf(h, SPG_ERR_INVALID_ARGUMENT, "%s has negative dimensions or nnz", name);
+  if (m->nnz >= ((int64_t)1 << 31)) return setf(h, SPG_ERR_INDEX_OVERFLOW, "%s.nnz >= 2^31", name);
+  if (!m->row_ptr) return setf(h, SPG_ERR_INVALID_ARGUMENT, "%s.row_ptr is NULL", name);
+  if (m->nnz > 0 && !m->col_idx) return setf(h, SPG_ERR_INVALID_ARGUMENT, "%s.col_idx is NULL", name);
+  if (need_vals && m->nnz > 0 && !m->vals) return setf(h, SPG_ERR_INVALID_ARGUMENT, "%s.vals is NULL", name);
+  return SPG_OK;
+}
+
+SymKey make_key(const spg_csr* A, const spg_csr* B) {
+  SymKey k;
+  std::memset(&k, 0, sizeof k);
+  k.Am = A->nrows; k.An = A->ncols; k.Bm = B->nrows; k.Bn = B->ncols;
+  k.Annz = A->nnz; k.Bnnz = B->nnz;
+  k.Arp = A->row_ptr; k.Aci = A->col_idx; k.Brp = B->row_ptr; k.Bci = B->col_idx;
+  return k;
+}
+
+template <typename V>
+Prob<V> make_prob(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow, int* ccol, void* cval) {
+  Prob<V> P;
+  P.rpA = A->row_ptr; P.colA = A->col_idx; P.valA = (const V*)A->vals;
+  P.rpB = B->row_ptr; P.colB = B->col_idx; P.valB = (const V*)B->vals;
+  P.row_begin = h->rb; P.crow = crow; P.ccol = ccol; P.cval = (V*)cval;
+  return P;
+}
+
+int class_rows_per_block(int c) {
+  switch (c) {
+    case CLS_SINGLE: case CLS_TINY: return 8;
+    case CLS_LIGHT: return LIGHT_WARPS;
+    default: return 1;
+  }
+}
+
+bool huge_supported(long long N) {
+  const long long nl1 = ((N + 31) / 32 + 31) / 32;
+  return nl1 * 4 <= 128 * 1024;
+}
+
+// Dense-accumulator workspace for the HUGE tier.
+template <typename V>
+spg_status ensure_huge(spg_handle h, long long N, bool numeric, int rows, HugeWs<V>& ws, int& grid) {
+  const long long nbw = (N + 31) / 32;
+  const long long nl1 = (nbw + 31) / 32;
+  if (nl1 * 4 > 128 * 1024)
+    return setf(h, SPG_ERR_NOT_SUPPORTED, "HUGE tier: N = %lld columns exceeds the 2^25 dense-accumulator limit", N);
+  long long slots = h->huge_slots_opt > 0 ? h->huge_slots_opt : h->sms;
+  if (numeric && rows < slots) slots = rows;
+  if (slots < 1) slots = 1;
+  if (h->huge_N != N) {  // geometry changed: drop old buffers
+    h->huge_bm.release();
+    h->huge_acc.release();
+    h->huge_bm_slots = h->huge_acc_slots = 0;
+    h->huge_N = N;
+  }
+  if (h->huge_bm_slots < slots) {
+    h->huge_bm.release();
+    CK(h->huge_bm.ensure((size_t)(slots * nbw * 4)));
+    CK(cudaMemsetAsync(h->huge_bm.p, 0, (size_t)(slots * nbw * 4), h->stream));
+    h->huge_bm_slots = slots;
+  }
+  if (numeric && h->huge_acc_slots < slots) {
+    h->huge_acc.release();
+    CK(h->huge_acc.ensure((size_t)(slots * N * sizeof(V))));
+    CK(cudaMemsetAsync(h->huge_acc.p, 0, (size_t)(slots * N * sizeof(V)), h->stream));
+    h->huge_acc_slots = slots;
+  }
+  ws.bm = h->huge_bm.as<unsigned>();
+  ws.acc = numeric ? h->huge_acc.as<V>() : nullptr;
+  ws.nbw = nbw;
+  ws.nl1 = (int)nl1;
+  ws.N = N;
+  grid = (int)slots;
+  return SPG_OK;
+}
+
+// Launch every class kernel of one phase.  Symbolic: counts unknown on the host, so each
+// class gets a full-occupancy persistent grid that exits immediately when its list is
+// empty.  Numeric: counts known from the symbolic readback; empty classes are skipped.
+template <typename V>
+spg_status run_classes(spg_handle h, const spg_csr* A, const spg_csr* B, bool numeric, long long* crow, int* ccol,
+                       void* cval) {
+  Prob<V> P = make_prob<V>(h, A, B, crow, ccol, cval);
+  Small* ds = h->small.as<Small>();
+  const int* cnt = ds->counts;
+  int* lists = h->lists.as<int>();
+  const long long Mloc = h->re - h->rb;
+  const bool conc = h->concurrent != 0;
+  HugeWs<V> ws{};
+  int huge_grid = 0;
+  // symbolic cannot know on the host whether HUGE rows exist; if N is beyond the dense tier
+  // the kernel is skipped and symbolic_impl reports NOT_SUPPORTED when the class is non-empty.
+  bool huge_ok = B->ncols > 0 && huge_supported(B->ncols);
+  const bool have_huge = !numeric || h->counts[CLS_HUGE] > 0;
+  if (have_huge && huge_ok) {
+    spg_status s = ensure_huge<V>(h, B->ncols, numeric, numeric ? h->counts[CLS_HUGE] : h->sms, ws, huge_grid);
+    if (s != SPG_OK) return s;
+  }
+  if (conc) CK(cudaEventRecord(h->ev_fork, h->stream));
+  const int order[] = {CLS_HUGE, CLS_HEAVY, CLS_MEDIUM, CLS_LIGHT, CLS_TINY, CLS_SINGLE};
+  for (int c : order) {
+    if (c == CLS_SINGLE && !numeric) continue;  // c_i = f_i written by classify
+    if (numeric && h->counts[c] == 0) continue;
+    if (c == CLS_HUGE && !huge_ok) continue;
+    cudaStream_t st = conc ? h->aux[c] : h->stream;
+    if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
+    const int* list = lists + (size_t)c * (size_t)(Mloc > 0 ? Mloc : 1);
+    const int rpb = class_rows_per_block(c);
+    long long maxg = (long long)h->max_bpsm[numeric][c] * h->sms;
+    long long grid = maxg;
+    if (numeric) {
+      long long need = (h->counts[c] + rpb - 1) / rpb;
+      if (need < grid) grid = need;
+    }
+    if (grid < 1) grid = 1;
+    const bool tm = numeric && h->timing;
+    if (tm) CK(cudaEventRecord(h->ev_c0[c], st));
+    cudaError_t e = cudaSuccess;
+    switch (c) {
+      case CLS_SINGLE: e = ClassLaunch<V>::single(st, (int)grid, P, list, cnt + c); break;
+      case CLS_TINY: e = ClassLaunch<V>::tiny(st, (int)grid, numeric, P, list, cnt + c); break;
+      case CLS_LIGHT: e = ClassLaunch<V>::light(st, (int)grid, numeric, P, list, cnt + c); break;
+      case CLS_MEDIUM: e = ClassLaunch<V>::medium(st, (int)grid, numeric, P, list, cnt + c); break;
+      case CLS_HEAVY: e = ClassLaunch<V>::heavy(st, (int)grid, numeric, P, list, cnt + c); break;
+      case CLS_HUGE: e = ClassLaunch<V>::huge(st, huge_grid, numeric, P, list, cnt + c, ws); break;
+    }
+    if (e != cudaSuccess)
+      return setf(h, SPG_ERR_CUDA, "%s %s kernel launch failed: %s", class_name(c), numeric ? "numeric" : "symbolic",
+                  cudaGetErrorString(e));
+    h->launches++;
+    if (tm) CK(cudaEventRecord(h->ev_c1[c], st));
+    h->class_timed[c] = tm;
+    if (conc) {
+      CK(cudaEventRecord(h->ev_join[c], st));
+      CK(cudaStreamWaitEvent(h->stream, h->ev_join[c], 0));
+    }
+  }
+  return SPG_OK;
+}
+
+spg_status ensure_ws(spg_handle h, int M) {
+  size_t m = (size_t)(M > 0 ? M : 1);
+  CK(h->f.ensure(m * sizeof(int)));
+  CK(h->nz.ensure(m));
+  CK(h->lists.ensure(m * NUM_CLS * sizeof(int)));
+  CK(h->small.ensure(sizeof(Small)));
+  CK(h->scan_tmp.ensure(scan_tmp_elems((long long)m + 1) * sizeof(long long)));
+  return SPG_OK;
+}
+
+// Row analysis over all rows (f_i, non-empty-run flag, log2 histogram).
+spg_status analysis(spg_handle h, const spg_csr* A, const spg_csr* B) {
+  Small* ds = h->small.as<Small>();
+  CK(cudaMemsetAsync(ds, 0, sizeof(Small), h->stream));
+  CK(launch_row_flops(h->stream, A->nrows, A->row_ptr, A->col_idx, B->nrows, B->row_ptr, h->f.as<int>(),
+                      h->nz.as<uint8_t>(), ds->hist, &ds->err));
+  h->launches += A->nrows > 0;
+  return SPG_OK;
+}
+
+// Flop prefix Pf (int64[M+1]) and split points s[0..P] on the device, copied to h->hr->splits.
+spg_status split_points(spg_handle h, int M, int P) {
+  if (P > 1024) return setf(h, SPG_ERR_INVALID_ARGUMENT, "at most 1024 parts");
+  CK(h->Pf.ensure(((size_t)M + 1) * sizeof(long long)));
+  CK(h->splits.ensure(((size_t)P + 1) * sizeof(int)));
+  long long* Pf = h->Pf.as<long long>();
+  CK(cudaMemsetAsync(Pf, 0, sizeof(long long), h->stream));
+  CK(launch_incl_scan<int>(h->stream, h->f.as<int>(), Pf + 1, M, h->scan_tmp.as<long long>()));
+  CK(launch_split_points(h->stream, Pf, M, P, h->splits.as<int>()));
+  h->launches += scan_launches(M) + 1;
+  CK(cudaMemcpyAsync(h->hr->splits, h->splits.p, ((size_t)P + 1) * sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaMemcpyAsync(&h->hr->nnz, Pf + M, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  return SPG_OK;
+}
+
+// SPG_OPT_VALIDATE: structural checks of both inputs on the device, before any kernel that
+// would index with them.  One extra stream sync.
+spg_status validate_device(spg_handle h, const spg_csr* A, const spg_csr* B) {
+  Small* ds = h->small.as<Small>();
+  CK(cudaMemsetAsync(&ds->err, 0, sizeof(int), h->stream));
+  CK(launch_validate(h->stream, h->sms, A->nrows, A->row_ptr, A->col_idx, A->ncols, A->nnz, 0, &ds->err));
+  CK(launch_validate(h->stream, h->sms, B->nrows, B->row_ptr, B->col_idx, B->ncols, B->nnz, 1, &ds->err));
+  int e = 0;
+  CK(cudaMemcpyAsync(&h->hr->small.err, &ds->err, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  e = h->hr->small.err;
+  if (e & 4) return setf(h, SPG_ERR_INVALID_ARGUMENT, "malformed row_ptr (not monotone, or row_ptr[0] != 0, or row_ptr[n] != nnz)");
+  if (e & 8) return setf(h, SPG_ERR_INVALID_ARGUMENT, "column index out of range");
+  if (e & 16)
+    return setf(h, SPG_ERR_INVALID_ARGUMENT,
+                "B rows are not strictly ascending (set SPG_OPT_INPUT_CANONICAL = 0 to let the library sort them)");
+  return SPG_OK;
+}
+
+template <typename V>
+spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64_t* C_row_ptr, int64_t* nnzC,
+                         int32_t* row_begin, int32_t* row_end) {
+  const int M = A->nrows;
+  spg_status s = ensure_ws(h, M);
+  if (s != SPG_OK) return s;
+  h->launches = 0;
+  if (h->validate && (s = validate_device(h, A, B)) != SPG_OK) return s;
+  h->sym_ok = false;
+  h->host_sym_ok = false;
+  if (h->timing) CK(cudaEventRecord(h->ev_t[0], h->stream));
+  if ((s = analysis(h, A, B)) != SPG_OK) return s;
+  long long F_total = -1;
+  if (h->nranks > 1) {
+    if ((s = split_points(h, M, h->nranks)) != SPG_OK) return s;
+    h->rb = h->hr->splits[h->rank];
+    h->re = h->hr->splits[h->rank + 1];
+    F_total = h->hr->nnz;
+  } else {
+    h->rb = 0;
+    h->re = M;
+  }
+  const long long Mloc = h->re - h->rb;
+  Small* ds = h->small.as<Small>();
+  ClassParams prm{h->light_max, h->medium_max, h->heavy_max, h->force, h->canonical ? 1 : 0};
+  ClassLists L;
+  int* lists = h->lists.as<int>();
+  for (int c = 0; c < NUM_CLS; ++c) L.rows[c] = lists + (size_t)c * (size_t)(Mloc > 0 ? Mloc : 1);
+  long long* crow = reinterpret_cast<long long*>(C_row_ptr);
+  CK(cudaMemsetAsync(crow, 0, sizeof(long long), h->stream));
+  CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, nullptr, prm, L,
+                     ds->counts, ds->cstats, crow));
+  h->launches += Mloc > 0;
+  if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));
+  if ((s = run_classes<V>(h, A, B, false, crow, nullptr, nullptr)) != SPG_OK) return s;
+  CK(launch_incl_scan<long long>(h->stream, crow + 1, crow + 1, Mloc, h->scan_tmp.as<long long>()));
+  h->launches += scan_launches(Mloc);
+  if (h->timing) CK(cudaEventRecord(h->ev_t[2], h->stream));
+  CK(cudaMemcpyAsync(&h->hr->small, ds, sizeof(Small), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaMemcpyAsync(&h->hr->nnz, crow + Mloc, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  const Small& hs = h->hr->small;
+  if (hs.err & 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "A has a column index outside [0, B.nrows)");
+  if (hs.counts[CLS_HUGE] > 0 && !huge_supported(B->ncols))
+    return setf(h, SPG_ERR_NOT_SUPPORTED, "HUGE tier: N = %d columns exceeds the 2^25 dense-accumulator limit",
+                B->ncols);
+  if (hs.err & 2) return setf(h, SPG_ERR_INDEX_OVERFLOW, "a row of A has >= 2^31 intermediate products");
+  h->nnzC = h->hr->nnz;
+  for (int c = 0; c < NUM_CLS; ++c) h->counts[c] = hs.counts[c];
+  spg_stats& st = h->stats;
+  std::memset(&st, 0, sizeof st);
+  st.flops = (int64_t)hs.cstats[2 * NUM_CLS + 1];
+  st.flops_total = F_total >= 0 ? F_total : st.flops;
+  st.f_max = (int64_t)hs.cstats[2 * NUM_CLS];
+  st.nnz_c = h->nnzC;
+  st.row_begin = h->rb;
+  st.row_end = h->re;
+  for (int c = 0; c < NUM_CLS; ++c) {
+    st.class_rows[c] = (int64_t)hs.cstats[c];
+    st.class_flops[c] = (int64_t)hs.cstats[NUM_CLS + c];
+  }
+  for (int b = 0; b < 65; ++b) st.bin_hist[b] = (int64_t)hs.hist[b];
+  st.launches_symbolic = h->launches;
+  if (h->timing) {
+    cudaEventElapsedTime(&st.ms_analysis, h->ev_t[0], h->ev_t[1]);
+    cudaEventElapsedTime(&st.ms_symbolic, h->ev_t[1], h->ev_t[2]);
+  }
+  h->key = make_key(A, B);
+  h->sym_ok = true;
+  h->num_timed = false;
+  if (nnzC) *nnzC = h->nnzC;
+  if (row_begin) *row_begin = h->rb;
+  if (row_end) *row_end = h->re;
+  return SPG_OK;
+}
+
+template <typename V>
+spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const int64_t* C_row_ptr, int32_t* C_col,
+                        void* C_val) {
+  if (h->timing) CK(cudaEventRecord(h->ev_t[3], h->stream));
+  h->launches = 0;
+  spg_status s = run_classes<V>(h, A, B, true, (long long*)C_row_ptr, C_col, C_val);
+  if (s != SPG_OK) return s;
+  h->stats.launches_numeric = h->launches;
+  if (h->timing) {
+    CK(cudaEventRecord(h->ev_t[4], h->stream));
+    h->num_timed = true;
+  }
+  return SPG_OK;
+}
+
+spg_status validate_pair(spg_handle h, const spg_csr* A, const spg_csr* B, bool need_vals) {
+  spg_status s;
+  if ((s = check_csr(h, A, "A", need_vals)) != SPG_OK) return s;
+  if ((s = check_csr(h, B, "B", need_vals)) != SPG_OK) return s;
+  if (A->ncols != B->nrows)
+    return setf(h, SPG_ERR_DIMENSION_MISMATCH, "A.ncols (%d) != B.nrows (%d)", A->ncols, B->nrows);
+  return SPG_OK;
+}
+
+spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dtype) {
+  if (!out) return SPG_ERR_INVALID_ARGUMENT;
+  *out = nullptr;
+  if (dtype != SPG_FP32 && dtype != SPG_FP64) return SPG_ERR_INVALID_ARGUMENT;
+  spg_ctx* h = new (std::nothrow) spg_ctx;
+  if (!h) return SPG_ERR_OUT_OF_MEMORY;
+  h->device = device;
+  h->stream = (cudaStream_t)stream;
+  h->dtype = dtype;
+  DeviceGuard g(device);
+  cudaError_t e = cudaSetDevice(device);
+  if (e != cudaSuccess) {
+    delete h;
+    return SPG_ERR_CUDA;
+  }
+  cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, device);
+  e = dtype == SPG_FP64 ? ClassLaunch<double>::configure() : ClassLaunch<float>::configure();
+  if (e == cudaSuccess) e = cudaHostAlloc((void**)&h->hr, sizeof(HostRead), cudaHostAllocDefault);
+  for (int c = 0; c < NUM_CLS && e == cudaSuccess; ++c) {
+    e = cudaStreamCreateWithFlags(&h->aux[c], cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_join[c], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreate(&h->ev_c0[c]);
+    if (e == cudaSuccess) e = cudaEventCreate(&h->ev_c1[c]);
+  }
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming);
+  for (int k = 0; k < 8 && e == cudaSuccess; ++k) e = cudaEventCreate(&h->ev_t[k]);
+  if (e != cudaSuccess) {
+    h->err = cudaGetErrorString(e);
+    spg_spgemm_free(h);
+    return SPG_ERR_CUDA;
+  }
+  for (int num = 0; num < 2; ++num)
+    for (int c = 0; c < NUM_CLS; ++c)
+      h->max_bpsm[num][c] = dtype == SPG_FP64 ? ClassLaunch<double>::max_blocks_per_sm(c, num)
+                                              : ClassLaunch<float>::max_blocks_per_sm(c, num);
+  cudaGetLastError();
+  *out = h;
+  return SPG_OK;
+}
+
+spg_status upload(spg_handle h, DevBuf& b, const void* src, size_t bytes) {
+  CK(b.ensure(bytes));
+  if (bytes) CK(cudaMemcpyAsync(b.p, src, bytes, cudaMemcpyHostToDevice, h->stream));
+  return SPG_OK;
+}
+
+}  // namespace
+
+// ===================================== ABI =====================================================
+extern "C" {
+
+const char* spg_version(void) { return "spg 0.1 (sm_100a, heavy/light-row Gustavson SpGEMM)"; }
+
+spg_status spg_create(spg_handle* h, int device, void* cuda_stream, spg_dtype dtype) {
+  return create_common(h, device, cuda_stream, dtype);
+}
+
+spg_status spg_spgemm_free(spg_handle h) {
+  if (!h) return SPG_ERR_INVALID_ARGUMENT;
+  {
+    DeviceGuard g(h->device);
+    cudaStreamSynchronize(h->stream);
+    DevBuf* bufs[] = {&h->f, &h->nz, &h->lists, &h->small, &h->scan_tmp, &h->Pf, &h->splits, &h->huge_bm,
+                      &h->huge_acc, &h->iota, &h->ones, &h->crow_tmp};
+    for (DevBuf* b : bufs) b->release();
+    for (auto& b : h->canonB) b.release();
+    for (auto& b : h->hbuf) b.release();
+    for (int c = 0; c < NUM_CLS; ++c) {
+      if (h->aux[c]) cudaStreamDestroy(h->aux[c]);
+      if (h->ev_join[c]) cudaEventDestroy(h->ev_join[c]);
+      if (h->ev_c0[c]) cudaEventDestroy(h->ev_c0[c]);
+      if (h->ev_c1[c]) cudaEventDestroy(h->ev_c1[c]);
+    }
+    if (h->ev_fork) cudaEventDestroy(h->ev_fork);
+    for (auto& e : h->ev_t)
+      if (e) cudaEventDestroy(e);
+    if (h->hr) cudaFreeHost(h->hr);
+    if (h->comm) ncclCommDestroy(h->comm);
+    cudaGetLastError();
+  }
+  delete h;
+  return SPG_OK;
+}
+
+const char* spg_last_error(spg_handle h) { return h ? h->err.c_str() : "null handle"; }
+
+spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
+  if (!h) return SPG_ERR_INVALID_ARGUMENT;
+  switch (opt) {
+    case SPG_OPT_LIGHT_MAX_FLOPS:
+      if (v < TINY_MAX || v > LIGHT_CAP) return setf(h, SPG_ERR_INVALID_ARGUMENT, "LIGHT_MAX_FLOPS must be in [32, 256]");
+      h->light_max = (int)v;
+      break;
+    case SPG_OPT_MEDIUM_MAX_FLOPS:
+      if (v < TINY_MAX || v > MEDIUM_CAP) return setf(h, SPG_ERR_INVALID_ARGUMENT, "MEDIUM_MAX_FLOPS must be in [32, 2048]");
+      h->medium_max = (int)v;
+      break;
+    case SPG_OPT_HEAVY_MAX_FLOPS:
+      if (v < TINY_MAX || v > HEAVY_CAP) return setf(h, SPG_ERR_INVALID_ARGUMENT, "HEAVY_MAX_FLOPS must be in [32, 8192]");
+      h->heavy_max = (int)v;
+      break;
+    case SPG_OPT_FORCE_CLASS:
+      if (v != -1 && (v < CLS_TINY || v > CLS_HUGE))
+        return setf(h, SPG_ERR_INVALID_ARGUMENT, "FORCE_CLASS must be -1 or a class id in [2, 6]");
+      h->force = (int)v;
+      break;
+    case SPG_OPT_VALIDATE: h->validate = v != 0; break;
+    case SPG_OPT_INPUT_CANONICAL: h->canonical = v != 0; break;
+    case SPG_OPT_TIMING: h->timing = v != 0; break;
+    case SPG_OPT_HUGE_SLOTS:
+      if (v < 0) return setf(h, SPG_ERR_INVALID_ARGUMENT, "HUGE_SLOTS must be >= 0");
+      h->huge_slots_opt = (int)v;
+      break;
+    case SPG_OPT_CONCURRENT: h->concurrent = v != 0; break;
+    default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
+  }
+  h->sym_ok = false;
+  return SPG_OK;
+}
+
+spg_status spg_get_option(spg_handle h, spg_option opt, int64_t* v) {
+  if (!h || !v) return SPG_ERR_INVALID_ARGUMENT;
+  switch (opt) {
+    case SPG_OPT_LIGHT_MAX_FLOPS: *v = h->light_max; break;
+    case SPG_OPT_MEDIUM_MAX_FLOPS: *v = h->medium_max; break;
+    case SPG_OPT_HEAVY_MAX_FLOPS: *v = h->heavy_max; break;
+    case SPG_OPT_FORCE_CLASS: *v = h->force; break;
+    case SPG_OPT_VALIDATE: *v = h->validate; break;
+    case SPG_OPT_INPUT_CANONICAL: *v = h->canonical; break;
+    case SPG_OPT_TIMING: *v = h->timing; break;
+    case SPG_OPT_HUGE_SLOTS: *v = h->huge_slots_opt; break;
+    case SPG_OPT_CONCURRENT: *v = h->concurrent; break;
+    default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
+  }
+  return SPG_OK;
+}
+
+spg_status spg_get_stats(spg_handle h, spg_stats* out) {
+  if (!h || !out) return SPG_ERR_INVALID_ARGUMENT;
+  DeviceGuard g(h->device);
+  if (h->num_timed) {
+    CK(cudaEventSynchronize(h->ev_t[4]));
+    cudaEventElapsedTime(&h->stats.ms_numeric, h->ev_t[3], h->ev_t[4]);
+    for (int c = 0; c < NUM_CLS; ++c) {
+      h->stats.ms_class_numeric[c] = 0;
+      if (h->class_timed[c]) cudaEventElapsedTime(&h->stats.ms_class_numeric[c], h->ev_c0[c], h->ev_c1[c]);
+    }
+  }
+  *out = h->stats;
+  return SPG_OK;
+}
+
+spg_status spg_spgemm_symbolic(spg_handle h, const spg_csr* A, const spg_csr* B, int64_t* C_row_ptr, int64_t* nnzC,
+                               int32_t* row_begin, int32_t* row_end) {
+  if (!h) return SPG_ERR_INVALID_ARGUMENT;
+  spg_status s = validate_pair(h, A, B, false);
+  if (s != SPG_OK) return s;
+  if (!C_row_ptr) return setf(h, SPG_ERR_INVALID_ARGUMENT, "C_row_ptr is NULL");
+  if (!h->canonical) return setf(h, SPG_ERR_NOT_SUPPORTED, "INPUT_CANONICAL = 0 is not implemented yet");
+  DeviceGuard g(h->device);
+  return h->dtype == SPG_FP64 ? symbolic_impl<double>(h, A, B, C_row_ptr, nnzC, row_begin, row_end)
+                              : symbolic_impl<float>(h, A, B, C_row_ptr, nnzC, row_begin, row_end);
+}
+
+spg_status spg_spgemm_numeric(spg_handle h, const spg_csr* A, const spg_csr* B, const int64_t* C_row_ptr,
+                              int32_t* C_col_idx, void* C_vals) {
+  if (!h) return SPG_ERR_INVALID_ARGUMENT;
+  spg_status s = validate_pair(h, A, B, true);
+  if (s != SPG_OK) return s;
+  if (!h->sym_ok) return setf(h, SPG_ERR_BAD_STATE, "spg_spgemm_numeric called before a successful symbolic");
+  if (!(make_key(A, B) == h->key))
+    return setf(h, SPG_ERR_BAD_STATE, "A/B structure differs from the last symbolic call");
+  if (!C_row_ptr || (h->nnzC > 0 && (!C_col_idx || !C_vals)))
+    return setf(h, SPG_ERR_INVALID_ARGUMENT, "C output pointer is NULL");
+  DeviceGuard g(h->device);
+  return h->dtype == SPG_FP64 ? numeric_impl<double>(h, A, B, C_row_ptr, C_col_idx, C_vals)
+                              : numeric_impl<float>(h, A, B, C_row_ptr, C_col_idx, C_vals);
+}
+
+// ---- end-to-end host path -------------------------------------------------------------------
+spg_status spg_spgemm_host_symbolic(spg_handle h, const spg_csr* A, const spg_csr* B, int64_t* C_row_ptr,
+                                    int64_t* nnzC) {
+  if (!h) return SPG_ERR_INVALID_ARGUMENT;
+  spg_status s = validate_pair(h, A, B, true);
+  if (s != SPG_OK) return s;
+  if (!C_row_ptr) return setf(h, SPG_ERR_INVALID_ARGUMENT, "C_row_ptr is NULL");
+  if (h->nranks > 1) return setf(h, SPG_ERR_NOT_SUPPORTED, "host path is single-GPU");
+  DeviceGuard g(h->device);
+  const size_t vb = h->dtype == SPG_FP64 ? 8 : 4;
+  const bool same = A->row_ptr == B->row_ptr && A->col_idx == B->col_idx && A->vals == B->vals &&
+                    A->nrows == B->nrows && A->nnz == B->nnz;
+  if ((s = upload(h, h->hbuf[0], A->row_ptr, ((size_t)A->nrows + 1) * 4)) != SPG_OK) return s;
+  if ((s = upload(h, h->hbuf[1], A->col_idx, (size_t)A->nnz * 4)) != SPG_OK) return s;
+  if ((s = upload(h, h->hbuf[2], A->vals, (size_t)A->nnz * vb)) != SPG_OK) return s;
+  h->hA = *A;
+  h->hA.row_ptr = h->hbuf[0].as<int32_t>();
+  h->hA.col_idx = h->hbuf[1].as<int32_t>();
+  h->hA.vals = h->hbuf[2].p;
+  if (same) {
+    h->hB = h->hA;
+  } else {
+    if ((s = upload(h, h->hbuf[3], B->row_ptr, ((size_t)B->nrows + 1) * 4)) != SPG_OK) return s;
+    if ((s = upload(h, h->hbuf[4], B->col_idx, (size_t)B->nnz * 4)) != SPG_OK) return s;
+    if ((s = upload(h, h->hbuf[5], B->vals, (size_t)B->nnz * vb)) != SPG_OK) return s;
+    h->hB = *B;
+    h->hB.row_ptr = h->hbuf[3].as<int32_t>();
+    h->hB.col_idx = h->hbuf[4].as<int32_t>();
+    h->hB.vals = h->hbuf[5].p;
+  }
+  CK(h->hbuf[6].ensure(((size_t)A->nrows + 1) * 8));
+  int64_t nnz = 0;
+  s = spg_spgemm_symbolic(h, &h->hA, &h->hB, h->hbuf[6].as<int64_t>(), &nnz, nullptr, nullptr);
+  if (s != SPG_OK) return s;
+  CK(cudaMemcpyAsync(C_row_ptr, h->hbuf[6].p, ((size_t)A->nrows + 1) * 8, cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  if (nnzC) *nnzC = nnz;
+  h->host_sym_ok = true;
+  return SPG_OK;
+}
+
+spg_status spg_spgemm_host_numeric(spg_handle h, int32_t* C_col_idx, void* C_vals) {
+  if (!h) return SPG_ERR_INVALID_ARGUMENT;
+  if (!h->host_sym_ok || !h->sym_ok) return setf(h, SPG_ERR_BAD_STATE, "host_numeric before host_symbolic");
+  if (h->nnzC > 0 && (!C_col_idx || !C_vals)) return setf(h, SPG_ERR_INVALID_ARGUMENT, "C output pointer is NULL");
+  DeviceGuard g(h->device);
+  const size_t vb = h->dtype == SPG_FP64 ? 8 : 4;
+  const size_t nnz = (size_t)h->nnzC;
+  CK(h->hbuf[7].ensure(nnz * 4));
+  CK(h->hbuf[8].ensure(nnz * vb));
+  spg_status s = spg_spgemm_numeric(h, &h->hA, &h->hB, h->hbuf[6].as<int64_t>(), h->hbuf[7].as<int32_t>(),
+                                    h->hbuf[8].p);
+  if (s != SPG_OK) return s;
+  if (nnz) {
+    CK(cudaMemcpyAsync(C_col_idx, h->hbuf[7].p, nnz * 4, cudaMemcpyDeviceToHost, h->stream));
+    CK(cudaMemcpyAsync(C_vals, h->hbuf[8].p, nnz * vb, cudaMemcpyDeviceToHost, h->stream));
+  }
+  CK(cudaStreamSynchronize(h->stream));
+  return SPG_OK;
+}
+
+// ---- split points / multi-GPU -------------------------------------------------------------
+spg_status spg_split_points(spg_handle h, const spg_csr* A, const spg_csr* B, int32_t P, int32_t* s_out) {
+  if (!h || !s_out || P < 1) return SPG_ERR_INVALID_ARGUMENT;
+  spg_status s = validate_pair(h, A, B, false);
+  if (s != SPG_OK) return s;
+  DeviceGuard g(h->device);
+  if ((s = ensure_ws(h, A->nrows)) != SPG_OK) return s;
+  if ((s = analysis(h, A, B)) != SPG_OK) return s;
+  if ((s = split_points(h, A->nrows, P)) != SPG_OK) return s;
+  std::memcpy(s_out, h->hr->splits, ((size_t)P + 1) * sizeof(int32_t));
+  h->sym_ok = false;
+  return SPG_OK;
+}
+
+spg_status spg_get_unique_id(void* id128) {
+  if (!id128) return SPG_ERR_INVALID_ARGUMENT;
+  ncclUniqueId id;
+  if (ncclGetUniqueId(&id) != ncclSuccess) return SPG_ERR_NCCL;
+  std::memcpy(id128, &id, sizeof id);
+  return SPG_OK;
+}
+
+spg_status spg_create_dist(spg_handle* out, int device, void* cuda_stream, spg_dtype dtype, const void* id128,
+                           int rank, int nranks) {
+  if (!out || !id128 || nranks < 1 || rank < 0 || rank >= nranks || nranks > 1024) return SPG_ERR_INVALID_ARGUMENT;
+  spg_status s = create_common(out, device, cuda_stream, dtype);
+  if (s != SPG_OK) return s;
+  spg_handle h = *out;
+  h->rank = rank;
+  h->nranks = nranks;
+  DeviceGuard g(device);
+  ncclUniqueId id;
+  std::memcpy(&id, id128, sizeof id);
+  ncclResult_t r = ncclCommInitRank(&h->comm, nranks, id, rank);
+  if (r != ncclSuccess) {
+    spg_spgemm_free(h);
+    *out = nullptr;
+    return SPG_ERR_NCCL;
+  }
+  return SPG_OK;
+}
+
+spg_status spg_broadcast_csr(spg_handle h, spg_csr* m, int root) {
+  if (!h || !m) return SPG_ERR_INVALID_ARGUMENT;
+  if (!h->comm) return setf(h, SPG_ERR_BAD_STATE, "handle has no communicator (use spg_create_dist)");
+  spg_status s = check_csr(h, m, "matrix", true);
+  if (s != SPG_OK) return s;
+  DeviceGuard g(h->device);
+  const ncclDataType_t vt = h->dtype == SPG_FP64 ? ncclFloat64 : ncclFloat32;
+  NK(ncclGroupStart());
+  NK(ncclBroadcast(m->row_ptr, (void*)m->row_ptr, (size_t)m->nrows + 1, ncclInt32, root, h->comm, h->stream));
+  if (m->nnz) {
+    NK(ncclBroadcast(m->col_idx, (void*)m->col_idx, (size_t)m->nnz, ncclInt32, root, h->comm, h->stream));
+    NK(ncclBroadcast(m->vals, (void*)m->vals, (size_t)m->nnz, vt, root, h->comm, h->stream));
+  }
+  NK(ncclGroupEnd());
+  return SPG_OK;
+}
+
+spg_status spg_allgather_nnz(spg_handle h, int64_t nnz_local, int64_t* nnz_total) {
+  if (!h || !nnz_total) return SPG_ERR_INVALID_ARGUMENT;
+  if (!h->comm) return setf(h, SPG_ERR_BAD_STATE, "handle has no communicator");
+  DeviceGuard g(h->device);
+  CK(h->crow_tmp.ensure(sizeof(long long) * (size_t)(h->nranks + 1)));
+  long long* d = h->crow_tmp.as<long long>();
+  long long v = nnz_local;
+  CK(cudaMemcpyAsync(d + h->nranks, &v, sizeof v, cudaMemcpyHostToDevice, h->stream));
+  NK(ncclAllGather(d + h->nranks, d, 1, ncclInt64, h->comm, h->stream));
+  std::vector<long long> all(h->nranks);
+  CK(cudaMemcpyAsync(all.data(), d, sizeof(long long) * h->nranks, cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  long long t = 0;
+  for (long long x : all) t += x;
+  *nnz_total = t;
+  return SPG_OK;
+}
+
+spg_status spg_allgatherv_c(spg_handle h, const int64_t* C_row_ptr_local, const int32_t* C_col_local,
+                            const void* C_val_local, int64_t* C_row_ptr_full, int32_t* C_col_full, void* C_val_full) {
+  if (!h) return SPG_ERR_INVALID_ARGUMENT;
+  if (!h->comm) return setf(h, SPG_ERR_BAD_STATE, "handle has no communicator");
+  if (!h->sym_ok) return setf(h, SPG_ERR_BAD_STATE, "allgatherv_c needs a preceding symbolic call");
+  if (!C_row_ptr_local || !C_row_ptr_full) return setf(h, SPG_ERR_INVALID_ARGUMENT, "C_row_ptr is NULL");
+  DeviceGuard g(h->device);
+  const int P = h->nranks;
+  // per-rank nnz
+  CK(h->crow_tmp.ensure(sizeof(long long) * (size_t)(2 * P + 2) + sizeof(int) * (size_t)(P + 1)));
+  long long* d = h->crow_tmp.as<long long>();
+  long long v = h->nnzC;
+  std::vector<long long> all(P), off(P + 1, 0);
+  CK(cudaMemcpyAsync(d + P, &v, sizeof v, cudaMemcpyHostToDevice, h->stream));
+  NK(ncclAllGather(d + P, d, 1, ncclInt64, h->comm, h->stream));
+  CK(cudaMemcpyAsync(all.data(), d, sizeof(long long) * P, cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  for (int r = 0; r < P; ++r) off[r + 1] = off[r] + all[r];
+  const int* sp = h->hr->splits;
+  const int M = sp[P];
+  const size_t vb = h->dtype == SPG_FP64 ? 8 : 4;
+  const ncclDataType_t vt = h->dtype == SPG_FP64 ? ncclFloat64 : ncclFloat32;
+  NK(ncclGroupStart());
+  for (int r = 0; r < P; ++r) {
+    const long long nr = sp[r + 1] - sp[r];
+    int64_t* rp_dst = C_row_ptr_full + sp[r];
+    if (nr > 0)
+      NK(ncclBroadcast(r == h->rank ? (const void*)C_row_ptr_local : (const void*)rp_dst, rp_dst, (size_t)nr,
+                       ncclInt64, r, h->comm, h->stream));
+    if (all[r] > 0) {
+      int32_t* cdst = C_col_full + off[r];
+      char* vdst = (char*)C_val_full + (size_t)off[r] * vb;
+      NK(ncclBroadcast(r == h->rank ? (const void*)C_col_local : (const void*)cdst, cdst, (size_t)all[r], ncclInt32, r,
+                       h->comm, h->stream));
+      NK(ncclBroadcast(r == h->rank ? C_val_local : (const void*)vdst, vdst, (size_t)all[r], vt, r, h->comm,
+                       h->stream));
+    }
+  }
+  NK(ncclGroupEnd());
+  // rebase: rows of rank r get + off[r]; row_ptr_full[M] = total
+  long long* doff = d + P + 1;  // P+1 int64 (reuses the tail of crow_tmp)
+  int* dsp = reinterpret_cast<int*>(d + 2 * P + 2);
+  CK(cudaMemcpyAsync(doff, off.data(), sizeof(long long) * (P + 1), cudaMemcpyHostToDevice, h->stream));
+  CK(cudaMemcpyAsync(dsp, sp, sizeof(int) * (P + 1), cudaMemcpyHostToDevice, h->stream));
+  CK(launch_rebase(h->stream, (long long*)C_row_ptr_full, M, P, dsp, doff));
+  CK(cudaStreamSynchronize(h->stream));
+  return SPG_OK;
+}
+
+}  // extern "C

@@ -1,0 +1,117 @@
+// common.cuh — shared device helpers for the SpGEMM kernels (sm_100a).
+#pragma once
+#include <cstdint>
+#include <climits>
+#include <cuda_runtime.h>
+
+namespace spg {
+
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int KEY_INF = INT_MAX;  // sentinel column (> any valid column: N <= INT_MAX)
+
+// Row classes — must match spg_row_class in include/spg.h.
+enum : int { CLS_EMPTY = 0, CLS_SINGLE, CLS_TINY, CLS_LIGHT, CLS_MEDIUM, CLS_HEAVY, CLS_HUGE, NUM_CLS };
+
+// Class-kernel geometry.
+constexpr int TINY_MAX = 32;          // one product per lane
+constexpr int LIGHT_CAP = 256;        // warp merge, per-warp shared memory
+constexpr int LIGHT_WARPS = 8;        // warps per block in the light kernel
+constexpr int MEDIUM_NT = 256;
+constexpr int MEDIUM_CAP = 2048;
+constexpr int HEAVY_NT = 512;
+constexpr int HEAVY_CAP = 8192;
+constexpr int HUGE_NT = 1024;
+
+// Shared-memory bytes a merge of f products (nr <= f runs) needs: values x2, keys x2, seg.
+template <typename V>
+__host__ __device__ constexpr int merge_smem_bytes(int cap) {
+  return cap * (int)(2 * sizeof(V) + 2 * sizeof(int)) + (cap + 1) * (int)sizeof(int);
+}
+
+__device__ __forceinline__ unsigned lanemask_lt() {
+  unsigned m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
+template <typename T>
+__device__ __forceinline__ T warp_incl_scan(T v) {
+  int lane = lane_id();
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    T o = __shfl_up_sync(FULL, v, d);
+    if (lane >= d) v += o;
+  }
+  return v;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+  for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(FULL, v, d);
+  return v;
+}
+
+// Group = one warp (G == 32) or the whole block (G == blockDim.x).
+template <int G>
+struct Group {
+  static_assert(G == 32 || (G % 32 == 0 && G <= 1024), "group size");
+  int rank;
+  int* scratch;  // block groups: >= G/32 + 1 ints of shared memory
+  __device__ __forceinline__ void sync() const {
+    if constexpr (G == 32) __syncwarp(); else __syncthreads();
+  }
+  // Exclusive scan of v over the group; *total = group sum.  All G threads must call.
+  __device__ __forceinline__ int excl_scan(int v, int& total) const {
+    int incl = warp_incl_scan(v);
+    if constexpr (G == 32) {
+      total = __shfl_sync(FULL, incl, 31);
+      return incl - v;
+    } else {
+      constexpr int NW = G / 32;
+      int w = rank >> 5, lane = rank & 31;
+      if (lane == 31) scratch[w] = incl;
+      __syncthreads();
+      if (w == 0) {
+        int x = lane < NW ? scratch[lane] : 0;
+        int xi = warp_incl_scan(x);
+        if (lane < NW) scratch[lane] = xi - x;
+        if (lane == NW - 1) scratch[NW] = xi;
+      }
+      __syncthreads();
+      int r = incl - v + scratch[w];
+      total = scratch[NW];
+      __syncthreads();
+      return r;
+    }
+  }
+  __device__ __forceinline__ long long sum(long long v) const {
+    v = warp_sum(v);
+    if constexpr (G == 32) {
+      return v;
+    } else {
+      constexpr int NW = G / 32;
+      __shared__ long long red[NW];
+      if ((rank & 31) == 0) red[rank >> 5] = v;
+      __syncthreads();
+      long long t = 0;
+#pragma unroll
+      for (int i = 0; i < NW; ++i) t += red[i];
+      __syncthreads();
+      return t;
+    }
+  }
+};
+
+// Largest r in [0, n) with a[r] <= x, given a non-decreasing and a[0] <= x.
+__device__ __forceinline__ int upper_idx(const int* a, int n, int x) {
+  int lo = 0, hi = n - 1;
+  while (lo < hi) {
+    int mid = (lo + hi + 1) >> 1;
+    if (a[mid] <= x) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+}  // namespace spg

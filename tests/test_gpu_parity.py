@@ -1,0 +1,257 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, element by element.
+
+Structure (row_ptr, col_idx) must be identical; values within |gpu - sum| <= rtol * sum|a*b|
+(rtol 1e-12 fp64, 1e-5 fp32 — BASELINE.json north_star) or bit-exact where the inputs make
+every partial sum exact (small integers, the Fig. 2 example)."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import workloads as W
+from tests._util import dense_to_csr, identity, permutation_matrix, read_golden
+from tests.gpu_util import compare, run_gpu, to_dev
+
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():  # collected on CPU boxes only with -m gpu
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+import paper_conf_ipps_ramamoorthybsk15_b200 as spg  # noqa: E402
+
+FORCE = [-1, 2, 3, 4, 5, 6]   # natural, TINY.. HUGE (TINY = SINGLE shortcut off)
+
+
+def test_native_library_is_loaded():
+    import paper_conf_ipps_ramamoorthybsk15_b200.binding as b
+    lib = b.load()
+    assert lib._name.endswith("libspg.so")
+    assert "sm_100a" in spg.spg_version()
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_fig2_bit_exact(dtype):
+    g = read_golden("fig2.txt")
+    A, B = dense_to_csr(g["A"], dtype), dense_to_csr(g["B"], dtype)
+    for force in FORCE:
+        got = run_gpu(A, B, force_class=force)
+        compare(A, B, got, exact_values=True)
+        np.testing.assert_array_equal(np.diff(got[0]), [2, 2, 3, 3])
+
+
+@pytest.mark.parametrize("seed", range(4))
+@pytest.mark.parametrize("shape", [(37, 29, 41), (200, 150, 300), (1, 50, 7), (64, 1, 64)])
+@pytest.mark.parametrize("force", FORCE)
+def test_random_int_exact(seed, shape, force):
+    M, K, N = shape
+    A = W.random_csr(M, K, 0.15, seed, values="int", empty_row_frac=0.1)
+    B = W.random_csr(K, N, 0.15, seed + 50, values="int", empty_row_frac=0.1)
+    compare(A, B, run_gpu(A, B, force_class=force), exact_values=True)
+
+
+@pytest.mark.parametrize("force", FORCE)
+def test_power_law_rows_span_all_classes(force):
+    """Chung-Lu rows from 1 to ~10k products: every class, several merge rounds, ragged tails."""
+    A, B = W.make("cl10k")
+    got = run_gpu(A, B, force_class=force)
+    compare(A, B, got)
+    st = got[3]
+    if force == -1:
+        for c in (1, 2, 3, 4, 5, 6):
+            assert st["class_rows"][c] > 0, (spg.CLASS_NAMES[c], st["class_rows"])
+    f = oracle.row_flops(A, B)
+    assert st["flops"] == f.sum() and st["f_max"] == f.max()
+    _, hist = oracle.bins(f)
+    np.testing.assert_array_equal(st["bin_hist"], hist)
+
+
+@pytest.mark.parametrize("heavy_max,medium_max,light_max", [(64, 48, 40), (256, 128, 64), (8192, 2048, 256),
+                                                            (33, 33, 32)])
+def test_thresholds_do_not_change_result(heavy_max, medium_max, light_max):
+    """the threshold moves work between kernels, never changes C."""
+    A, B = W.make("cl10k")
+    ref = oracle.spgemm(A, B, nthreads=8)
+    got = run_gpu(A, B, heavy_max_flops=heavy_max, medium_max_flops=medium_max, light_max_flops=light_max)
+    compare(A, B, got, ref=ref)
+
+
+def test_fp32_power_law():
+    A = W.chung_lu(20000, 20000, 2.1, 80000, 3000, 3000, 6.0, 1.1, 5, np.float32)
+    B = W.chung_lu(20000, 20000, 3.0, 160000, 1000, 1000, -1.0, 1.0, 6, np.float32)
+    for force in (-1, 6):
+        compare(A, B, run_gpu(A, B, force_class=force))
+
+
+def test_rectangular_and_empty():
+    cases = [(0, 5, 3, 0.0), (4, 0, 3, 0.0), (4, 5, 0, 0.0), (6, 6, 6, 0.0), (1, 1, 1, 1.0), (300, 2, 500, 0.4)]
+    for (M, K, N, d) in cases:
+        A = W.random_csr(M, K, d, 1, values="int")
+        B = W.random_csr(K, N, d, 2, values="int")
+        for force in (-1, 3, 6):
+            compare(A, B, run_gpu(A, B, force_class=force), exact_values=True)
+
+
+def test_noncanonical_A():
+    """A with duplicate and unsorted entries (B canonical): duplicates are summed."""
+    A = W.random_csr(300, 200, 0.05, 3, values="int", canonical=False)
+    rng = np.random.default_rng(0)
+    for i in range(A.nrows):
+        s, e = A.row_ptr[i], A.row_ptr[i + 1]
+        p = rng.permutation(e - s) + s
+        A.col_idx[s:e], A.vals[s:e] = A.col_idx[p], A.vals[p]
+    B = W.random_csr(200, 250, 0.05, 4, values="int")
+    for force in FORCE:
+        compare(A, B, run_gpu(A, B, force_class=force), exact_values=True)
+
+
+def test_identity_permutation():
+    A, _ = W.make("cl10k")
+    I = identity(A.nrows)
+    for (X, Y) in [(A, I), (I, A)]:
+        rp, col, val, _ = run_gpu(X, Y)
+        np.testing.assert_array_equal(rp, A.row_ptr)
+        np.testing.assert_array_equal(col, A.col_idx)
+        np.testing.assert_array_equal(val, A.vals)
+    perm = np.random.default_rng(1).permutation(A.nrows)
+    rp, col, val, _ = run_gpu(permutation_matrix(perm), A)
+    lens = np.diff(A.row_ptr)[perm]
+    np.testing.assert_array_equal(np.diff(rp), lens)
+
+
+def test_long_rows_huge_tier_dense():
+    """Rows of up to ~60k products over a 40k-column space: HUGE tier with dense extraction."""
+    rng = np.random.default_rng(7)
+    K, N = 400, 40000
+    B = W.random_csr(K, N, 0.004, 8)                        # ~160 per row
+    A = W.random_csr(64, K, 0.9, 9)                         # ~360 B rows per A row
+    compare(A, B, run_gpu(A, B))
+    compare(A, B, run_gpu(A, B, force_class=6, huge_slots=3))
+
+
+def test_numeric_rerun_new_values():
+    A, B = W.make("cl10k")
+    dA = to_dev(A)
+    plan = spg.SpGEMM(0, torch.float64)
+    C = plan.symbolic(dA, dA)
+    plan.numeric(dA, dA, C)
+    # same structure pointers, new values: the plan is reusable
+    dA2 = spg.DeviceCSR(dA.nrows, dA.ncols, dA.row_ptr, dA.col_idx, dA.vals * 2.0)
+    plan.numeric(dA2, dA2, C)
+    torch.cuda.synchronize()
+    A2 = W.CSR(A.nrows, A.ncols, A.row_ptr, A.col_idx, A.vals * 2.0)
+    compare(A2, A2, (C.row_ptr.cpu().numpy(), C.col_idx.cpu().numpy(), C.vals.cpu().numpy()))
+    plan.close()
+
+
+def test_host_path_matches_device_path():
+    A, B = W.make("cl10k")
+    h = spg.spg_create(0, None, torch.float64)
+    try:
+        rp = np.empty(A.nrows + 1, np.int64)
+        nnz = spg.spg_spgemm_host_symbolic(h, A, A, rp)
+        col = np.empty(nnz, np.int32)
+        val = np.empty(nnz, np.float64)
+        spg.spg_spgemm_host_numeric(h, col, val)
+    finally:
+        spg.spg_spgemm_free(h)
+    compare(A, B, (rp, col, val))
+
+
+def test_split_points_exact():
+    A, B = W.make("cl10k")
+    f = oracle.row_flops(A, B)
+    h = spg.spg_create(0, None, torch.float64)
+    try:
+        dA = to_dev(A)
+        for P in (1, 2, 3, 4, 8, 13):
+            s = spg.spg_split_points(h, dA, dA, P)
+            np.testing.assert_array_equal(s, oracle.split_points(f, P))
+    finally:
+        spg.spg_spgemm_free(h)
+
+
+def test_error_paths():
+    A = W.random_csr(10, 8, 0.3, 1)
+    B = W.random_csr(9, 8, 0.3, 2)
+    dA, dB = to_dev(A), to_dev(B)
+    plan = spg.SpGEMM(0, torch.float64)
+    with pytest.raises(spg.SpgError, match="DIMENSION_MISMATCH"):
+        plan.symbolic(dA, dB)
+    B2 = W.random_csr(8, 8, 0.3, 2)
+    dB2 = to_dev(B2)
+    C = spg.DeviceCSR64(10, 8, torch.zeros(11, dtype=torch.int64, device="cuda"),
+                        torch.empty(0, dtype=torch.int32, device="cuda"),
+                        torch.empty(0, dtype=torch.float64, device="cuda"))
+    with pytest.raises(spg.SpgError, match="BAD_STATE"):
+        plan.numeric(dA, dB2, C)
+    with pytest.raises(spg.SpgError, match="INVALID_ARGUMENT"):
+        plan.set_option("force_class", 1)
+    with pytest.raises(spg.SpgError, match="INVALID_ARGUMENT"):
+        plan.set_option("light_max_flops", 1000)
+    # validation: unsorted B rows and out-of-range columns are reported, not executed
+    plan.set_option("validate", 1)
+    Bu = W.random_csr(8, 8, 0.5, 3)
+    r = int(np.argmax(np.diff(Bu.row_ptr) >= 2))
+    s0 = Bu.row_ptr[r]
+    Bu.col_idx[s0], Bu.col_idx[s0 + 1] = Bu.col_idx[s0 + 1], Bu.col_idx[s0]
+    with pytest.raises(spg.SpgError, match="strictly ascending"):
+        plan.symbolic(dA, to_dev(Bu))
+    bad = W.random_csr(8, 8, 0.3, 4)
+    bad.col_idx[0] = 99
+    with pytest.raises(spg.SpgError, match="out of range"):
+        plan.symbolic(dA, to_dev(bad))
+    plan.close()
+
+
+def test_concurrent_and_serial_agree():
+    A, B = W.make("cl10k")
+    ref = oracle.spgemm(A, B, nthreads=8)
+    compare(A, B, run_gpu(A, B, concurrent=0), ref=ref)
+    compare(A, B, run_gpu(A, B, concurrent=1, timing=1), ref=ref)
+
+
+# ---- BASELINE.json configs at full size --------------------------------------------------
+@pytest.mark.parametrize("name", ["webbase1m", "webgoogle", "citpatents", "ab2m"])
+def test_config_full_parity(name):
+    A, B = W.make(name)
+    got = run_gpu(A, B)
+    compare(A, B, got, nthreads=max(1, __import__("os").cpu_count() or 1))
+    st = got[3]
+    assert st["flops"] == int(oracle.row_flops(A, B).sum())
+
+
+@pytest.mark.slow
+def test_rmat23_sampled_and_row_sums():
+    """R-MAT scale 23 (nnz(C) ~ 5.3e9): sampled rows against the oracle + the row-sum
+    invariant C.1 = A.(B.1) on every row (computed on the device, fp64)."""
+    A, _ = W.make("rmat23")
+    dA = to_dev(A)
+    plan = spg.SpGEMM(0, torch.float64)
+    C = plan(dA, dA)
+    torch.cuda.synchronize()
+    f = oracle.row_flops(A, A)
+    rng = np.random.default_rng(0)
+    rows = np.unique(np.concatenate([rng.integers(0, A.nrows, 300), np.argsort(f)[-100:]]))
+    rp = C.row_ptr.cpu().numpy()
+    for r in rows:
+        orp, ocol, oval, oabs = oracle.spgemm(A, A, int(r), int(r) + 1)
+        s, e = int(rp[r]), int(rp[r + 1])
+        assert e - s == orp[-1]
+        np.testing.assert_array_equal(C.col_idx[s:e].cpu().numpy(), ocol)
+        v = C.vals[s:e].cpu().numpy()
+        assert np.all(np.abs(v - oval) <= 1e-12 * oabs)
+    # row sums on the device in chunks of rows
+    x = torch.ones(A.ncols, dtype=torch.float64, device="cuda")
+    Bx = torch.sparse_csr_tensor(dA.row_ptr.long(), dA.col_idx.long(), dA.vals, (A.nrows, A.ncols)) @ x
+    ref = torch.sparse_csr_tensor(dA.row_ptr.long(), dA.col_idx.long(), dA.vals, (A.nrows, A.ncols)) @ Bx
+    got = torch.empty(A.nrows, dtype=torch.float64, device="cuda")
+    step = 1 << 18
+    for r0 in range(0, A.nrows, step):
+        r1 = min(A.nrows, r0 + step)
+        s, e = int(rp[r0]), int(rp[r1])
+        off = C.row_ptr[r0:r1 + 1] - s
+        got[r0:r1] = torch.segment_reduce(C.vals[s:e], "sum", offsets=off, axis=0)
+    torch.testing.assert_close(got, ref, rtol=1e-12, atol=0)
+    plan.close()

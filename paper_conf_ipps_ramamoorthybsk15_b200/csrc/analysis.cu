@@ -98,7 +98,7 @@ __global__ void __launch_bounds__(256) k_classify(const int* __restrict__ f, con
       fmax = max(fmax, (unsigned long long)fi);
       ftot += fi;
     }
-    const bool listed = act && cls >= CLS_TINY;
+    const bool listed = act && cls >= CLS_SINGLE;
     const unsigned grp = __match_any_sync(FULL, listed ? cls : -1);
     const int leader = __ffs(grp) - 1;
     int pos = 0;

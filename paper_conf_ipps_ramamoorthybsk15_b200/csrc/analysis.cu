@@ -1,126 +1,188 @@
 // analysis.cu — Phase I of the method: per-row intermediate-product
 // counts, classification of rows into light/heavy classes (the paper's Boolean H/L array,
-// generalised to a few classes), log2 flop histogram, and the scans/split points the
-// symbolic phase and the multi-GPU partitioner need.
+// generalised to a few classes and bins), the log2 flop histogram, and the scans / split
+// points the symbolic phase and the multi-GPU partitioner need.
+//
+// No 64-bit shared-memory atomics anywhere: on sm_100a they compile to ATOMS.CAST.SPIN.64
+// CAS loops that serialise under contention (hub rows, 7-way class counters).  Sums are
+// pre-reduced per warp with MATCH.ANY + REDUX (split in 16-bit halves so they cannot wrap)
+// and accumulated with native 32-bit ATOMS.
 #include "kernels.cuh"
 
 namespace spg {
 
-// f_i = sum over stored A(i,k) of len_B(k); nz_i = #entries with len_B(k) > 0 (capped at 2).
-// One block owns ROWS consecutive rows; its threads stride over the rows' A entries
-// (coalesced colA loads), find the owning row by binary search in the cached row_ptr
-// tile, and accumulate with shared-memory atomics.  Hub rows (thousands of entries) are
-// thereby spread over the whole block instead of one thread.
+// f_i = sum over stored A(i,k) of len_B(k); nz_i = #entries with len_B(k) > 0 (capped at 2);
+// sp_i = index of one entry with len_B > 0 (the only one when nz_i = 1).  One block owns ROWS
+// consecutive rows; its threads stride over the rows' A entries (coalesced), find the owning
+// row by binary search in the cached row_ptr tile, pre-reduce per warp and row, and add into
+// shared 32-bit accumulators.
 template <int ROWS>
 __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict__ rpA, const int* __restrict__ colA,
                                                     int K, const int* __restrict__ rpB, int* __restrict__ f_out,
-                                                    uint8_t* __restrict__ nz_out, unsigned long long* __restrict__ hist,
-                                                    int* __restrict__ err) {
+                                                    uint8_t* __restrict__ nz_out, int* __restrict__ sp_out,
+                                                    unsigned long long* __restrict__ hist, int* __restrict__ err,
+                                                    int* __restrict__ amax) {
   __shared__ int s_rp[ROWS + 1];
-  __shared__ unsigned long long s_f[ROWS];
+  __shared__ unsigned s_f[ROWS];
   __shared__ int s_nz[ROWS];
+  __shared__ int s_sp[ROWS];
   __shared__ unsigned s_hist[65];
-  const int t = threadIdx.x;
+  __shared__ int s_amax;
+  const int t = threadIdx.x, lane = t & 31;
   const int r0 = blockIdx.x * ROWS;
   const int nr = min(ROWS, M - r0);
   if (t <= nr) s_rp[t] = rpA[r0 + t];
   if (t == 0 && nr == ROWS) s_rp[ROWS] = rpA[r0 + ROWS];
   s_f[t] = 0;
   s_nz[t] = 0;
+  s_sp[t] = -1;
   if (t < 65) s_hist[t] = 0;
+  if (t == 0) s_amax = 0;
   __syncthreads();
   const int e0 = s_rp[0], e1 = s_rp[nr];
   int bad = 0;
-  for (int e = e0 + t; e < e1; e += ROWS) {
-    int k = colA[e];
-    if ((unsigned)k >= (unsigned)K) { bad = 1; continue; }
-    int L = rpB[k + 1] - rpB[k];
-    int r = upper_idx(s_rp, nr, e);
-    atomicAdd(&s_f[r], (unsigned long long)L);
-    if (L > 0) atomicAdd(&s_nz[r], 1);
+  for (int base = e0; base < e1; base += ROWS) {  // uniform trip count: warp collectives below
+    const int e = base + t;
+    bool act = e < e1;
+    int L = 0, r = -1;
+    if (act) {
+      const int k = colA[e];
+      if ((unsigned)k >= (unsigned)K) {
+        bad |= 1;
+      } else {
+        L = rpB[k + 1] - rpB[k];
+        r = upper_idx(s_rp, nr, e);
+      }
+    }
+    act = r >= 0;
+    const unsigned nzb = __ballot_sync(FULL, act && L > 0);
+    const unsigned grp = __match_any_sync(FULL, r);
+    if (act) {
+      const unsigned lo = __reduce_add_sync(grp, (unsigned)L & 0xffffu);
+      const unsigned hi = __reduce_add_sync(grp, (unsigned)L >> 16);
+      if (lane == __ffs(grp) - 1) {
+        const unsigned long long tot = ((unsigned long long)hi << 16) + lo;
+        if (tot > (unsigned long long)INT_MAX) {
+          bad |= 2;
+        } else {
+          const unsigned old = atomicAdd(&s_f[r], (unsigned)tot);
+          if ((unsigned long long)old + tot > (unsigned long long)INT_MAX) bad |= 2;
+        }
+        atomicAdd(&s_nz[r], __popc(grp & nzb));
+      }
+      if (L > 0) s_sp[r] = e;
+    }
   }
   __syncthreads();
   if (t < nr) {
-    unsigned long long f = s_f[t];
-    if (f > (unsigned long long)INT_MAX) { bad |= 2; f = INT_MAX; }
+    unsigned f = s_f[t];
+    if (f > (unsigned)INT_MAX) f = INT_MAX;
     f_out[r0 + t] = (int)f;
     nz_out[r0 + t] = (uint8_t)min(s_nz[t], 2);
-    int b = f == 0 ? 0 : 1 + (f == 1 ? 0 : 32 - __clz((int)f - 1));
+    sp_out[r0 + t] = s_sp[t];
+    const int b = f == 0 ? 0 : 1 + (f == 1 ? 0 : 32 - __clz((int)f - 1));
     atomicAdd(&s_hist[b], 1u);
+    atomicMax(&s_amax, s_rp[t + 1] - s_rp[t]);
   }
   if (bad) atomicOr(err, bad);
   __syncthreads();
   if (t < 65 && s_hist[t]) atomicAdd(&hist[t], (unsigned long long)s_hist[t]);
+  if (t == 0) atomicMax(amax, s_amax);
 }
 
-__device__ __forceinline__ int classify(int f, int nz, const ClassParams& p) {
-  if (f == 0) return CLS_EMPTY;
-  if (p.force < 0 && nz == 1 && p.single_ok) return CLS_SINGLE;
-  int c;
-  if (f <= TINY_MAX) c = CLS_TINY;
-  else if (f <= p.light_max) c = CLS_LIGHT;
-  else if (f <= p.medium_max) c = CLS_MEDIUM;
-  else if (f <= p.heavy_max) c = CLS_HEAVY;
-  else c = CLS_HUGE;
-  if (p.force > c) c = p.force;
-  return c;
+__device__ __forceinline__ int classify_bin(int f, int nz, const ClassParams& p) {
+  if (f == 0) return -1;
+  if (p.force < 0 && nz == 1 && p.single_ok) return BIN_SINGLE;
+  int b;
+  if (f <= 4) b = BIN_T4;
+  else if (f <= 8) b = BIN_T8;
+  else if (f <= 16) b = BIN_T16;
+  else if (f <= TINY_MAX) b = BIN_T32;
+  else if (f <= p.light_max) b = BIN_LIGHT;
+  else if (f <= p.medium_max) b = f <= MED1_CAP ? BIN_MED1 : BIN_MED2;
+  else if (f <= p.heavy_max) b = BIN_HEAVY;
+  else b = BIN_HUGE;
+  if (p.force > CLS_TINY) {  // forced class: smallest bin of that class at least
+    const int fb = class_first_bin(p.force);
+    if (fb > b) b = fb;
+  }
+  return b;
 }
 
-// Classify this rank's rows [rb, re): append each row to its class list (warp-aggregated
-// atomics), write c_i for rows whose nnz(C) is known without work (EMPTY: 0; SINGLE: f_i,
-// B canonical), and accumulate per-class row/flop statistics.
-__global__ void __launch_bounds__(256) k_classify(const int* __restrict__ f, const uint8_t* __restrict__ nz,
-                                                  int rb_h, int re_h, const int* __restrict__ range_d,
-                                                  ClassParams prm, ClassLists lists, int* __restrict__ counts,
-                                                  unsigned long long* __restrict__ cstats /* [2*NUM_CLS + 2] */,
-                                                  long long* __restrict__ crow) {
-  const int rb = range_d ? range_d[0] : rb_h;
-  const int re = range_d ? range_d[1] : re_h;
-  const int lane = lane_id();
-  __shared__ unsigned long long s_rows[NUM_CLS], s_flops[NUM_CLS], s_fmax, s_ftot;
-  if (threadIdx.x < NUM_CLS) { s_rows[threadIdx.x] = 0; s_flops[threadIdx.x] = 0; }
-  if (threadIdx.x == 0) { s_fmax = 0; s_ftot = 0; }
+// Classify this rank's rows [rb, re): append every row with work to its bin list, write c_i for
+// rows whose nnz(C) needs no work (EMPTY: 0; SINGLE: f_i, B canonical), accumulate per-class
+// statistics.  List positions come from shared counters (warp-aggregated) and ONE global
+// atomic per bin per 2048-row tile; statistics are flushed per tile.
+constexpr int CL_NT = 256, CL_IPT = 8, CL_TILE = CL_NT * CL_IPT;
+
+__global__ void __launch_bounds__(CL_NT) k_classify(const int* __restrict__ f, const uint8_t* __restrict__ nz,
+                                                    int rb, int re, ClassParams prm, BinLists lists,
+                                                    int* __restrict__ counts,
+                                                    unsigned long long* __restrict__ cstats /* [2*NUM_CLS+2] */,
+                                                    long long* __restrict__ crow) {
+  __shared__ int s_cnt[NUM_BINS], s_base[NUM_BINS];
+  __shared__ unsigned s_rows[NUM_CLS], s_flo[NUM_CLS], s_fhi[NUM_CLS], s_fmax;
+  const int tid = threadIdx.x, lane = tid & 31;
+  if (tid < NUM_BINS) s_cnt[tid] = 0;
+  if (tid < NUM_CLS) { s_rows[tid] = 0; s_flo[tid] = 0; s_fhi[tid] = 0; }
+  if (tid == 0) s_fmax = 0;
   __syncthreads();
-  unsigned long long fmax = 0, ftot = 0;
-  // every warp runs the same number of iterations so the warp collectives are uniform
   const long long n = (long long)re - rb;
-  const long long stride = (long long)gridDim.x * blockDim.x;
-  for (long long base = (long long)blockIdx.x * blockDim.x; base < n; base += stride) {
-    const long long li = base + threadIdx.x;
-    const bool act = li < n;
-    int cls = -1, fi = 0;
-    if (act) {
-      const int i = rb + (int)li;
-      fi = f[i];
-      cls = classify(fi, nz[i], prm);
-      if (cls == CLS_EMPTY) crow[li + 1] = 0;
-      else if (cls == CLS_SINGLE) crow[li + 1] = fi;
-      fmax = max(fmax, (unsigned long long)fi);
-      ftot += fi;
+  for (long long tile = (long long)blockIdx.x * CL_TILE; tile < n; tile += (long long)gridDim.x * CL_TILE) {
+    int mybin[CL_IPT], mypos[CL_IPT];
+#pragma unroll
+    for (int it = 0; it < CL_IPT; ++it) {
+      const long long li = tile + it * CL_NT + tid;
+      const bool act = li < n;
+      int fi = 0, bin = -1, cls = -1;
+      if (act) {
+        fi = f[rb + li];
+        bin = classify_bin(fi, nz[rb + li], prm);
+        cls = bin < 0 ? CLS_EMPTY : bin_class(bin);
+        if (bin < 0) crow[li + 1] = 0;
+        else if (bin == BIN_SINGLE) crow[li + 1] = fi;
+      }
+      const unsigned gc = __match_any_sync(FULL, cls);
+      if (act) {
+        const unsigned lo = __reduce_add_sync(gc, (unsigned)fi & 0xffffu);
+        const unsigned hi = __reduce_add_sync(gc, (unsigned)fi >> 16);
+        if (lane == __ffs(gc) - 1) {
+          atomicAdd(&s_rows[cls], (unsigned)__popc(gc));
+          atomicAdd(&s_flo[cls], lo);
+          atomicAdd(&s_fhi[cls], hi);
+        }
+      }
+      const unsigned fm = __reduce_max_sync(FULL, (unsigned)fi);
+      if (lane == 0 && fm) atomicMax(&s_fmax, fm);
+      const unsigned gb = __match_any_sync(FULL, bin);
+      int pos = 0;
+      if (bin >= 0) {
+        const int leader = __ffs(gb) - 1;
+        if (lane == leader) pos = atomicAdd(&s_cnt[bin], __popc(gb));
+        pos = __shfl_sync(gb, pos, leader) + __popc(gb & lanemask_lt());
+      }
+      mybin[it] = bin;
+      mypos[it] = pos;
     }
-    const bool listed = act && cls >= CLS_SINGLE;
-    const unsigned grp = __match_any_sync(FULL, listed ? cls : -1);
-    const int leader = __ffs(grp) - 1;
-    int pos = 0;
-    if (listed && lane == leader) pos = atomicAdd(&counts[cls], __popc(grp));
-    pos = __shfl_sync(FULL, pos, leader);
-    if (listed) lists.rows[cls][pos + __popc(grp & lanemask_lt())] = rb + (int)li;
-    if (act) {
-      atomicAdd(&s_rows[cls], 1ull);
-      atomicAdd(&s_flops[cls], (unsigned long long)fi);
+    __syncthreads();
+    if (tid < NUM_BINS) {
+      const int c = s_cnt[tid];
+      s_base[tid] = c ? atomicAdd(&counts[tid], c) : 0;
+      s_cnt[tid] = 0;
     }
+    if (tid < NUM_CLS) {
+      const unsigned long long fl = ((unsigned long long)s_fhi[tid] << 16) + s_flo[tid];
+      if (s_rows[tid]) atomicAdd(&cstats[tid], (unsigned long long)s_rows[tid]);
+      if (fl) atomicAdd(&cstats[NUM_CLS + tid], fl);
+      s_rows[tid] = 0; s_flo[tid] = 0; s_fhi[tid] = 0;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int it = 0; it < CL_IPT; ++it)
+      if (mybin[it] >= 0) lists.rows[mybin[it]][s_base[mybin[it]] + mypos[it]] = rb + (int)(tile + it * CL_NT + tid);
+    __syncthreads();
   }
-  atomicMax(&s_fmax, fmax);
-  atomicAdd(&s_ftot, ftot);
-  __syncthreads();
-  if (threadIdx.x < NUM_CLS) {
-    if (s_rows[threadIdx.x]) atomicAdd(&cstats[threadIdx.x], s_rows[threadIdx.x]);
-    if (s_flops[threadIdx.x]) atomicAdd(&cstats[NUM_CLS + threadIdx.x], s_flops[threadIdx.x]);
-  }
-  if (threadIdx.x == 0) {
-    atomicMax(&cstats[2 * NUM_CLS], s_fmax);
-    atomicAdd(&cstats[2 * NUM_CLS + 1], s_ftot);
-  }
+  if (tid == 0 && s_fmax) atomicMax(&cstats[2 * NUM_CLS], (unsigned long long)s_fmax);
 }
 
 // ---- inclusive scan to int64 (three passes: tile scan, tile-sum scan, add) -------------------
@@ -243,21 +305,21 @@ __global__ void k_rebase(long long* __restrict__ rp, int M, int P, const int* __
 
 // ---- host launchers ------------------------------------------------------------------------
 cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB,
-                             int* f, uint8_t* nz, unsigned long long* hist, int* err) {
+                             int* f, uint8_t* nz, int* sp, unsigned long long* hist, int* err, int* amax) {
   if (M <= 0) return cudaSuccess;
   constexpr int ROWS = 256;
-  k_row_flops<ROWS><<<(M + ROWS - 1) / ROWS, ROWS, 0, st>>>(M, rpA, colA, K, rpB, f, nz, hist, err);
+  k_row_flops<ROWS><<<(M + ROWS - 1) / ROWS, ROWS, 0, st>>>(M, rpA, colA, K, rpB, f, nz, sp, hist, err, amax);
   return cudaGetLastError();
 }
 
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
-                            const int* range_d, const ClassParams& prm, const ClassLists& lists, int* counts,
-                            unsigned long long* cstats, long long* crow) {
-  long long n = range_d ? (long long)re : (long long)re - rb;  // range_d: re is an upper bound on the count
+                            const ClassParams& prm, const BinLists& lists, int* counts, unsigned long long* cstats,
+                            long long* crow) {
+  const long long n = (long long)re - rb;
   if (n <= 0) return cudaSuccess;
-  long long blocks = (n + 255) / 256;
-  if (blocks > (long long)sms * 8) blocks = (long long)sms * 8;
-  k_classify<<<(int)blocks, 256, 0, st>>>(f, nz, rb, re, range_d, prm, lists, counts, cstats, crow);
+  long long blocks = (n + CL_TILE - 1) / CL_TILE;
+  if (blocks > (long long)sms * 4) blocks = (long long)sms * 4;
+  k_classify<<<(int)blocks, CL_NT, 0, st>>>(f, nz, rb, re, prm, lists, counts, cstats, crow);
   return cudaGetLastError();
 }
 

@@ -41,10 +41,10 @@ struct DevBuf {
 
 // Small per-call device scratch (zeroed at the start of every symbolic call).
 struct Small {
-  int counts[8];
+  int counts[16];  // per bin
   int err;
   int range[2];
-  int pad;
+  int amax;       // longest row of A
   unsigned long long hist[65];
   unsigned long long cstats[2 * NUM_CLS + 2];
 };
@@ -93,21 +93,20 @@ struct spg_ctx {
   int light_max = 256, medium_max = MEDIUM_CAP, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
   // workspace
-  DevBuf f, nz, lists, small, scan_tmp, Pf, splits, huge_bm, huge_acc, canonB[3], iota, ones, crow_tmp;
-  long long huge_bm_slots = 0, huge_acc_slots = 0, huge_N = -1;
+  DevBuf f, nz, sp, lists, small, scan_tmp, Pf, splits, canonB[3], iota, ones, crow_tmp;
   HostRead* hr = nullptr;
-  cudaStream_t aux[NUM_CLS] = {};
-  cudaEvent_t ev_fork = nullptr, ev_join[NUM_CLS] = {};
+  cudaStream_t aux[NUM_BINS] = {};
+  cudaEvent_t ev_fork = nullptr, ev_join[NUM_BINS] = {};
   cudaEvent_t ev_t[8] = {};
-  cudaEvent_t ev_c0[NUM_CLS] = {}, ev_c1[NUM_CLS] = {};
-  bool class_timed[NUM_CLS] = {};
-  int max_bpsm[2][NUM_CLS] = {};
+  cudaEvent_t ev_c0[NUM_BINS] = {}, ev_c1[NUM_BINS] = {};
+  bool bin_timed[NUM_BINS] = {};
+  int max_bpsm[2][NUM_BINS] = {};
   // cached symbolic state
   bool sym_ok = false;
   SymKey key{};
   int32_t rb = 0, re = 0;
   int64_t nnzC = 0;
-  int counts[NUM_CLS] = {};
+  int counts[NUM_BINS] = {};
   spg_stats stats{};
   bool num_timed = false;
   int launches = 0;  // kernels launched by the current phase
@@ -173,119 +172,56 @@ Prob<V> make_prob(spg_handle h, const spg_csr* A, const spg_csr* B, long long* c
   Prob<V> P;
   P.rpA = A->row_ptr; P.colA = A->col_idx; P.valA = (const V*)A->vals;
   P.rpB = B->row_ptr; P.colB = B->col_idx; P.valB = (const V*)B->vals;
+  P.sp = h->sp.as<int>(); P.frow = h->f.as<int>();
   P.row_begin = h->rb; P.crow = crow; P.ccol = ccol; P.cval = (V*)cval;
   return P;
 }
 
-int class_rows_per_block(int c) {
-  switch (c) {
-    case CLS_SINGLE: case CLS_TINY: return 8;
-    case CLS_LIGHT: return LIGHT_WARPS;
-    default: return 1;
-  }
-}
-
-bool huge_supported(long long N) {
-  const long long nl1 = ((N + 31) / 32 + 31) / 32;
-  return nl1 * 4 <= 128 * 1024;
-}
-
-// Dense-accumulator workspace for the HUGE tier.
+// Launch every bin's kernel for one phase.  Symbolic: bin sizes are not known on the host, so
+// each bin gets a full-occupancy persistent grid that exits at once when its list is empty.
+// Numeric: sizes known from the symbolic readback; empty bins are skipped.  Bins run on their
+// own streams (forked from / joined to the handle stream) so light and heavy rows overlap —
+// the paper's concurrent CPU and GPU legs of Phases II/III recast as
+// concurrent kernels on one GPU.
 template <typename V>
-spg_status ensure_huge(spg_handle h, long long N, bool numeric, int rows, HugeWs<V>& ws, int& grid) {
-  const long long nbw = (N + 31) / 32;
-  const long long nl1 = (nbw + 31) / 32;
-  if (nl1 * 4 > 128 * 1024)
-    return setf(h, SPG_ERR_NOT_SUPPORTED, "HUGE tier: N = %lld columns exceeds the 2^25 dense-accumulator limit", N);
-  long long slots = h->huge_slots_opt > 0 ? h->huge_slots_opt : h->sms;
-  if (numeric && rows < slots) slots = rows;
-  if (slots < 1) slots = 1;
-  if (h->huge_N != N) {  // geometry changed: drop old buffers
-    h->huge_bm.release();
-    h->huge_acc.release();
-    h->huge_bm_slots = h->huge_acc_slots = 0;
-    h->huge_N = N;
-  }
-  if (h->huge_bm_slots < slots) {
-    h->huge_bm.release();
-    CK(h->huge_bm.ensure((size_t)(slots * nbw * 4)));
-    CK(cudaMemsetAsync(h->huge_bm.p, 0, (size_t)(slots * nbw * 4), h->stream));
-    h->huge_bm_slots = slots;
-  }
-  if (numeric && h->huge_acc_slots < slots) {
-    h->huge_acc.release();
-    CK(h->huge_acc.ensure((size_t)(slots * N * sizeof(V))));
-    CK(cudaMemsetAsync(h->huge_acc.p, 0, (size_t)(slots * N * sizeof(V)), h->stream));
-    h->huge_acc_slots = slots;
-  }
-  ws.bm = h->huge_bm.as<unsigned>();
-  ws.acc = numeric ? h->huge_acc.as<V>() : nullptr;
-  ws.nbw = nbw;
-  ws.nl1 = (int)nl1;
-  ws.N = N;
-  grid = (int)slots;
-  return SPG_OK;
-}
-
-// Launch every class kernel of one phase.  Symbolic: counts unknown on the host, so each
-// class gets a full-occupancy persistent grid that exits immediately when its list is
-// empty.  Numeric: counts known from the symbolic readback; empty classes are skipped.
-template <typename V>
-spg_status run_classes(spg_handle h, const spg_csr* A, const spg_csr* B, bool numeric, long long* crow, int* ccol,
-                       void* cval) {
+spg_status run_bins(spg_handle h, const spg_csr* A, const spg_csr* B, bool numeric, long long* crow, int* ccol,
+                    void* cval) {
   Prob<V> P = make_prob<V>(h, A, B, crow, ccol, cval);
   Small* ds = h->small.as<Small>();
   const int* cnt = ds->counts;
   int* lists = h->lists.as<int>();
   const long long Mloc = h->re - h->rb;
   const bool conc = h->concurrent != 0;
-  HugeWs<V> ws{};
-  int huge_grid = 0;
-  // symbolic cannot know on the host whether HUGE rows exist; if N is beyond the dense tier
-  // the kernel is skipped and symbolic_impl reports NOT_SUPPORTED when the class is non-empty.
-  bool huge_ok = B->ncols > 0 && huge_supported(B->ncols);
-  const bool have_huge = !numeric || h->counts[CLS_HUGE] > 0;
-  if (have_huge && huge_ok) {
-    spg_status s = ensure_huge<V>(h, B->ncols, numeric, numeric ? h->counts[CLS_HUGE] : h->sms, ws, huge_grid);
-    if (s != SPG_OK) return s;
-  }
   if (conc) CK(cudaEventRecord(h->ev_fork, h->stream));
-  const int order[] = {CLS_HUGE, CLS_HEAVY, CLS_MEDIUM, CLS_LIGHT, CLS_TINY, CLS_SINGLE};
-  for (int c : order) {
-    if (c == CLS_SINGLE && !numeric) continue;  // c_i = f_i written by classify
-    if (numeric && h->counts[c] == 0) continue;
-    if (c == CLS_HUGE && !huge_ok) continue;
-    cudaStream_t st = conc ? h->aux[c] : h->stream;
+  const int order[] = {BIN_HUGE, BIN_HEAVY, BIN_MED2, BIN_MED1, BIN_LIGHT, BIN_T32, BIN_T16, BIN_T8, BIN_T4,
+                       BIN_SINGLE};
+  for (int b : order) {
+    if (b == BIN_SINGLE && !numeric) continue;  // c_i = f_i written by classify
+    if (numeric && h->counts[b] == 0) continue;
+    cudaStream_t st = conc ? h->aux[b] : h->stream;
     if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
-    const int* list = lists + (size_t)c * (size_t)(Mloc > 0 ? Mloc : 1);
-    const int rpb = class_rows_per_block(c);
-    long long maxg = (long long)h->max_bpsm[numeric][c] * h->sms;
-    long long grid = maxg;
+    const int* list = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
+    const int rpb = BinLaunch<V>::rows_per_block(b);
+    long long grid = (long long)h->max_bpsm[numeric][b] * h->sms;
+    if ((b == BIN_HEAVY || b == BIN_HUGE) && h->huge_slots_opt > 0 && h->huge_slots_opt < grid)
+      grid = h->huge_slots_opt;
     if (numeric) {
-      long long need = (h->counts[c] + rpb - 1) / rpb;
+      const long long need = (h->counts[b] + rpb - 1) / rpb;
       if (need < grid) grid = need;
     }
     if (grid < 1) grid = 1;
     const bool tm = numeric && h->timing;
-    if (tm) CK(cudaEventRecord(h->ev_c0[c], st));
-    cudaError_t e = cudaSuccess;
-    switch (c) {
-      case CLS_SINGLE: e = ClassLaunch<V>::single(st, (int)grid, P, list, cnt + c); break;
-      case CLS_TINY: e = ClassLaunch<V>::tiny(st, (int)grid, numeric, P, list, cnt + c); break;
-      case CLS_LIGHT: e = ClassLaunch<V>::light(st, (int)grid, numeric, P, list, cnt + c); break;
-      case CLS_MEDIUM: e = ClassLaunch<V>::medium(st, (int)grid, numeric, P, list, cnt + c); break;
-      case CLS_HEAVY: e = ClassLaunch<V>::heavy(st, (int)grid, numeric, P, list, cnt + c); break;
-      case CLS_HUGE: e = ClassLaunch<V>::huge(st, huge_grid, numeric, P, list, cnt + c, ws); break;
-    }
+    if (tm) CK(cudaEventRecord(h->ev_c0[b], st));
+    const cudaError_t e = BinLaunch<V>::launch(b, st, (int)grid, numeric, P, list, cnt + b, B->ncols);
     if (e != cudaSuccess)
-      return setf(h, SPG_ERR_CUDA, "%s %s kernel launch failed: %s", class_name(c), numeric ? "numeric" : "symbolic",
-                  cudaGetErrorString(e));
+      return setf(h, SPG_ERR_CUDA, "%s bin %d %s kernel launch failed: %s", class_name(bin_class(b)), b,
+                  numeric ? "numeric" : "symbolic", cudaGetErrorString(e));
     h->launches++;
-    if (tm) CK(cudaEventRecord(h->ev_c1[c], st));
-    h->class_timed[c] = tm;
+    if (tm) CK(cudaEventRecord(h->ev_c1[b], st));
+    h->bin_timed[b] = tm;
     if (conc) {
-      CK(cudaEventRecord(h->ev_join[c], st));
-      CK(cudaStreamWaitEvent(h->stream, h->ev_join[c], 0));
+      CK(cudaEventRecord(h->ev_join[b], st));
+      CK(cudaStreamWaitEvent(h->stream, h->ev_join[b], 0));
     }
   }
   return SPG_OK;
@@ -295,7 +231,8 @@ spg_status ensure_ws(spg_handle h, int M) {
   size_t m = (size_t)(M > 0 ? M : 1);
   CK(h->f.ensure(m * sizeof(int)));
   CK(h->nz.ensure(m));
-  CK(h->lists.ensure(m * NUM_CLS * sizeof(int)));
+  CK(h->sp.ensure(m * sizeof(int)));
+  CK(h->lists.ensure(m * NUM_BINS * sizeof(int)));
   CK(h->small.ensure(sizeof(Small)));
   CK(h->scan_tmp.ensure(scan_tmp_elems((long long)m + 1) * sizeof(long long)));
   return SPG_OK;
@@ -306,7 +243,7 @@ spg_status analysis(spg_handle h, const spg_csr* A, const spg_csr* B) {
   Small* ds = h->small.as<Small>();
   CK(cudaMemsetAsync(ds, 0, sizeof(Small), h->stream));
   CK(launch_row_flops(h->stream, A->nrows, A->row_ptr, A->col_idx, B->nrows, B->row_ptr, h->f.as<int>(),
-                      h->nz.as<uint8_t>(), ds->hist, &ds->err));
+                      h->nz.as<uint8_t>(), h->sp.as<int>(), ds->hist, &ds->err, &ds->amax));
   h->launches += A->nrows > 0;
   return SPG_OK;
 }
@@ -371,16 +308,16 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   const long long Mloc = h->re - h->rb;
   Small* ds = h->small.as<Small>();
   ClassParams prm{h->light_max, h->medium_max, h->heavy_max, h->force, h->canonical ? 1 : 0};
-  ClassLists L;
+  BinLists L;
   int* lists = h->lists.as<int>();
-  for (int c = 0; c < NUM_CLS; ++c) L.rows[c] = lists + (size_t)c * (size_t)(Mloc > 0 ? Mloc : 1);
+  for (int b = 0; b < NUM_BINS; ++b) L.rows[b] = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
   long long* crow = reinterpret_cast<long long*>(C_row_ptr);
   CK(cudaMemsetAsync(crow, 0, sizeof(long long), h->stream));
-  CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, nullptr, prm, L,
-                     ds->counts, ds->cstats, crow));
+  CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm, L, ds->counts,
+                     ds->cstats, crow));
   h->launches += Mloc > 0;
   if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));
-  if ((s = run_classes<V>(h, A, B, false, crow, nullptr, nullptr)) != SPG_OK) return s;
+  if ((s = run_bins<V>(h, A, B, false, crow, nullptr, nullptr)) != SPG_OK) return s;
   CK(launch_incl_scan<long long>(h->stream, crow + 1, crow + 1, Mloc, h->scan_tmp.as<long long>()));
   h->launches += scan_launches(Mloc);
   if (h->timing) CK(cudaEventRecord(h->ev_t[2], h->stream));
@@ -389,15 +326,13 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   CK(cudaStreamSynchronize(h->stream));
   const Small& hs = h->hr->small;
   if (hs.err & 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "A has a column index outside [0, B.nrows)");
-  if (hs.counts[CLS_HUGE] > 0 && !huge_supported(B->ncols))
-    return setf(h, SPG_ERR_NOT_SUPPORTED, "HUGE tier: N = %d columns exceeds the 2^25 dense-accumulator limit",
-                B->ncols);
   if (hs.err & 2) return setf(h, SPG_ERR_INDEX_OVERFLOW, "a row of A has >= 2^31 intermediate products");
   h->nnzC = h->hr->nnz;
-  for (int c = 0; c < NUM_CLS; ++c) h->counts[c] = hs.counts[c];
+  for (int b = 0; b < NUM_BINS; ++b) h->counts[b] = hs.counts[b];
   spg_stats& st = h->stats;
   std::memset(&st, 0, sizeof st);
-  st.flops = (int64_t)hs.cstats[2 * NUM_CLS + 1];
+  st.flops = 0;
+  for (int c = 0; c < NUM_CLS; ++c) st.flops += (int64_t)hs.cstats[NUM_CLS + c];
   st.flops_total = F_total >= 0 ? F_total : st.flops;
   st.f_max = (int64_t)hs.cstats[2 * NUM_CLS];
   st.nnz_c = h->nnzC;
@@ -427,7 +362,7 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
                         void* C_val) {
   if (h->timing) CK(cudaEventRecord(h->ev_t[3], h->stream));
   h->launches = 0;
-  spg_status s = run_classes<V>(h, A, B, true, (long long*)C_row_ptr, C_col, C_val);
+  spg_status s = run_bins<V>(h, A, B, true, (long long*)C_row_ptr, C_col, C_val);
   if (s != SPG_OK) return s;
   h->stats.launches_numeric = h->launches;
   if (h->timing) {
@@ -462,9 +397,9 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     return SPG_ERR_CUDA;
   }
   cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, device);
-  e = dtype == SPG_FP64 ? ClassLaunch<double>::configure() : ClassLaunch<float>::configure();
+  e = dtype == SPG_FP64 ? BinLaunch<double>::configure() : BinLaunch<float>::configure();
   if (e == cudaSuccess) e = cudaHostAlloc((void**)&h->hr, sizeof(HostRead), cudaHostAllocDefault);
-  for (int c = 0; c < NUM_CLS && e == cudaSuccess; ++c) {
+  for (int c = 0; c < NUM_BINS && e == cudaSuccess; ++c) {
     e = cudaStreamCreateWithFlags(&h->aux[c], cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_join[c], cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreate(&h->ev_c0[c]);
@@ -478,9 +413,9 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     return SPG_ERR_CUDA;
   }
   for (int num = 0; num < 2; ++num)
-    for (int c = 0; c < NUM_CLS; ++c)
-      h->max_bpsm[num][c] = dtype == SPG_FP64 ? ClassLaunch<double>::max_blocks_per_sm(c, num)
-                                              : ClassLaunch<float>::max_blocks_per_sm(c, num);
+    for (int b = 0; b < NUM_BINS; ++b)
+      h->max_bpsm[num][b] = dtype == SPG_FP64 ? BinLaunch<double>::max_blocks_per_sm(b, num)
+                                              : BinLaunch<float>::max_blocks_per_sm(b, num);
   cudaGetLastError();
   *out = h;
   return SPG_OK;
@@ -508,12 +443,12 @@ spg_status spg_spgemm_free(spg_handle h) {
   {
     DeviceGuard g(h->device);
     cudaStreamSynchronize(h->stream);
-    DevBuf* bufs[] = {&h->f, &h->nz, &h->lists, &h->small, &h->scan_tmp, &h->Pf, &h->splits, &h->huge_bm,
-                      &h->huge_acc, &h->iota, &h->ones, &h->crow_tmp};
+    DevBuf* bufs[] = {&h->f, &h->nz, &h->sp, &h->lists, &h->small, &h->scan_tmp, &h->Pf, &h->splits, &h->iota,
+                      &h->ones, &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
     for (auto& b : h->hbuf) b.release();
-    for (int c = 0; c < NUM_CLS; ++c) {
+    for (int c = 0; c < NUM_BINS; ++c) {
       if (h->aux[c]) cudaStreamDestroy(h->aux[c]);
       if (h->ev_join[c]) cudaEventDestroy(h->ev_join[c]);
       if (h->ev_c0[c]) cudaEventDestroy(h->ev_c0[c]);
@@ -589,9 +524,11 @@ spg_status spg_get_stats(spg_handle h, spg_stats* out) {
   if (h->num_timed) {
     CK(cudaEventSynchronize(h->ev_t[4]));
     cudaEventElapsedTime(&h->stats.ms_numeric, h->ev_t[3], h->ev_t[4]);
-    for (int c = 0; c < NUM_CLS; ++c) {
-      h->stats.ms_class_numeric[c] = 0;
-      if (h->class_timed[c]) cudaEventElapsedTime(&h->stats.ms_class_numeric[c], h->ev_c0[c], h->ev_c1[c]);
+    for (int c = 0; c < NUM_CLS; ++c) h->stats.ms_class_numeric[c] = 0;
+    for (int b = 0; b < NUM_BINS; ++b) {
+      float ms = 0;
+      if (h->bin_timed[b] && cudaEventElapsedTime(&ms, h->ev_c0[b], h->ev_c1[b]) == cudaSuccess)
+        h->stats.ms_class_numeric[bin_class(b)] += ms;
     }
   }
   *out = h->stats;

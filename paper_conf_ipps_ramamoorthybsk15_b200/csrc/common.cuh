@@ -12,15 +12,36 @@ constexpr int KEY_INF = INT_MAX;  // sentinel column (> any valid column: N <= I
 // Row classes — must match spg_row_class in include/spg.h.
 enum : int { CLS_EMPTY = 0, CLS_SINGLE, CLS_TINY, CLS_LIGHT, CLS_MEDIUM, CLS_HEAVY, CLS_HUGE, NUM_CLS };
 
+// Internal work lists ("bins"): a class may be split by kernel geometry (TINY by sub-warp width).
+enum : int {
+  BIN_SINGLE = 0, BIN_T4, BIN_T8, BIN_T16, BIN_T32, BIN_LIGHT, BIN_MED1, BIN_MED2, BIN_HEAVY, BIN_HUGE, NUM_BINS
+};
+__host__ __device__ constexpr int bin_class(int b) {
+  return b == BIN_SINGLE ? CLS_SINGLE
+       : b <= BIN_T32   ? CLS_TINY
+       : b == BIN_LIGHT ? CLS_LIGHT
+       : b <= BIN_MED2  ? CLS_MEDIUM
+       : b == BIN_HEAVY ? CLS_HEAVY : CLS_HUGE;
+}
+__host__ __device__ constexpr int class_first_bin(int c) {
+  return c == CLS_SINGLE ? BIN_SINGLE
+       : c == CLS_TINY   ? BIN_T4
+       : c == CLS_LIGHT  ? BIN_LIGHT
+       : c == CLS_MEDIUM ? BIN_MED1
+       : c == CLS_HEAVY  ? BIN_HEAVY : BIN_HUGE;
+}
+
 // Class-kernel geometry.
-constexpr int TINY_MAX = 32;          // one product per lane
+constexpr int TINY_MAX = 32;          // one product per lane of a 4/8/16/32-lane group
 constexpr int LIGHT_CAP = 256;        // warp merge, per-warp shared memory
 constexpr int LIGHT_WARPS = 8;        // warps per block in the light kernel
-constexpr int MEDIUM_NT = 256;
+constexpr int MEDIUM_NT = 128;
+constexpr int MED1_CAP = 1024;        // MEDIUM rows split by shared-memory footprint
 constexpr int MEDIUM_CAP = 2048;
-constexpr int HEAVY_NT = 512;
-constexpr int HEAVY_CAP = 8192;
-constexpr int HUGE_NT = 1024;
+constexpr int HEAVY_CAP = 8192;       // largest f of the shared-memory-values bitmap mode
+constexpr int BMP_NT = 1024;          // bitmap kernel block size (one block per SM)
+constexpr int MERGE_VT_MIN = 4;       // outputs per thread per merge round: clamp(f / G, 4, 16)
+constexpr int MERGE_VT_MAX = 16;
 
 // Shared-memory bytes a merge of f products (nr <= f runs) needs: values x2, keys x2, seg.
 template <typename V>
@@ -84,6 +105,22 @@ struct Group {
       total = scratch[NW];
       __syncthreads();
       return r;
+    }
+  }
+  __device__ __forceinline__ int max(int v) const {
+    v = __reduce_max_sync(FULL, v);
+    if constexpr (G == 32) {
+      return v;
+    } else {
+      constexpr int NW = G / 32;
+      __shared__ int redm[NW];
+      if ((rank & 31) == 0) redm[rank >> 5] = v;
+      __syncthreads();
+      int t = redm[0];
+#pragma unroll
+      for (int i = 1; i < NW; ++i) t = t > redm[i] ? t : redm[i];
+      __syncthreads();
+      return t;
     }
   }
   __device__ __forceinline__ long long sum(long long v) const {

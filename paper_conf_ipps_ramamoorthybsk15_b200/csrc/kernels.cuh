@@ -12,8 +12,8 @@ struct ClassParams {
   int single_ok;   // B rows canonical -> SINGLE shortcut allowed
 };
 
-struct ClassLists {
-  int* rows[NUM_CLS];
+struct BinLists {
+  int* rows[NUM_BINS];
 };
 
 // Problem view passed to the class kernels.  crow is the int64 C row-offset array of this
@@ -26,28 +26,20 @@ struct Prob {
   const int* __restrict__ rpB;
   const int* __restrict__ colB;
   const V* __restrict__ valB;
+  const int* sp;    // per row: index of one A entry whose B row is non-empty (row analysis)
+  const int* frow;  // per row: f_i (row analysis)
   int row_begin;
   long long* crow;
   int* ccol;
   V* cval;
 };
 
-// Dense-accumulator workspace of the HUGE tier (one slot per resident block).
-template <typename V>
-struct HugeWs {
-  unsigned* bm;     // [slots][nbw] touched-column bitmap words (kept zero between rows)
-  V* acc;           // [slots][N]   dense PartialOutput (kept zero between rows; numeric only)
-  long long nbw;    // bitmap words per slot = ceil(N / 32)
-  int nl1;          // level-1 summary words = ceil(nbw / 32) (in shared memory)
-  long long N;
-};
-
 // analysis.cu
 cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB, int* f,
-                             uint8_t* nz, unsigned long long* hist, int* err);
+                             uint8_t* nz, int* sp, unsigned long long* hist, int* err, int* amax);
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
-                            const int* range_d, const ClassParams& prm, const ClassLists& lists, int* counts,
-                            unsigned long long* cstats, long long* crow);
+                            const ClassParams& prm, const BinLists& lists, int* counts, unsigned long long* cstats,
+                            long long* crow);
 size_t scan_tmp_elems(long long n);
 int scan_launches(long long n);
 template <typename Tin>
@@ -57,20 +49,15 @@ cudaError_t launch_validate(cudaStream_t st, int sms, int M, const int* rp, cons
                             int check_sorted, int* err);
 cudaError_t launch_rebase(cudaStream_t st, long long* rp_full, int M, int P, const int* splits, const long long* off);
 
-// kernels.cu — one launcher per (class, phase).  `count` is the device-side class size;
-// `grid` is chosen by the caller (persistent grid-stride loops inside).
+// Class kernels: one launcher per bin and phase.  `count` is the device-side bin size; `grid`
+// is chosen by the caller (persistent grid-stride loops inside).  N = columns of B.
 template <typename V>
-struct ClassLaunch {
-  static cudaError_t tiny(cudaStream_t, int grid, bool numeric, const Prob<V>&, const int* list, const int* count);
-  static cudaError_t light(cudaStream_t, int grid, bool numeric, const Prob<V>&, const int* list, const int* count);
-  static cudaError_t medium(cudaStream_t, int grid, bool numeric, const Prob<V>&, const int* list, const int* count);
-  static cudaError_t heavy(cudaStream_t, int grid, bool numeric, const Prob<V>&, const int* list, const int* count);
-  static cudaError_t single(cudaStream_t, int grid, const Prob<V>&, const int* list, const int* count);
-  static cudaError_t huge(cudaStream_t, int grid, bool numeric, const Prob<V>&, const int* list, const int* count,
-                          const HugeWs<V>&);
+struct BinLaunch {
+  static cudaError_t launch(int bin, cudaStream_t st, int grid, bool numeric, const Prob<V>& P, const int* list,
+                            const int* count, long long N);
+  static int rows_per_block(int bin);
+  static int max_blocks_per_sm(int bin, bool numeric);
   static cudaError_t configure();  // opt-in dynamic shared memory sizes (once per device)
-  static int max_blocks_per_sm(int cls, bool numeric);
-  static size_t huge_smem(int nl1);
 };
 
 }  // namespace spg

@@ -1,0 +1,197 @@
+// merge.cuh — in-row run merge for LIGHT (warp) and MEDIUM (block) rows.
+//
+// The products of row i are the union of the B rows its A entries select ("runs"), each
+// already sorted by column (B canonical).  The row is produced by merging the runs pairwise
+// in shared memory (merge path, stable), then adding like-tuples (equal adjacent columns) and
+// writing the compacted, sorted row straight into CSR: the Phase IV merge of PAPER.md
+// L154-156 (sort by (r,c), mark, scan, one master thread adds, compact) done per row.
+//
+// Scale-free rows are skewed: one long B row (a hub) usually carries most of the products
+// (DESIGN.md §4).  The longest run is therefore moved to the end and
+// merged last, so the log2(#runs) rounds only touch the short runs' products and the hub's
+// products move once.  Each thread emits 4..16 outputs per round so the merge-path search
+// (log2 of the run length) is amortised.
+#pragma once
+#include "kernels.cuh"
+
+namespace spg {
+
+template <typename V, bool NUM>
+__host__ __device__ constexpr int msmem(int cap) {
+  return (NUM ? cap * (int)(2 * sizeof(V)) : 0) + cap * 2 * (int)sizeof(int) + (cap + 1) * (int)sizeof(int);
+}
+template <typename V, bool NUM>
+__host__ __device__ constexpr int msmem_aligned(int cap) {
+  return (msmem<V, NUM>(cap) + 15) & ~15;
+}
+
+// Merge the segment pairs of one round: segments are groups of `w` consecutive runs (run r
+// spans [seg[r], seg[r+1])), pairs (2m, 2m+1) over runs [0, nr); output elements [0, fr).
+template <int G, bool NUM, typename V>
+__device__ __forceinline__ void merge_round(const int* sk, int* dk, const V* sv, V* dv, const int* seg, int nr, int w,
+                                            int fr, int rank) {
+  const int lw2 = 31 - __clz(2 * w);
+  const int npairs = (nr + 2 * w - 1) >> lw2;
+  const int vt = min(MERGE_VT_MAX, max(MERGE_VT_MIN, (fr + G - 1) / G));
+  for (int o0 = rank * vt; o0 < fr; o0 += G * vt) {
+    int o = o0;
+    const int oend = min(o0 + vt, fr);
+    int lo = 0, hi = npairs - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (seg[mid << lw2] <= o) lo = mid; else hi = mid - 1;
+    }
+    int m = lo;
+    while (o < oend) {
+      const int ra = m << lw2, rb = min(ra + w, nr), rc = min(ra + 2 * w, nr);
+      const int a0 = seg[ra], a1 = seg[rb], a2 = seg[rc];
+      const int n = min(oend, a2) - o;
+      const int d = o - a0, La = a1 - a0, Lb = a2 - a1;
+      int x0 = max(0, d - Lb), x1 = min(d, La);
+      while (x0 < x1) {
+        const int mid = (x0 + x1) >> 1;
+        if (sk[a0 + mid] <= sk[a1 + d - 1 - mid]) x0 = mid + 1; else x1 = mid;
+      }
+      int ia = a0 + x0, ib = a1 + (d - x0);
+      int ka = ia < a1 ? sk[ia] : KEY_INF;
+      int kb = ib < a2 ? sk[ib] : KEY_INF;
+      for (int t = 0; t < n; ++t) {  // branchless: one key load per output
+        const bool ta = ka <= kb;
+        const int src = ta ? ia : ib;
+        dk[o + t] = ta ? ka : kb;
+        if (NUM) dv[o + t] = sv[src];
+        const int nx = src + 1, lim = ta ? a1 : a2;
+        const int kn = nx < lim ? sk[nx] : KEY_INF;
+        ia += ta;
+        ib += !ta;
+        ka = ta ? kn : ka;
+        kb = ta ? kb : kn;
+      }
+      o += n;
+      ++m;
+    }
+  }
+}
+
+// Shared-memory layout for capacity CAP (bytes = msmem<V,NUM>(CAP)):
+//   valX[CAP] valY[CAP] (numeric only) | keyX[CAP] keyY[CAP] | seg[CAP+1]
+template <int G, int CAP, bool NUM, typename V>
+__device__ __forceinline__ void merge_row(const Prob<V>& P, const int i, const Group<G>& g, char* smem) {
+  V* valX = reinterpret_cast<V*>(smem);
+  V* valY = valX + CAP;
+  int* keyX = reinterpret_cast<int*>(smem + (NUM ? 2 * CAP * sizeof(V) : 0));
+  int* keyY = keyX + CAP;
+  int* seg = keyY + CAP;
+  const int pa0 = P.rpA[i], pa1 = P.rpA[i + 1];
+
+  // 1. runs: compact the non-empty B rows this A row selects; seg = run offsets; track the
+  //    longest run.  (run start bs stashed in keyY, scale a in valY — free until round 1)
+  int nr = 0, f = 0, best = -1;
+  for (int p0 = pa0; p0 < pa1; p0 += G) {
+    const int p = p0 + g.rank;
+    int L = 0, bs = 0;
+    V a = V(0);
+    if (p < pa1) {
+      const int k = P.colA[p];
+      bs = P.rpB[k];
+      L = P.rpB[k + 1] - bs;
+      if (NUM) a = P.valA[p];
+    }
+    // pack (length, non-empty flag): f <= CAP <= 8192 and G <= 1024 keep the fields apart
+    int tot;
+    const int ex = g.excl_scan((L << 16) | (L > 0 ? 1 : 0), tot);
+    const int slot = nr + (ex & 0xffff);
+    if (L > 0) {
+      seg[slot] = f + (ex >> 16);
+      keyY[slot] = bs;
+      if (NUM) valY[slot] = a;
+    }
+    best = max(best, L > 0 ? (L << 13) | slot : -1);  // L <= 8192, slot < 8192
+    nr += tot & 0xffff;
+    f += tot >> 16;
+  }
+  best = g.max(best);
+  if (g.rank == 0) seg[nr] = f;
+  g.sync();
+
+  // 2. hub last: swap the longest run into the last slot (only the seg entries between the
+  //    two slots move) when that saves element moves.
+  const int Lbest = best >> 13, m = best & 8191;
+  bool hub = nr >= 3 && 4 * Lbest >= f;
+  if (hub && m != nr - 1) {
+    const int Llast = seg[nr] - seg[nr - 1];
+    const int sh = Llast - Lbest;
+    int bsm = 0, bsl = 0;
+    V am = V(0), al = V(0);
+    if (g.rank == 0) { bsm = keyY[m]; bsl = keyY[nr - 1]; if (NUM) { am = valY[m]; al = valY[nr - 1]; } }
+    g.sync();
+    for (int r = m + 1 + g.rank; r <= nr - 1; r += G) seg[r] += sh;
+    if (g.rank == 0) {
+      keyY[m] = bsl; keyY[nr - 1] = bsm;
+      if (NUM) { valY[m] = al; valY[nr - 1] = am; }
+    }
+    g.sync();
+  }
+
+  // 3. expand: product j of run r -> keyX[j] = colB, valX[j] = a_r * valB (coalesced per run)
+  for (int j = g.rank; j < f; j += G) {
+    const int r = upper_idx(seg, nr, j);
+    const int q = keyY[r] + (j - seg[r]);
+    keyX[j] = P.colB[q];
+    if (NUM) valX[j] = valY[r] * P.valB[q];
+  }
+  g.sync();
+  const int nrs = hub ? nr - 1 : nr;
+  const int fs = seg[nrs];
+  if (hub) {  // the hub's products never move during the short-run rounds: mirror them once
+    for (int j = fs + g.rank; j < f; j += G) {
+      keyY[j] = keyX[j];
+      if (NUM) valY[j] = valX[j];
+    }
+    g.sync();
+  }
+
+  // 4. pairwise rounds over the short runs (all runs when there is no hub), then the hub
+  int* sk = keyX;
+  int* dk = keyY;
+  V* sv = valX;
+  V* dv = valY;
+  for (int w = 1; w < nrs; w <<= 1) {
+    merge_round<G, NUM, V>(sk, dk, sv, dv, seg, nrs, w, fs, g.rank);
+    g.sync();
+    int* tk = sk; sk = dk; dk = tk;
+    V* tv = sv; sv = dv; dv = tv;
+  }
+  if (hub) {
+    // two segments [0, fs) and [fs, f): the round reads seg[0], seg[1], seg[2]
+    g.sync();
+    if (g.rank == 0) { seg[1] = fs; seg[2] = f; }
+    g.sync();
+    merge_round<G, NUM, V>(sk, dk, sv, dv, seg, 2, 1, f, g.rank);
+    g.sync();
+    int* tk = sk; sk = dk; dk = tk;
+    V* tv = sv; sv = dv; dv = tv;
+  }
+
+  // 5. like-tuples: head = first of each equal-column group; heads add their group and write
+  const long long rowoff = NUM ? P.crow[i - P.row_begin] : 0;
+  int base = 0;
+  for (int j0 = 0; j0 < f; j0 += G) {
+    const int j = j0 + g.rank;
+    const int kj = j < f ? sk[j] : KEY_INF;
+    const bool head = j < f && (j == 0 || sk[j - 1] != kj);
+    int tot;
+    const int pos = g.excl_scan(head ? 1 : 0, tot);
+    if (NUM && head) {
+      V s = sv[j];
+      for (int t = j + 1; t < f && sk[t] == kj; ++t) s += sv[t];
+      P.ccol[rowoff + base + pos] = kj;
+      P.cval[rowoff + base + pos] = s;
+    }
+    base += tot;
+  }
+  if (!NUM && g.rank == 0) P.crow[i - P.row_begin + 1] = base;
+  g.sync();
+}
+
+}  // namespace spg

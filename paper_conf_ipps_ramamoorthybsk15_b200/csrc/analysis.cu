@@ -78,7 +78,9 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
     unsigned f = s_f[t];
     if (f > (unsigned)INT_MAX) f = INT_MAX;
     f_out[r0 + t] = (int)f;
-    nz_out[r0 + t] = (uint8_t)min(s_nz[t], 2);
+    // bit 7: the A row has more entries than one bitmap-tier run chunk (HEAVY caches products
+    // of single-chunk rows in registers; longer rows take the HUGE path)
+    nz_out[r0 + t] = (uint8_t)(min(s_nz[t], 2) | (s_rp[t + 1] - s_rp[t] > BMP_NT ? 0x80 : 0));
     sp_out[r0 + t] = s_sp[t];
     const int b = f == 0 ? 0 : 1 + (f == 1 ? 0 : 32 - __clz((int)f - 1));
     atomicAdd(&s_hist[b], 1u);
@@ -92,6 +94,8 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
 
 __device__ __forceinline__ int classify_bin(int f, int nz, const ClassParams& p) {
   if (f == 0) return -1;
+  const bool longrow = nz & 0x80;
+  nz &= 0x7f;
   if (p.force < 0 && nz == 1 && p.single_ok) return BIN_SINGLE;
   int b;
   if (f <= 4) b = BIN_T4;
@@ -106,6 +110,7 @@ __device__ __forceinline__ int classify_bin(int f, int nz, const ClassParams& p)
     const int fb = class_first_bin(p.force);
     if (fb > b) b = fb;
   }
+  if (b == BIN_HEAVY && longrow) b = BIN_HUGE;
   return b;
 }
 

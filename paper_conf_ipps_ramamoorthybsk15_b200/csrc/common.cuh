@@ -40,8 +40,8 @@ constexpr int MED1_CAP = 1024;        // MEDIUM rows split by shared-memory foot
 constexpr int MEDIUM_CAP = 2048;
 constexpr int HEAVY_CAP = 8192;       // largest f of the shared-memory-values bitmap mode
 constexpr int BMP_NT = 1024;          // bitmap kernel block size (one block per SM)
-constexpr int MERGE_VT_MIN = 4;       // outputs per thread per merge round: clamp(f / G, 4, 16)
-constexpr int MERGE_VT_MAX = 16;
+constexpr int MERGE_VT_MIN = 4;       // outputs per thread per merge round: clamp(f / G, 4, 14) | 1
+constexpr int MERGE_VT_MAX = 14;
 
 // Shared-memory bytes a merge of f products (nr <= f runs) needs: values x2, keys x2, seg.
 template <typename V>
@@ -113,14 +113,16 @@ struct Group {
       return v;
     } else {
       constexpr int NW = G / 32;
-      __shared__ int redm[NW];
+      __shared__ int redm[NW + 1];
       if ((rank & 31) == 0) redm[rank >> 5] = v;
       __syncthreads();
-      int t = redm[0];
-#pragma unroll
-      for (int i = 1; i < NW; ++i) t = t > redm[i] ? t : redm[i];
+      if (rank < 32) {
+        int x = rank < NW ? redm[rank] : INT_MIN;
+        x = __reduce_max_sync(FULL, x);
+        if (rank == 0) redm[NW] = x;
+      }
       __syncthreads();
-      return t;
+      return redm[NW];
     }
   }
   __device__ __forceinline__ long long sum(long long v) const {
@@ -129,14 +131,16 @@ struct Group {
       return v;
     } else {
       constexpr int NW = G / 32;
-      __shared__ long long red[NW];
+      __shared__ long long red[NW + 1];
       if ((rank & 31) == 0) red[rank >> 5] = v;
       __syncthreads();
-      long long t = 0;
-#pragma unroll
-      for (int i = 0; i < NW; ++i) t += red[i];
+      if (rank < 32) {
+        long long x = rank < NW ? red[rank] : 0;
+        x = warp_sum(x);
+        if (rank == 0) red[NW] = x;
+      }
       __syncthreads();
-      return t;
+      return red[NW];
     }
   }
 };

@@ -20,14 +20,16 @@
 // power of two whose structures plus expected values fit (2^20 columns for webbase-sized N, so
 // these rows take a single tile); a tile whose distinct columns overflow the value slots falls
 // back to RED.ADD into C_val in L2 (correct, slower).
+#include <type_traits>
+
 #include "kernels.cuh"
 
 namespace spg {
 
 constexpr int BMP_RCAP = 1024;       // runs gathered per chunk (one per thread)
 constexpr int BMP_CTCAP = 2048;      // 32-product windows per chunk with a precomputed run index
-constexpr int BMP_SLOTS = 8;         // products per lane cached in registers across passes
-constexpr int MODE_SYM = 0, MODE_NUM = 1;
+constexpr int BMP_SLOTS = 8;         // products per lane cached in registers (HEAVY: f <= 8192)
+constexpr int MODE_SYM = 0, MODE_HEAVY = 1, MODE_HUGE = 2;
 
 __host__ __device__ constexpr int al16(int x) { return (x + 15) & ~15; }
 
@@ -37,20 +39,23 @@ __host__ __device__ constexpr int bmp_fixed_bytes() {
 }
 constexpr int BMP_SMEM = 226 * 1024;  // dynamic shared memory per block (1 block / SM; static on top)
 
-// Region bytes for a 2^lw column tile: bitmap, level-1 summary (one bit per bitmap word), the
-// rank prefixes (int per 1024 columns, u16 per 256 columns relative to its 1024) and — numeric —
-// first-claim flags (f bits).
-__device__ __forceinline__ int bmp_struct(int lw, int f, bool numeric, bool flags) {
+// Region bytes of a 2^lw column tile: bitmap, level-1 summary (one bit per bitmap word) and —
+// numeric — rank prefixes (int per 1024 columns, u16 per 256 columns relative to its 1024),
+// first-claim flags (f bits, HEAVY) and, HEAVY, `nv` staged (value, column) slots.
+template <int MODE, typename V>
+__device__ __forceinline__ int bmp_need(int lw, int f, int nv) {
   const int words = 1 << (lw - 5), nl1 = 1 << (lw - 10);
   int need = 4 * words + 4 * nl1;
-  if (numeric) need += 4 * nl1 + 8 * nl1 + (flags ? 4 * ((f + 31) >> 5) : 0) + 16;
+  if (MODE != MODE_SYM) need += 12 * nl1 + 16;
+  if (MODE == MODE_HEAVY) need += 4 * ((f + 31) >> 5) + ((int)sizeof(V) + 4) * nv + 16;
   return need;
 }
 
 template <int MODE, typename V>
 __global__ void __launch_bounds__(BMP_NT, 1) k_bitmap(Prob<V> P, const int* __restrict__ list,
                                                      const int* __restrict__ count, int lwmax, int N) {
-  constexpr bool NUM = MODE == MODE_NUM;
+  constexpr bool NUM = MODE != MODE_SYM;
+  constexpr bool HEAVY = MODE == MODE_HEAVY;
   extern __shared__ __align__(16) unsigned char sm[];
   int* seg = reinterpret_cast<int*>(sm);                                   // run -> product offset
   int* sbs = reinterpret_cast<int*>(sm + al16((BMP_RCAP + 1) * 4));        // run -> B row start
@@ -73,31 +78,30 @@ __global__ void __launch_bounds__(BMP_NT, 1) k_bitmap(Prob<V> P, const int* __re
     const int i = list[t];
     const int pa0 = P.rpA[i], pa1 = P.rpA[i + 1];
     const int f = P.frow[i];
-    // Column tile: the widest one whose structures fit (one tile for N <= 2^20).  Values are
-    // staged in shared memory when the tile's distinct columns fit the remaining space, else
-    // they are added into C_val in L2 (rows with tens of thousands of distinct columns).
-    const bool useflags = NUM && f <= 32 * BMP_NT * 4;
+    // Column tile.  HEAVY: the widest tile whose structures AND a (value, column) slot for every
+    // column it can hold (min(f, Wt)) fit — never overflows.  SYM / HUGE: the widest tile whose
+    // structures fit (one tile for N <= 2^20); HUGE adds values into C_val in L2.
     int lw = lwmax;
-    while (lw > 10 && bmp_struct(lw, f, NUM, useflags) > REGION) --lw;
+    while (lw > 10 && bmp_need<MODE, V>(lw, f, HEAVY ? min(f, 1 << lw) : 0) > REGION) --lw;
     const int Wt = 1 << lw, words = Wt >> 5, nl1 = 1 << (lw - 10);
     unsigned* bm = reinterpret_cast<unsigned*>(region);
     unsigned* l1 = bm + words;
     int* sbp = reinterpret_cast<int*>(l1 + nl1);                          // rank prefix / 1024 columns
     unsigned short* sbq = reinterpret_cast<unsigned short*>(sbp + (NUM ? nl1 : 0));  // .. / 256 columns
     unsigned* flags = reinterpret_cast<unsigned*>(sbq + (NUM ? 4 * nl1 : 0));
-    const int nfw = useflags ? (f + 31) >> 5 : 0;
+    const int nfw = HEAVY ? (f + 31) >> 5 : 0;
     const int voff = (4 * (words + (NUM ? 4 : 1) * nl1 + nfw) + 15) & ~15;
     V* val = reinterpret_cast<V*>(region + voff);
-    const int vcap = useflags ? (REGION - voff) / (int)sizeof(V) : 0;
+    const int nv = HEAVY ? min(f, Wt) : 0;
+    int* colbuf = reinterpret_cast<int*>(val + nv);
     const int ntiles = (int)(((long long)N + Wt - 1) >> lw);
     const int nchunks = (pa1 - pa0 + BMP_RCAP - 1) / BMP_RCAP;
     const long long rowoff = NUM ? P.crow[i - P.row_begin] : 0;
     long long cnt = 0;
     int out = 0;
     int nz = 0, Lt = 0;  // current chunk: runs, products
-    // register cache of this lane's products (B position, column, run) for single-chunk rows
-    const bool cached = NUM && pa1 - pa0 <= BMP_RCAP && f <= BMP_SLOTS * BMP_NT;
-    int cq[BMP_SLOTS], cc[BMP_SLOTS], cr[BMP_SLOTS];
+    int cc[BMP_SLOTS];   // HEAVY: this lane's products (column, a*b), cached in registers
+    V cv[BMP_SLOTS];
 
     auto gather = [&](int c) {
       const int p = pa0 + c * BMP_RCAP + tid;
@@ -133,44 +137,66 @@ __global__ void __launch_bounds__(BMP_NT, 1) k_bitmap(Prob<V> P, const int* __re
       return rb + __popc(M & upto);
     };
 
-    // Visit the products of the current chunk that fall in [lo, lo+Wt).  Each warp takes 32
-    // consecutive products (coalesced within a B row): one binary search finds the run of the
-    // first; the runs starting inside the window form a bitmask (REDUX.OR) and each lane's run is
-    // the first run + popcount of the starts at or below it.
-    auto for_products = [&](int lo, auto&& fn) {
-      if (cached) {
+    // Visit the products of the current chunk in [lo, lo+Wt): fn(j, lc, v) with j the product
+    // index, lc the tile-local column, v = a*b (when VALS).  HEAVY: from the register cache.
+    // Otherwise each warp takes 32-product windows (coalesced within a B row), BATCH windows'
+    // loads issued together.
+    constexpr int BATCH = 4;
+    auto for_products = [&](int lo, auto vals_tag, auto&& fn) {
+      constexpr bool VALS = decltype(vals_tag)::value;
+      if constexpr (HEAVY) {
 #pragma unroll
         for (int s = 0; s < BMP_SLOTS; ++s) {
           const int j = warp * 32 + s * BMP_NT + lane;
           const unsigned lc = (unsigned)(cc[s] - lo);
-          if (j < Lt && lc < (unsigned)Wt) fn(j, cq[s], lc, cr[s]);
+          if (j < Lt && lc < (unsigned)Wt) fn(j, lc, cv[s]);
         }
-        return;
-      }
-      for (int j0 = warp * 32; j0 < Lt; j0 += BMP_NT) {
-        const int r = lane_run(j0);
-        const int j = j0 + lane;
-        if (j < Lt) {
-          const int q = sbs[r] + (j - seg[r]);
-          const unsigned lc = (unsigned)(P.colB[q] - lo);
-          if (lc < (unsigned)Wt) fn(j, q, lc, r);
+      } else {
+        for (int j00 = warp * 32; j00 < Lt; j00 += BATCH * BMP_NT) {
+          int q[BATCH], col[BATCH], r[BATCH];
+          V b[BATCH];
+#pragma unroll
+          for (int u = 0; u < BATCH; ++u) {
+            const int j0 = j00 + u * BMP_NT;
+            q[u] = -1;
+            r[u] = 0;
+            if (j0 < Lt) {
+              r[u] = lane_run(j0);
+              if (j0 + lane < Lt) q[u] = sbs[r[u]] + (j0 + lane - seg[r[u]]);
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < BATCH; ++u) {
+            col[u] = q[u] >= 0 ? P.colB[q[u]] : -1;
+            if (VALS) b[u] = q[u] >= 0 ? P.valB[q[u]] : V(0);
+          }
+#pragma unroll
+          for (int u = 0; u < BATCH; ++u) {
+            const unsigned lc = (unsigned)(col[u] - lo);
+            if (q[u] >= 0 && lc < (unsigned)Wt) fn(j00 + u * BMP_NT + lane, lc, VALS ? sa[r[u]] * b[u] : V(0));
+          }
         }
       }
     };
     auto fill_cache = [&]() {
+      int q[BMP_SLOTS], r[BMP_SLOTS];
 #pragma unroll
       for (int s = 0; s < BMP_SLOTS; ++s) {
         const int j0 = warp * 32 + s * BMP_NT;
-        cq[s] = 0; cr[s] = 0; cc[s] = -1;
+        q[s] = -1;
+        r[s] = 0;
         if (j0 < Lt) {
-          const int r = lane_run(j0);
-          if (j0 + lane < Lt) {
-            cr[s] = r;
-            cq[s] = sbs[r] + (j0 + lane - seg[r]);
-            cc[s] = P.colB[cq[s]];
-          }
+          r[s] = lane_run(j0);
+          if (j0 + lane < Lt) q[s] = sbs[r[s]] + (j0 + lane - seg[r[s]]);
         }
       }
+#pragma unroll
+      for (int s = 0; s < BMP_SLOTS; ++s) {
+        cc[s] = q[s] >= 0 ? P.colB[q[s]] : -1;
+        cv[s] = q[s] >= 0 ? P.valB[q[s]] : V(0);
+      }
+#pragma unroll
+      for (int s = 0; s < BMP_SLOTS; ++s) cv[s] *= sa[r[s]];
     };
 
     // rank of a tile-local column among the tile's claimed columns: prefix of its 1024- and
@@ -196,85 +222,135 @@ __global__ void __launch_bounds__(BMP_NT, 1) k_bitmap(Prob<V> P, const int* __re
       for (int c = 0; c < nchunks; ++c) {
         if (nchunks > 1 || tile == 0) {
           gather(c);
-          if (cached) fill_cache();
+          if constexpr (HEAVY) fill_cache();
         }
-        for_products(lo, [&](int j, int q, unsigned lc, int r) {
-          const int w = lc >> 5;
-          const unsigned b = 1u << (lc & 31);
-          const unsigned old = atomicOr(&bm[w], b);
-          if (!(old & b)) {
-            if (!NUM) ++cnt;
-            else if (useflags) atomicOr(&flags[(cbase + j) >> 5], 1u << ((cbase + j) & 31));
+        if constexpr (HEAVY) {
+          // cached windows start at multiples of 32: one ballot word of first-claim flags each
+#pragma unroll
+          for (int s = 0; s < BMP_SLOTS; ++s) {
+            const int j0 = warp * 32 + s * BMP_NT;
+            const unsigned lc = (unsigned)(cc[s] - lo);
+            bool first = false;
+            if (j0 + lane < Lt && lc < (unsigned)Wt) {
+              const int w = lc >> 5;
+              const unsigned b = 1u << (lc & 31);
+              const unsigned old = atomicOr(&bm[w], b);
+              first = !(old & b);
+              if (old == 0) atomicOr(&l1[w >> 5], 1u << (w & 31));
+              ++inprod;
+            }
+            const unsigned fm = __ballot_sync(FULL, first);
+            if (lane == 0 && j0 < Lt) flags[j0 >> 5] = fm;
           }
-          if (old == 0) atomicOr(&l1[w >> 5], 1u << (w & 31));
-          ++inprod;
-        });
+        } else {
+          for_products(lo, std::false_type{}, [&](int j, unsigned lc, V) {
+            const int w = lc >> 5;
+            const unsigned b = 1u << (lc & 31);
+            const unsigned old = atomicOr(&bm[w], b);
+            if (!NUM && !(old & b)) ++cnt;
+            if (old == 0) atomicOr(&l1[w >> 5], 1u << (w & 31));
+            ++inprod;
+          });
+        }
         cbase += Lt;
         __syncthreads();
       }
-      if (NUM) {
-        // ---- build: superblock rank prefixes and the columns of C in order --------------------
+      if constexpr (NUM) {
+        // ---- build: rank prefixes per 1024- and 256-column block (HEAVY: dense and uniform;
+        //      HUGE: only touched words, and C_col written here in column order) --------------
         int pcarry = 0;
         for (int u0 = 0; u0 < nl1; u0 += BMP_NT) {
           const int u = u0 + tid;
           const unsigned x = u < nl1 ? l1[u] : 0u;
           int pc = 0;
-          for (unsigned y = x; y; y &= y - 1) pc += __popc(bm[(u << 5) + __ffs(y) - 1]);
+          unsigned short q4[4] = {0, 0, 0, 0};
+          if constexpr (HEAVY) {
+            if (x) {
+              // all 32 words of the superblock; the 16-byte reads are rotated by lane so a warp's
+              // loads spread over all banks (a straight walk would be a 32-way conflict)
+              int sub[4] = {0, 0, 0, 0};
+#pragma unroll
+              for (int k = 0; k < 8; ++k) {
+                const int m = (k + tid) & 7;
+                const uint4 a = reinterpret_cast<const uint4*>(bm)[8 * u + m];
+                const int c4 = __popc(a.x) + __popc(a.y) + __popc(a.z) + __popc(a.w);
+#pragma unroll
+                for (int h = 0; h < 4; ++h) sub[h] += (m >> 1) == h ? c4 : 0;
+              }
+              q4[0] = 0;
+              q4[1] = (unsigned short)sub[0];
+              q4[2] = (unsigned short)(sub[0] + sub[1]);
+              q4[3] = (unsigned short)(sub[0] + sub[1] + sub[2]);
+              pc = sub[0] + sub[1] + sub[2] + sub[3];
+            }
+          } else {
+            for (unsigned y = x; y; y &= y - 1) pc += __popc(bm[(u << 5) + __ffs(y) - 1]);
+          }
           int ptot;
           int pp = pcarry + g.excl_scan(pc, ptot);
-          if (x) sbp[u] = pp;  // only touched superblocks are ever queried (and cleared)
-          const int p0 = pp;
-          int qdone = 0;
-          for (unsigned y = x; y; y &= y - 1) {
-            const int wl = __ffs(y) - 1, w = (u << 5) + wl;
-            while (qdone <= (wl >> 3)) sbq[4 * u + qdone++] = (unsigned short)(pp - p0);
-            for (unsigned z = bm[w]; z; z &= z - 1) P.ccol[rowoff + out + pp++] = lo + (w << 5) + (__ffs(z) - 1);
+          if (x) {  // only touched superblocks are ever queried (and cleared)
+            sbp[u] = pp;
+            if constexpr (HEAVY) {
+              reinterpret_cast<unsigned long long*>(sbq)[u] =
+                  (unsigned long long)q4[0] | ((unsigned long long)q4[1] << 16) |
+                  ((unsigned long long)q4[2] << 32) | ((unsigned long long)q4[3] << 48);
+            } else {
+              const int p0 = pp;
+              int qdone = 0;
+              for (unsigned y = x; y; y &= y - 1) {
+                const int wl = __ffs(y) - 1, w = (u << 5) + wl;
+                while (qdone <= (wl >> 3)) sbq[4 * u + qdone++] = (unsigned short)(pp - p0);
+                for (unsigned z = bm[w]; z; z &= z - 1) P.ccol[rowoff + out + pp++] = lo + (w << 5) + (__ffs(z) - 1);
+              }
+              while (qdone < 4) sbq[4 * u + qdone++] = (unsigned short)(pp - p0);
+            }
           }
-          if (x) while (qdone < 4) sbq[4 * u + qdone++] = (unsigned short)(pp - p0);
           pcarry += ptot;
         }
         const int ctile = pcarry;
-        const bool sv = ctile <= vcap;                 // values staged in shared memory this tile
-        const int ndup = (int)g.sum(inprod) - ctile;   // block-uniform
-        if (!sv) {
+        if constexpr (!HEAVY) {
           for (int r = tid; r < ctile; r += BMP_NT) P.cval[rowoff + out + r] = V(0);
           __threadfence();
         }
         __syncthreads();
-        // ---- pass 2: first claimers store (smem) / every product adds (L2) ------------------------
+        // ---- pass 2: first claimers stage (value, column) in shared memory (HEAVY) / every
+        //      product adds into C_val in L2 (HUGE) -------------------------------------------------
         cbase = 0;
+        int ndup = 0;
         for (int c = 0; c < nchunks; ++c) {
           if (nchunks > 1) gather(c);
-          for_products(lo, [&](int j, int q, unsigned lc, int r) {
-            if (sv) {
-              if (flags[(cbase + j) >> 5] & (1u << ((cbase + j) & 31))) val[rank_of(lc)] = sa[r] * P.valB[q];
+          for_products(lo, std::true_type{}, [&](int j, unsigned lc, V v) {
+            if constexpr (HEAVY) {
+              if (flags[(cbase + j) >> 5] & (1u << ((cbase + j) & 31))) {
+                const int r = rank_of(lc);
+                val[r] = v;
+                colbuf[r] = lo + (int)lc;
+              } else {
+                ++ndup;
+              }
             } else {
-              atomicAdd(&P.cval[rowoff + out + rank_of(lc)], sa[r] * P.valB[q]);
+              atomicAdd(&P.cval[rowoff + out + rank_of(lc)], v);
             }
           });
           cbase += Lt;
           __syncthreads();
         }
-        if (sv) {
+        if constexpr (HEAVY) {
           // ---- pass 3: duplicates, after the first claimers' stores ------------------------------
-          if (ndup > 0) {
-            cbase = 0;
-            for (int c = 0; c < nchunks; ++c) {
-              if (nchunks > 1) gather(c);
-              for_products(lo, [&](int j, int q, unsigned lc, int r) {
-                if (!(flags[(cbase + j) >> 5] & (1u << ((cbase + j) & 31))))
-                  atomicAdd(&val[rank_of(lc)], sa[r] * P.valB[q]);
-              });
-              cbase += Lt;
-              __syncthreads();
-            }
+          if (__syncthreads_or(ndup)) {
+            for_products(lo, std::true_type{}, [&](int j, unsigned lc, V v) {
+              if (!(flags[j >> 5] & (1u << (j & 31)))) atomicAdd(&val[rank_of(lc)], v);
+            });
+            __syncthreads();
           }
           for (int r = tid; r < ctile; r += BMP_NT) {
+            P.ccol[rowoff + out + r] = colbuf[r];
             P.cval[rowoff + out + r] = val[r];
             val[r] = V(0);
+            colbuf[r] = 0;
           }
+          for (int x = tid; x < nfw; x += BMP_NT) flags[x] = 0;
         }
-        for (int x = tid; x < nfw; x += BMP_NT) flags[x] = 0;
         out += ctile;
       }
       // ---- restore the zero invariant: touched bitmap words, summary, prefixes -----------------
@@ -304,13 +380,15 @@ __global__ void __launch_bounds__(BMP_NT, 1) k_bitmap(Prob<V> P, const int* __re
 
 // ================================ launch glue ====================================================
 template <typename V>
-static const void* bitmap_kernel(int, bool numeric) {
-  return numeric ? (const void*)k_bitmap<MODE_NUM, V> : (const void*)k_bitmap<MODE_SYM, V>;
+static const void* bitmap_kernel(int bin, bool numeric) {
+  if (!numeric) return (const void*)k_bitmap<MODE_SYM, V>;
+  return bin == BIN_HEAVY ? (const void*)k_bitmap<MODE_HEAVY, V> : (const void*)k_bitmap<MODE_HUGE, V>;
 }
 
 template <typename V>
 cudaError_t bitmap_configure() {
-  for (const void* k : {(const void*)k_bitmap<MODE_SYM, V>, (const void*)k_bitmap<MODE_NUM, V>}) {
+  for (const void* k : {(const void*)k_bitmap<MODE_SYM, V>, (const void*)k_bitmap<MODE_HEAVY, V>,
+                        (const void*)k_bitmap<MODE_HUGE, V>}) {
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, BMP_SMEM);
     if (e != cudaSuccess) return e;
   }

@@ -32,7 +32,9 @@ __device__ __forceinline__ void merge_round(const int* sk, int* dk, const V* sv,
                                             int fr, int rank) {
   const int lw2 = 31 - __clz(2 * w);
   const int npairs = (nr + 2 * w - 1) >> lw2;
-  const int vt = min(MERGE_VT_MAX, max(MERGE_VT_MIN, (fr + G - 1) / G));
+  // odd: each thread writes vt consecutive outputs, so an even vt would put lanes on the same
+  // shared-memory banks (vt = 16 is a 16-way conflict)
+  const int vt = min(MERGE_VT_MAX, max(MERGE_VT_MIN, (fr + G - 1) / G)) | 1;
   for (int o0 = rank * vt; o0 < fr; o0 += G * vt) {
     int o = o0;
     const int oend = min(o0 + vt, fr);

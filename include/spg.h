@@ -166,6 +166,9 @@ spg_status spg_spgemm_host_numeric(spg_handle h, int32_t* C_col_idx, void* C_val
  * Rank r computes rows [s_r, s_{r+1}) of C.  B (and A) must be resident on every rank —
  * spg_broadcast_csr replicates a matrix from `root` over NCCL. */
 spg_status spg_get_unique_id(void* id128);   /* ncclGetUniqueId (128 bytes), call on one rank */
+/* A handle for rank `rank` of `nranks`: symbolic/numeric compute only this rank's rows.
+ * id128 = NULL creates a VIRTUAL rank (no communicator; collectives return BAD_STATE) — the
+ * partitioned pipeline can then be run block by block on one GPU. */
 spg_status spg_create_dist(spg_handle* h, int device, void* cuda_stream, spg_dtype dtype, const void* id128,
                            int rank, int nranks);
 /* In-place broadcast of a device CSR (row_ptr, col_idx, vals) whose buffers are already

@@ -259,11 +259,12 @@ def spg_get_unique_id() -> bytes:
     return buf.raw
 
 
-def spg_create_dist(device: int, stream, dtype, uid: bytes, rank: int, nranks: int) -> int:
+def spg_create_dist(device: int, stream, dtype, uid, rank: int, nranks: int) -> int:
+    """uid = None creates a virtual rank (partitioned rows, no communicator)."""
     h = c_void_p()
     with torch.cuda.device(device):
         st = _stream_ptr(stream)
-    buf = ctypes.create_string_buffer(uid, 128)
+    buf = ctypes.create_string_buffer(uid, 128) if uid is not None else None
     _check(None, load().spg_create_dist(byref(h), device, st, _dt(dtype), buf, rank, nranks))
     return h.value
 

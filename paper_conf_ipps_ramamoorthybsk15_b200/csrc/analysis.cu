@@ -308,6 +308,21 @@ __global__ void k_rebase(long long* __restrict__ rp, int M, int P, const int* __
   }
 }
 
+// Canonicalisation helpers (SPG_OPT_INPUT_CANONICAL = 0): iota, constant fill, narrowing copy.
+__global__ void k_iota(int* __restrict__ p, long long n) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+    p[i] = (int)i;
+}
+template <typename V>
+__global__ void k_fill(V* __restrict__ p, long long n, V v) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+    p[i] = v;
+}
+__global__ void k_narrow(const long long* __restrict__ in, int* __restrict__ out, long long n) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+    out[i] = (int)in[i];
+}
+
 // ---- host launchers ------------------------------------------------------------------------
 cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB,
                              int* f, uint8_t* nz, int* sp, unsigned long long* hist, int* err, int* amax) {
@@ -358,6 +373,23 @@ cudaError_t launch_rebase(cudaStream_t st, long long* rp_full, int M, int P, con
   int grid = (M + 1 + 255) / 256;
   if (grid > 4096) grid = 4096;
   k_rebase<<<grid, 256, 0, st>>>(rp_full, M, P, splits, off);
+  return cudaGetLastError();
+}
+
+static int grid_for(long long n) { long long g = (n + 255) / 256; return (int)(g < 1 ? 1 : (g > 4096 ? 4096 : g)); }
+cudaError_t launch_iota(cudaStream_t st, int* p, long long n) {
+  if (n > 0) k_iota<<<grid_for(n), 256, 0, st>>>(p, n);
+  return cudaGetLastError();
+}
+template <typename V>
+cudaError_t launch_fill(cudaStream_t st, V* p, long long n, V v) {
+  if (n > 0) k_fill<V><<<grid_for(n), 256, 0, st>>>(p, n, v);
+  return cudaGetLastError();
+}
+template cudaError_t launch_fill<double>(cudaStream_t, double*, long long, double);
+template cudaError_t launch_fill<float>(cudaStream_t, float*, long long, float);
+cudaError_t launch_narrow(cudaStream_t st, const long long* in, int* out, long long n) {
+  if (n > 0) k_narrow<<<grid_for(n), 256, 0, st>>>(in, out, n);
   return cudaGetLastError();
 }
 

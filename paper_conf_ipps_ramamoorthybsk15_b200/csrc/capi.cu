@@ -93,7 +93,10 @@ struct spg_ctx {
   int light_max = 256, medium_max = MEDIUM_CAP, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
   // workspace
-  DevBuf f, nz, sp, lists, small, scan_tmp, Pf, splits, canonB[3], iota, ones, crow_tmp;
+  DevBuf f, nz, sp, lists, small, scan_tmp, Pf, splits, canonB[4], iota, ones, crow_tmp;
+  spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
+  spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
+  long long iota_n = -1, ones_n = -1;
   HostRead* hr = nullptr;
   cudaStream_t aux[NUM_BINS] = {};
   cudaEvent_t ev_fork = nullptr, ev_join[NUM_BINS] = {};
@@ -264,6 +267,50 @@ spg_status split_points(spg_handle h, int M, int P) {
   return SPG_OK;
 }
 
+spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dtype);
+
+// SPG_OPT_INPUT_CANONICAL = 0: B' = canonical B (rows sorted, duplicates summed), computed by
+// this library's own SpGEMM as A' x B'' with A' = pattern of B with unit values (columns =
+// positions 0..nnzB-1) and B'' = one row per stored entry of B — every stored entry becomes a
+// one-product run, so the row merge / bitmap kernels sort and add them.  values_only: reuse the
+// structure of the last call and recompute the values (numeric on new B values).
+template <typename V>
+spg_status canonicalize(spg_handle h, const spg_csr* B, bool values_only) {
+  const long long nnzB = B->nnz;
+  if (!h->canon) {
+    spg_status s = create_common(&h->canon, h->device, h->stream, h->dtype);
+    if (s != SPG_OK) return setf(h, s, "cannot create the canonicalisation sub-handle");
+    h->canon->concurrent = h->concurrent;
+  }
+  spg_handle c = h->canon;
+  if (h->iota_n != nnzB) {
+    CK(h->iota.ensure(((size_t)nnzB + 1) * sizeof(int)));
+    CK(launch_iota(h->stream, h->iota.as<int>(), nnzB + 1));
+    CK(h->ones.ensure(((size_t)nnzB + 1) * sizeof(V)));
+    CK(launch_fill<V>(h->stream, h->ones.as<V>(), nnzB, V(1)));
+    h->iota_n = nnzB;
+    values_only = false;
+  }
+  spg_csr A1{B->nrows, (int32_t)nnzB, nnzB, B->row_ptr, h->iota.as<int32_t>(), h->ones.p};
+  spg_csr B1{(int32_t)nnzB, B->ncols, nnzB, h->iota.as<int32_t>(), B->col_idx, B->vals};
+  spg_status s;
+  if (!values_only || !c->sym_ok) {
+    CK(h->canonB[3].ensure(((size_t)B->nrows + 1) * sizeof(long long)));
+    int64_t nc = 0;
+    if ((s = spg_spgemm_symbolic(c, &A1, &B1, h->canonB[3].as<int64_t>(), &nc, nullptr, nullptr)) != SPG_OK)
+      return setf(h, s, "canonicalising B: %s", c->err.c_str());
+    CK(h->canonB[0].ensure(((size_t)B->nrows + 1) * sizeof(int)));
+    CK(h->canonB[1].ensure((size_t)(nc > 0 ? nc : 1) * sizeof(int)));
+    CK(h->canonB[2].ensure((size_t)(nc > 0 ? nc : 1) * sizeof(V)));
+    CK(launch_narrow(h->stream, h->canonB[3].as<long long>(), h->canonB[0].as<int>(), (long long)B->nrows + 1));
+    h->Bc = spg_csr{B->nrows, B->ncols, nc, h->canonB[0].as<int32_t>(), h->canonB[1].as<int32_t>(), h->canonB[2].p};
+  }
+  if ((s = spg_spgemm_numeric(c, &A1, &B1, h->canonB[3].as<int64_t>(), h->canonB[1].as<int32_t>(), h->canonB[2].p)) !=
+      SPG_OK)
+    return setf(h, s, "canonicalising B: %s", c->err.c_str());
+  return SPG_OK;
+}
+
 // SPG_OPT_VALIDATE: structural checks of both inputs on the device, before any kernel that
 // would index with them.  One extra stream sync.
 spg_status validate_device(spg_handle h, const spg_csr* A, const spg_csr* B) {
@@ -304,6 +351,8 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   } else {
     h->rb = 0;
     h->re = M;
+    h->hr->splits[0] = 0;
+    h->hr->splits[1] = M;
   }
   const long long Mloc = h->re - h->rb;
   Small* ds = h->small.as<Small>();
@@ -447,6 +496,7 @@ spg_status spg_spgemm_free(spg_handle h) {
                       &h->ones, &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
+    if (h->canon) spg_spgemm_free(h->canon);
     for (auto& b : h->hbuf) b.release();
     for (int c = 0; c < NUM_BINS; ++c) {
       if (h->aux[c]) cudaStreamDestroy(h->aux[c]);
@@ -541,10 +591,18 @@ spg_status spg_spgemm_symbolic(spg_handle h, const spg_csr* A, const spg_csr* B,
   spg_status s = validate_pair(h, A, B, false);
   if (s != SPG_OK) return s;
   if (!C_row_ptr) return setf(h, SPG_ERR_INVALID_ARGUMENT, "C_row_ptr is NULL");
-  if (!h->canonical) return setf(h, SPG_ERR_NOT_SUPPORTED, "INPUT_CANONICAL = 0 is not implemented yet");
   DeviceGuard g(h->device);
-  return h->dtype == SPG_FP64 ? symbolic_impl<double>(h, A, B, C_row_ptr, nnzC, row_begin, row_end)
-                              : symbolic_impl<float>(h, A, B, C_row_ptr, nnzC, row_begin, row_end);
+  const spg_csr* Bx = B;
+  if (!h->canonical) {
+    if (!B->vals && B->nnz > 0) return setf(h, SPG_ERR_INVALID_ARGUMENT, "INPUT_CANONICAL = 0 needs B.vals");
+    s = h->dtype == SPG_FP64 ? canonicalize<double>(h, B, false) : canonicalize<float>(h, B, false);
+    if (s != SPG_OK) return s;
+    Bx = &h->Bc;
+  }
+  s = h->dtype == SPG_FP64 ? symbolic_impl<double>(h, A, Bx, C_row_ptr, nnzC, row_begin, row_end)
+                           : symbolic_impl<float>(h, A, Bx, C_row_ptr, nnzC, row_begin, row_end);
+  if (s == SPG_OK) h->key = make_key(A, B);
+  return s;
 }
 
 spg_status spg_spgemm_numeric(spg_handle h, const spg_csr* A, const spg_csr* B, const int64_t* C_row_ptr,
@@ -558,8 +616,14 @@ spg_status spg_spgemm_numeric(spg_handle h, const spg_csr* A, const spg_csr* B, 
   if (!C_row_ptr || (h->nnzC > 0 && (!C_col_idx || !C_vals)))
     return setf(h, SPG_ERR_INVALID_ARGUMENT, "C output pointer is NULL");
   DeviceGuard g(h->device);
-  return h->dtype == SPG_FP64 ? numeric_impl<double>(h, A, B, C_row_ptr, C_col_idx, C_vals)
-                              : numeric_impl<float>(h, A, B, C_row_ptr, C_col_idx, C_vals);
+  const spg_csr* Bx = B;
+  if (!h->canonical) {
+    s = h->dtype == SPG_FP64 ? canonicalize<double>(h, B, true) : canonicalize<float>(h, B, true);
+    if (s != SPG_OK) return s;
+    Bx = &h->Bc;
+  }
+  return h->dtype == SPG_FP64 ? numeric_impl<double>(h, A, Bx, C_row_ptr, C_col_idx, C_vals)
+                              : numeric_impl<float>(h, A, Bx, C_row_ptr, C_col_idx, C_vals);
 }
 
 // ---- end-to-end host path -------------------------------------------------------------------
@@ -647,12 +711,13 @@ spg_status spg_get_unique_id(void* id128) {
 
 spg_status spg_create_dist(spg_handle* out, int device, void* cuda_stream, spg_dtype dtype, const void* id128,
                            int rank, int nranks) {
-  if (!out || !id128 || nranks < 1 || rank < 0 || rank >= nranks || nranks > 1024) return SPG_ERR_INVALID_ARGUMENT;
+  if (!out || nranks < 1 || rank < 0 || rank >= nranks || nranks > 1024) return SPG_ERR_INVALID_ARGUMENT;
   spg_status s = create_common(out, device, cuda_stream, dtype);
   if (s != SPG_OK) return s;
   spg_handle h = *out;
   h->rank = rank;
   h->nranks = nranks;
+  if (!id128) return SPG_OK;  // virtual rank: partitioned rows, no communicator
   DeviceGuard g(device);
   ncclUniqueId id;
   std::memcpy(&id, id128, sizeof id);

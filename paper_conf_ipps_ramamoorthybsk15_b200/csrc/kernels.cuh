@@ -48,6 +48,10 @@ cudaError_t launch_split_points(cudaStream_t st, const long long* Pf, int M, int
 cudaError_t launch_validate(cudaStream_t st, int sms, int M, const int* rp, const int* ci, int ncols, long long nnz,
                             int check_sorted, int* err);
 cudaError_t launch_rebase(cudaStream_t st, long long* rp_full, int M, int P, const int* splits, const long long* off);
+cudaError_t launch_iota(cudaStream_t st, int* p, long long n);
+template <typename V>
+cudaError_t launch_fill(cudaStream_t st, V* p, long long n, V v);
+cudaError_t launch_narrow(cudaStream_t st, const long long* in, int* out, long long n);
 
 // Class kernels: one launcher per bin and phase.  `count` is the device-side bin size; `grid`
 // is chosen by the caller (persistent grid-stride loops inside).  N = columns of B.

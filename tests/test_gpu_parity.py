@@ -255,3 +255,91 @@ def test_rmat23_sampled_and_row_sums():
         got[r0:r1] = torch.segment_reduce(C.vals[s:e], "sum", offsets=off, axis=0)
     torch.testing.assert_close(got, ref, rtol=1e-12, atol=0)
     plan.close()
+
+
+# ---- non-canonical B (SPG_OPT_INPUT_CANONICAL = 0) -----------------------------------------
+@pytest.mark.parametrize("force", [-1, 3, 6])
+def test_noncanonical_B_library_sorts(force):
+    A = W.random_csr(120, 90, 0.08, 11, values="int", canonical=False)
+    B = W.random_csr(90, 140, 0.08, 12, values="int", canonical=False)
+    rng = np.random.default_rng(3)
+    for M in (A, B):
+        for i in range(M.nrows):
+            s, e = M.row_ptr[i], M.row_ptr[i + 1]
+            p = rng.permutation(e - s) + s
+            M.col_idx[s:e], M.vals[s:e] = M.col_idx[p], M.vals[p]
+    got = run_gpu(A, B, input_canonical=0, force_class=force)
+    compare(A, B, got, exact_values=True)
+
+
+def test_noncanonical_B_numeric_rerun():
+    A, _ = W.make("cl10k")
+    Bn = W.random_csr(A.ncols, 3000, 0.002, 4, canonical=False)
+    dA, dB = to_dev(A), to_dev(Bn)
+    plan = spg.SpGEMM(0, torch.float64, input_canonical=0)
+    C = plan.symbolic(dA, dB)
+    plan.numeric(dA, dB, C)
+    dB2 = spg.DeviceCSR(dB.nrows, dB.ncols, dB.row_ptr, dB.col_idx, dB.vals * 3.0)
+    plan.numeric(dA, dB2, C)
+    torch.cuda.synchronize()
+    B2 = W.CSR(Bn.nrows, Bn.ncols, Bn.row_ptr, Bn.col_idx, Bn.vals * 3.0)
+    compare(A, B2, (C.row_ptr.cpu().numpy(), C.col_idx.cpu().numpy(), C.vals.cpu().numpy()))
+    plan.close()
+
+
+# ---- multi-GPU pipeline: virtual ranks (partitioned rows on one GPU) and a real 1-rank comm --
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+def test_virtual_ranks_concatenate_to_full(P):
+    A, B = W.make("cl10k")
+    ref = oracle.spgemm(A, B, nthreads=8)
+    f = oracle.row_flops(A, B)
+    s_ref = oracle.split_points(f, P)
+    dA = to_dev(A)
+    rps, cols, vals = [], [], []
+    for r in range(P):
+        h = spg.spg_create_dist(0, None, torch.float64, None, r, P)
+        try:
+            rp = torch.empty(A.nrows + 1, dtype=torch.int64, device="cuda")
+            nnz, rb, re = spg.spg_spgemm_symbolic(h, dA, dA, rp)
+            assert (rb, re) == (int(s_ref[r]), int(s_ref[r + 1]))
+            col = torch.empty(max(nnz, 1), dtype=torch.int32, device="cuda")
+            val = torch.empty(max(nnz, 1), dtype=torch.float64, device="cuda")
+            spg.spg_spgemm_numeric(h, dA, dA, rp, col, val)
+            torch.cuda.synchronize()
+            st = spg.spg_get_stats(h)
+            assert st["flops_total"] == f.sum() and st["flops"] == f[rb:re].sum()
+            rps.append(rp[: re - rb + 1].cpu().numpy())
+            cols.append(col[:nnz].cpu().numpy())
+            vals.append(val[:nnz].cpu().numpy())
+        finally:
+            spg.spg_spgemm_free(h)
+    off = 0
+    full_rp = [np.zeros(1, np.int64)]
+    for rp in rps:
+        full_rp.append(rp[1:] + off)
+        off += int(rp[-1])
+    got = (np.concatenate(full_rp), np.concatenate(cols), np.concatenate(vals))
+    compare(A, B, got, ref=ref)
+
+
+def test_nccl_single_rank_broadcast_allgatherv():
+    A, B = W.make("cl10k")
+    uid = spg.spg_get_unique_id()
+    h = spg.spg_create_dist(0, None, torch.float64, uid, 0, 1)
+    try:
+        dA = to_dev(A)
+        spg.spg_broadcast_csr(h, dA, 0)
+        rp = torch.empty(A.nrows + 1, dtype=torch.int64, device="cuda")
+        nnz, rb, re = spg.spg_spgemm_symbolic(h, dA, dA, rp)
+        col = torch.empty(nnz, dtype=torch.int32, device="cuda")
+        val = torch.empty(nnz, dtype=torch.float64, device="cuda")
+        spg.spg_spgemm_numeric(h, dA, dA, rp, col, val)
+        assert spg.spg_allgather_nnz(h, nnz) == nnz
+        full = spg.DeviceCSR64(A.nrows, A.ncols, torch.empty(A.nrows + 1, dtype=torch.int64, device="cuda"),
+                               torch.empty(nnz, dtype=torch.int32, device="cuda"),
+                               torch.empty(nnz, dtype=torch.float64, device="cuda"))
+        spg.spg_allgatherv_c(h, spg.DeviceCSR64(A.nrows, A.ncols, rp, col, val), full)
+        torch.cuda.synchronize()
+        compare(A, B, (full.row_ptr.cpu().numpy(), full.col_idx.cpu().numpy(), full.vals.cpu().numpy()))
+    finally:
+        spg.spg_spgemm_free(h)

@@ -40,8 +40,7 @@ constexpr int MED1_CAP = 1024;        // MEDIUM rows split by shared-memory foot
 constexpr int MEDIUM_CAP = 2048;
 constexpr int HEAVY_CAP = 8192;       // largest f of the shared-memory-values bitmap mode
 constexpr int BMP_NT = 1024;          // bitmap kernel block size (one block per SM)
-constexpr int MERGE_VT_MIN = 4;       // outputs per thread per merge round: clamp(f / G, 4, 14) | 1
-constexpr int MERGE_VT_MAX = 14;
+constexpr int MERGE_VT_MAX = 14;      // outputs per thread per merge round: min(ceil(f / G), 14) | 1
 
 // Shared-memory bytes a merge of f products (nr <= f runs) needs: values x2, keys x2, seg.
 template <typename V>

@@ -9,8 +9,8 @@
 // Scale-free rows are skewed: one long B row (a hub) usually carries most of the products
 // (DESIGN.md §4).  The longest run is therefore moved to the end and
 // merged last, so the log2(#runs) rounds only touch the short runs' products and the hub's
-// products move once.  Each thread emits 4..16 outputs per round so the merge-path search
-// (log2 of the run length) is amortised.
+// products move once.  Each thread emits ceil(round size / threads) outputs per round (odd,
+// <= 15), so every lane works and the merge-path search is amortised on long rounds.
 #pragma once
 #include "kernels.cuh"
 
@@ -34,7 +34,8 @@ __device__ __forceinline__ void merge_round(const int* sk, int* dk, const V* sv,
   const int npairs = (nr + 2 * w - 1) >> lw2;
   // odd: each thread writes vt consecutive outputs, so an even vt would put lanes on the same
   // shared-memory banks (vt = 16 is a 16-way conflict)
-  const int vt = min(MERGE_VT_MAX, max(MERGE_VT_MIN, (fr + G - 1) / G)) | 1;
+  // (and as small as covers the round with every thread: idle lanes still pay each instruction)
+  const int vt = min(MERGE_VT_MAX, (fr + G - 1) / G) | 1;
   for (int o0 = rank * vt; o0 < fr; o0 += G * vt) {
     int o = o0;
     const int oend = min(o0 + vt, fr);

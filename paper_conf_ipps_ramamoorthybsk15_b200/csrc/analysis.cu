@@ -78,9 +78,10 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
     unsigned f = s_f[t];
     if (f > (unsigned)INT_MAX) f = INT_MAX;
     f_out[r0 + t] = (int)f;
-    // bit 7: the A row has more entries than one bitmap-tier run chunk (HEAVY caches products
-    // of single-chunk rows in registers; longer rows take the HUGE path)
-    nz_out[r0 + t] = (uint8_t)(min(s_nz[t], 2) | (s_rp[t + 1] - s_rp[t] > BMP_NT ? 0x80 : 0));
+    // bits 6/7: the A row has more entries than a 512- / 1024-thread bitmap block gathers in one
+    // chunk (HEAVY kernels cache single-chunk rows' products in registers; longer rows move up)
+    const int alen = s_rp[t + 1] - s_rp[t];
+    nz_out[r0 + t] = (uint8_t)(min(s_nz[t], 2) | (alen > BMP_NT_S ? 0x40 : 0) | (alen > BMP_NT ? 0x80 : 0));
     sp_out[r0 + t] = s_sp[t];
     const int b = f == 0 ? 0 : 1 + (f == 1 ? 0 : 32 - __clz((int)f - 1));
     atomicAdd(&s_hist[b], 1u);
@@ -94,8 +95,8 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
 
 __device__ __forceinline__ int classify_bin(int f, int nz, const ClassParams& p) {
   if (f == 0) return -1;
-  const bool longrow = nz & 0x80;
-  nz &= 0x7f;
+  const bool long1 = nz & 0x40, long2 = nz & 0x80;
+  nz &= 0x3f;
   if (p.force < 0 && nz == 1 && p.single_ok) return BIN_SINGLE;
   int b;
   if (f <= 4) b = BIN_T4;
@@ -104,13 +105,14 @@ __device__ __forceinline__ int classify_bin(int f, int nz, const ClassParams& p)
   else if (f <= TINY_MAX) b = BIN_T32;
   else if (f <= p.light_max) b = BIN_LIGHT;
   else if (f <= p.medium_max) b = f <= MED1_CAP ? BIN_MED1 : BIN_MED2;
-  else if (f <= p.heavy_max) b = BIN_HEAVY;
+  else if (f <= p.heavy_max) b = f <= HEAVY1_CAP ? BIN_HEAVY : BIN_HEAVY2;
   else b = BIN_HUGE;
   if (p.force > CLS_TINY) {  // forced class: smallest bin of that class at least
     const int fb = class_first_bin(p.force);
     if (fb > b) b = fb;
   }
-  if (b == BIN_HEAVY && longrow) b = BIN_HUGE;
+  if (b == BIN_HEAVY && long1) b = BIN_HEAVY2;
+  if (b == BIN_HEAVY2 && long2) b = BIN_HUGE;
   return b;
 }
 

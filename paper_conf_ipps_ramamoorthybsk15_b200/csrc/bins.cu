@@ -11,10 +11,11 @@ template <typename V> int small_occupancy(int, bool);
 template <typename V>
 cudaError_t small_launch(int, cudaStream_t, int, bool, const Prob<V>&, const int*, const int*);
 template <typename V> cudaError_t bitmap_configure();
+template <typename V> int bitmap_occupancy(int, bool);
 template <typename V>
 cudaError_t bitmap_launch(int, cudaStream_t, int, bool, const Prob<V>&, const int*, const int*, long long);
 
-static bool is_bitmap(int bin) { return bin == BIN_HEAVY || bin == BIN_HUGE; }
+static bool is_bitmap(int bin) { return bin == BIN_HEAVY || bin == BIN_HEAVY2 || bin == BIN_HUGE; }
 
 template <typename V>
 cudaError_t BinLaunch<V>::launch(int bin, cudaStream_t st, int grid, bool numeric, const Prob<V>& P, const int* list,
@@ -30,7 +31,7 @@ int BinLaunch<V>::rows_per_block(int bin) {
 
 template <typename V>
 int BinLaunch<V>::max_blocks_per_sm(int bin, bool numeric) {
-  return is_bitmap(bin) ? 1 : small_occupancy<V>(bin, numeric);
+  return is_bitmap(bin) ? bitmap_occupancy<V>(bin, numeric) : small_occupancy<V>(bin, numeric);
 }
 
 template <typename V>

@@ -42,6 +42,7 @@ struct DevBuf {
 // Small per-call device scratch (zeroed at the start of every symbolic call).
 struct Small {
   int counts[16];  // per bin
+  int qhead[16];   // per bin: dynamic row-queue heads of the bitmap kernels (counts + 16)
   int err;
   int range[2];
   int amax;       // longest row of A
@@ -195,9 +196,10 @@ spg_status run_bins(spg_handle h, const spg_csr* A, const spg_csr* B, bool numer
   int* lists = h->lists.as<int>();
   const long long Mloc = h->re - h->rb;
   const bool conc = h->concurrent != 0;
+  CK(cudaMemsetAsync(ds->qhead, 0, sizeof(ds->qhead), h->stream));
   if (conc) CK(cudaEventRecord(h->ev_fork, h->stream));
-  const int order[] = {BIN_HUGE, BIN_HEAVY, BIN_MED2, BIN_MED1, BIN_LIGHT, BIN_T32, BIN_T16, BIN_T8, BIN_T4,
-                       BIN_SINGLE};
+  const int order[] = {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY, BIN_MED2, BIN_MED1, BIN_LIGHT, BIN_T32, BIN_T16, BIN_T8,
+                       BIN_T4, BIN_SINGLE};
   for (int b : order) {
     if (b == BIN_SINGLE && !numeric) continue;  // c_i = f_i written by classify
     if (numeric && h->counts[b] == 0) continue;
@@ -206,7 +208,7 @@ spg_status run_bins(spg_handle h, const spg_csr* A, const spg_csr* B, bool numer
     const int* list = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
     const int rpb = BinLaunch<V>::rows_per_block(b);
     long long grid = (long long)h->max_bpsm[numeric][b] * h->sms;
-    if ((b == BIN_HEAVY || b == BIN_HUGE) && h->huge_slots_opt > 0 && h->huge_slots_opt < grid)
+    if ((b == BIN_HEAVY || b == BIN_HEAVY2 || b == BIN_HUGE) && h->huge_slots_opt > 0 && h->huge_slots_opt < grid)
       grid = h->huge_slots_opt;
     if (numeric) {
       const long long need = (h->counts[b] + rpb - 1) / rpb;

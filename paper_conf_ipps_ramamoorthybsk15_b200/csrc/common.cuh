@@ -14,14 +14,15 @@ enum : int { CLS_EMPTY = 0, CLS_SINGLE, CLS_TINY, CLS_LIGHT, CLS_MEDIUM, CLS_HEA
 
 // Internal work lists ("bins"): a class may be split by kernel geometry (TINY by sub-warp width).
 enum : int {
-  BIN_SINGLE = 0, BIN_T4, BIN_T8, BIN_T16, BIN_T32, BIN_LIGHT, BIN_MED1, BIN_MED2, BIN_HEAVY, BIN_HUGE, NUM_BINS
+  BIN_SINGLE = 0, BIN_T4, BIN_T8, BIN_T16, BIN_T32, BIN_LIGHT, BIN_MED1, BIN_MED2, BIN_HEAVY, BIN_HEAVY2, BIN_HUGE,
+  NUM_BINS
 };
 __host__ __device__ constexpr int bin_class(int b) {
   return b == BIN_SINGLE ? CLS_SINGLE
        : b <= BIN_T32   ? CLS_TINY
        : b == BIN_LIGHT ? CLS_LIGHT
        : b <= BIN_MED2  ? CLS_MEDIUM
-       : b == BIN_HEAVY ? CLS_HEAVY : CLS_HUGE;
+       : b <= BIN_HEAVY2 ? CLS_HEAVY : CLS_HUGE;
 }
 __host__ __device__ constexpr int class_first_bin(int c) {
   return c == CLS_SINGLE ? BIN_SINGLE
@@ -38,8 +39,10 @@ constexpr int LIGHT_WARPS = 8;        // warps per block in the light kernel
 constexpr int MEDIUM_NT = 128;
 constexpr int MED1_CAP = 1024;        // MEDIUM rows split by shared-memory footprint
 constexpr int MEDIUM_CAP = 2048;
-constexpr int HEAVY_CAP = 8192;       // largest f of the shared-memory-values bitmap mode
-constexpr int BMP_NT = 1024;          // bitmap kernel block size (one block per SM)
+constexpr int HEAVY_CAP = 8192;       // largest f of the register-cached bitmap mode
+constexpr int HEAVY1_CAP = 4096;      // HEAVY rows up to this f run as 512-thread blocks, 2 per SM
+constexpr int BMP_NT = 1024;          // bitmap kernel block size for HEAVY2 / HUGE (one block per SM)
+constexpr int BMP_NT_S = 512;         // ... for HEAVY (two blocks per SM)
 constexpr int MERGE_VT_MAX = 14;      // outputs per thread per merge round: min(ceil(f / G), 14) | 1
 
 // Shared-memory bytes a merge of f products (nr <= f runs) needs: values x2, keys x2, seg.

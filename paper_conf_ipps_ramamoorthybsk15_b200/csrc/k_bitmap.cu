@@ -26,18 +26,19 @@
 
 namespace spg {
 
-constexpr int BMP_RCAP = 1024;       // runs gathered per chunk (one per thread)
 constexpr int BMP_CTCAP = 2048;      // 32-product windows per chunk with a precomputed run index
 constexpr int BMP_SLOTS = 8;         // products per lane cached in registers (HEAVY: f <= 8192)
 constexpr int MODE_SYM = 0, MODE_HEAVY = 1, MODE_HUGE = 2;
 
 __host__ __device__ constexpr int al16(int x) { return (x + 15) & ~15; }
 
-template <typename V>
+// runs gathered per chunk = one per thread (NT); dynamic shared memory per block SMEM
+template <typename V, int NT>
 __host__ __device__ constexpr int bmp_fixed_bytes() {
-  return 2 * al16((BMP_RCAP + 1) * 4) + al16(BMP_RCAP * (int)sizeof(V)) + al16(BMP_CTCAP * 2);
+  return 2 * al16((NT + 1) * 4) + al16(NT * (int)sizeof(V)) + al16(BMP_CTCAP * 2);
 }
-constexpr int BMP_SMEM = 226 * 1024;  // dynamic shared memory per block (1 block / SM; static on top)
+constexpr int BMP_SMEM_L = 226 * 1024;  // 1024-thread blocks, one per SM (static smem on top)
+constexpr int BMP_SMEM_S = 112 * 1024;  // 512-thread blocks, two per SM
 
 // Region bytes of a 2^lw column tile: bitmap, level-1 summary (one bit per bitmap word) and —
 // numeric — rank prefixes (int per 1024 columns, u16 per 256 columns relative to its 1024),
@@ -51,9 +52,11 @@ __device__ __forceinline__ int bmp_need(int lw, int f, int nv) {
   return need;
 }
 
-template <int MODE, typename V>
-__global__ void __launch_bounds__(BMP_NT, 1) k_bitmap(Prob<V> P, const int* __restrict__ list,
-                                                     const int* __restrict__ count, int lwmax, int N) {
+template <int MODE, typename V, int BMP_NT, int BMP_SMEM>
+__global__ void __launch_bounds__(BMP_NT, BMP_SMEM > 120 * 1024 ? 1 : 2) k_bitmap(Prob<V> P, const int* __restrict__ list,
+                                                                                 const int* __restrict__ count,
+                                                                                 int lwmax, int N) {
+  constexpr int BMP_RCAP = BMP_NT;
   constexpr bool NUM = MODE != MODE_SYM;
   constexpr bool HEAVY = MODE == MODE_HEAVY;
   extern __shared__ __align__(16) unsigned char sm[];
@@ -62,8 +65,8 @@ __global__ void __launch_bounds__(BMP_NT, 1) k_bitmap(Prob<V> P, const int* __re
   V* sa = reinterpret_cast<V*>(sm + 2 * al16((BMP_RCAP + 1) * 4));         // run -> A value
   unsigned short* ctab = reinterpret_cast<unsigned short*>(sm + 2 * al16((BMP_RCAP + 1) * 4) +
                                                            al16(BMP_RCAP * (int)sizeof(V)));  // window -> run
-  unsigned char* region = sm + bmp_fixed_bytes<V>();
-  constexpr int REGION = BMP_SMEM - bmp_fixed_bytes<V>();
+  unsigned char* region = sm + bmp_fixed_bytes<V, BMP_NT>();
+  constexpr int REGION = BMP_SMEM - bmp_fixed_bytes<V, BMP_NT>();
   __shared__ int scratch[BMP_NT / 32 + 1];
   const Group<BMP_NT> g{(int)threadIdx.x, scratch};
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -73,8 +76,17 @@ __global__ void __launch_bounds__(BMP_NT, 1) k_bitmap(Prob<V> P, const int* __re
   for (int x = tid; x < REGION / 4; x += BMP_NT) reinterpret_cast<unsigned*>(region)[x] = 0;
   __syncthreads();
 
-  const int n = *count;
-  for (int t = blockIdx.x; t < n; t += gridDim.x) {
+  // Rows are taken from a dynamic queue (one atomic per row): the bin's rows differ in size by
+  // up to an order of magnitude, so static striding would leave a long tail — the paper's work
+  // queue in its intra-GPU form.  count[0] = rows, count[16] = queue head.
+  const int n = count[0];
+  __shared__ int s_next;
+  for (;;) {
+    if (tid == 0) s_next = atomicAdd(const_cast<int*>(count) + 16, 1);
+    __syncthreads();
+    const int t = s_next;
+    __syncthreads();
+    if (t >= n) break;
     const int i = list[t];
     const int pa0 = P.rpA[i], pa1 = P.rpA[i + 1];
     const int f = P.frow[i];
@@ -381,18 +393,30 @@ __global__ void __launch_bounds__(BMP_NT, 1) k_bitmap(Prob<V> P, const int* __re
 // ================================ launch glue ====================================================
 template <typename V>
 static const void* bitmap_kernel(int bin, bool numeric) {
-  if (!numeric) return (const void*)k_bitmap<MODE_SYM, V>;
-  return bin == BIN_HEAVY ? (const void*)k_bitmap<MODE_HEAVY, V> : (const void*)k_bitmap<MODE_HUGE, V>;
+  if (!numeric) return (const void*)k_bitmap<MODE_SYM, V, BMP_NT, BMP_SMEM_L>;
+  return bin == BIN_HUGE ? (const void*)k_bitmap<MODE_HUGE, V, BMP_NT, BMP_SMEM_L>
+                         : (const void*)k_bitmap<MODE_HEAVY, V, BMP_NT, BMP_SMEM_L>;
 }
+static int bitmap_threads(int) { return BMP_NT; }
+static int bitmap_smem(int) { return BMP_SMEM_L; }
 
 template <typename V>
 cudaError_t bitmap_configure() {
-  for (const void* k : {(const void*)k_bitmap<MODE_SYM, V>, (const void*)k_bitmap<MODE_HEAVY, V>,
-                        (const void*)k_bitmap<MODE_HUGE, V>}) {
-    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, BMP_SMEM);
-    if (e != cudaSuccess) return e;
-  }
+  for (int bin : {BIN_HEAVY, BIN_HEAVY2, BIN_HUGE})
+    for (int num = 0; num < 2; ++num) {
+      cudaError_t e = cudaFuncSetAttribute(bitmap_kernel<V>(bin, num), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           bitmap_smem(bin));
+      if (e != cudaSuccess) return e;
+    }
   return cudaSuccess;
+}
+
+template <typename V>
+int bitmap_occupancy(int bin, bool numeric) {
+  int nb = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, bitmap_kernel<V>(bin, numeric), bitmap_threads(bin),
+                                                bitmap_smem(bin));
+  return nb < 1 ? 1 : nb;
 }
 
 template <typename V>
@@ -402,14 +426,16 @@ cudaError_t bitmap_launch(int bin, cudaStream_t st, int grid, bool numeric, cons
   while (lwmax < 20 && ((long long)1 << lwmax) < N) ++lwmax;
   int n32 = (int)N;
   void* args[] = {(void*)&P, (void*)&list, (void*)&count, (void*)&lwmax, (void*)&n32};
-  return cudaLaunchKernel(bitmap_kernel<V>(bin, numeric), dim3(grid), dim3(BMP_NT), args, BMP_SMEM, st);
+  return cudaLaunchKernel(bitmap_kernel<V>(bin, numeric), dim3(grid), dim3(bitmap_threads(bin)), args,
+                          bitmap_smem(bin), st);
 }
 
-template cudaError_t bitmap_configure<double>();
-template cudaError_t bitmap_configure<float>();
-template cudaError_t bitmap_launch<double>(int, cudaStream_t, int, bool, const Prob<double>&, const int*, const int*,
-                                           long long);
-template cudaError_t bitmap_launch<float>(int, cudaStream_t, int, bool, const Prob<float>&, const int*, const int*,
-                                          long long);
+#define INST(V)                                                                                                   \
+  template cudaError_t bitmap_configure<V>();                                                                     \
+  template int bitmap_occupancy<V>(int, bool);                                                                    \
+  template cudaError_t bitmap_launch<V>(int, cudaStream_t, int, bool, const Prob<V>&, const int*, const int*, long long);
+INST(double)
+INST(float)
+#undef INST
 
 }  // namespace spg

@@ -195,9 +195,94 @@ __global__ void __launch_bounds__(NT) k_block(Prob<V> P, const int* __restrict__
   for (int t = blockIdx.x; t < n; t += gridDim.x) merge_row<NT, CAP, NUM, V>(P, list[t], g, smem);
 }
 
+// ================================ hash-set symbolic (LIGHT, MEDIUM) ==============================
+// Symbolic only needs c_i = |distinct columns|: insert each product's column into an
+// open-addressing set in shared memory (2f..4f slots, key = col + 1, ATOMS.CAS — native on
+// sm_100a, half the STS rate) and count the successful claims.  No merge, no sort.
+template <int G, int TCAP>
+__device__ __forceinline__ void hash_count_row(const Prob<double>& P0, const int* __restrict__ rpA,
+                                               const int* __restrict__ colA, const int* __restrict__ rpB,
+                                               const int* __restrict__ colB, int i, int f, const Group<G>& g,
+                                               unsigned* table, int* seg, int* sbs, long long* crow, int row_begin) {
+  (void)P0;
+  int lt = 1;
+  while ((1 << lt) < 2 * f) ++lt;  // table size 2^lt >= 2f
+  const int T = 1 << lt;
+  for (int x = g.rank; x < T; x += G) table[x] = 0u;
+  const int pa0 = rpA[i], pa1 = rpA[i + 1];
+  int nr = 0, tot = 0;
+  for (int p0 = pa0; p0 < pa1; p0 += G) {
+    const int p = p0 + g.rank;
+    int L = 0, bs = 0;
+    if (p < pa1) {
+      const int k = colA[p];
+      bs = rpB[k];
+      L = rpB[k + 1] - bs;
+    }
+    int t2;
+    const int ex = g.excl_scan((L << 16) | (L > 0 ? 1 : 0), t2);  // f <= 2048, G <= 128
+    if (L > 0) {
+      seg[nr + (ex & 0xffff)] = tot + (ex >> 16);
+      sbs[nr + (ex & 0xffff)] = bs;
+    }
+    nr += t2 & 0xffff;
+    tot += t2 >> 16;
+  }
+  if (g.rank == 0) seg[nr] = tot;
+  g.sync();
+  int cnt = 0;
+  for (int j = g.rank; j < tot; j += G) {
+    const int r = upper_idx(seg, nr, j);
+    const unsigned key = (unsigned)colB[sbs[r] + (j - seg[r])] + 1u;
+    unsigned h = (key * 0x9E3779B1u) >> (32 - lt);
+    while (true) {
+      const unsigned old = atomicCAS(&table[h], 0u, key);
+      if (old == 0u) { ++cnt; break; }
+      if (old == key) break;
+      h = (h + 1) & (T - 1);
+    }
+  }
+  const long long c = g.sum(cnt);
+  if (g.rank == 0) crow[i - row_begin + 1] = c;
+  g.sync();
+}
+
+template <typename V, int TCAP>
+__global__ void __launch_bounds__(LIGHT_WARPS * 32) k_hsym_warp(Prob<V> P, const int* __restrict__ list,
+                                                               const int* __restrict__ count) {
+  __shared__ unsigned s_table[LIGHT_WARPS][TCAP];
+  __shared__ int s_seg[LIGHT_WARPS][TCAP / 2 + 1];
+  __shared__ int s_bs[LIGHT_WARPS][TCAP / 2];
+  const int warp = threadIdx.x >> 5;
+  const Group<32> g{lane_id(), nullptr};
+  const int n = *count;
+  for (int t = blockIdx.x * LIGHT_WARPS + warp; t < n; t += gridDim.x * LIGHT_WARPS) {
+    const int i = list[t];
+    hash_count_row<32, TCAP>(Prob<double>{}, P.rpA, P.colA, P.rpB, P.colB, i, P.frow[i], g, s_table[warp],
+                             s_seg[warp], s_bs[warp], P.crow, P.row_begin);
+  }
+}
+
+template <typename V, int NT, int TCAP>
+__global__ void __launch_bounds__(NT) k_hsym_block(Prob<V> P, const int* __restrict__ list,
+                                                  const int* __restrict__ count) {
+  __shared__ unsigned s_table[TCAP];
+  __shared__ int s_seg[TCAP / 2 + 1];
+  __shared__ int s_bs[TCAP / 2];
+  __shared__ int scratch[NT / 32 + 1];
+  const Group<NT> g{(int)threadIdx.x, scratch};
+  const int n = *count;
+  for (int t = blockIdx.x; t < n; t += gridDim.x) {
+    const int i = list[t];
+    hash_count_row<NT, TCAP>(Prob<double>{}, P.rpA, P.colA, P.rpB, P.colB, i, P.frow[i], g, s_table, s_seg, s_bs,
+                             P.crow, P.row_begin);
+  }
+}
+
 // ================================ launch glue ====================================================
 template <typename V>
 size_t small_smem(int bin, bool numeric) {
+  if (!numeric && (bin == BIN_LIGHT || bin == BIN_MED1 || bin == BIN_MED2)) return 0;  // hash symbolic: static
   if (bin == BIN_LIGHT) return LIGHT_WARPS * (numeric ? msmem_aligned<V, true>(LIGHT_CAP) : msmem_aligned<V, false>(LIGHT_CAP));
   if (bin == BIN_MED1) return numeric ? msmem_aligned<V, true>(MED1_CAP) : msmem_aligned<V, false>(MED1_CAP);
   if (bin == BIN_MED2) return numeric ? msmem_aligned<V, true>(MEDIUM_CAP) : msmem_aligned<V, false>(MEDIUM_CAP);
@@ -228,13 +313,14 @@ static const void* small_kernel(int bin, bool numeric) {
     case BIN_T8: return numeric ? (const void*)k_tiny<8, true, V> : (const void*)k_tiny<8, false, V>;
     case BIN_T16: return numeric ? (const void*)k_tiny<16, true, V> : (const void*)k_tiny<16, false, V>;
     case BIN_T32: return numeric ? (const void*)k_tiny<32, true, V> : (const void*)k_tiny<32, false, V>;
-    case BIN_LIGHT: return numeric ? (const void*)k_light<true, V> : (const void*)k_light<false, V>;
+    case BIN_LIGHT:
+      return numeric ? (const void*)k_light<true, V> : (const void*)k_hsym_warp<V, 2 * LIGHT_CAP>;
     case BIN_MED1:
       return numeric ? (const void*)k_block<MEDIUM_NT, MED1_CAP, true, V>
-                     : (const void*)k_block<MEDIUM_NT, MED1_CAP, false, V>;
+                     : (const void*)k_hsym_block<V, MEDIUM_NT, 2 * MED1_CAP>;
     case BIN_MED2:
       return numeric ? (const void*)k_block<MEDIUM_NT, MEDIUM_CAP, true, V>
-                     : (const void*)k_block<MEDIUM_NT, MEDIUM_CAP, false, V>;
+                     : (const void*)k_hsym_block<V, MEDIUM_NT, 2 * MEDIUM_CAP>;
   }
   return nullptr;
 }
@@ -242,7 +328,7 @@ static const void* small_kernel(int bin, bool numeric) {
 template <typename V>
 cudaError_t small_configure() {
   for (int bin : {BIN_LIGHT, BIN_MED1, BIN_MED2})
-    for (int num = 0; num < 2; ++num) {
+    for (int num = 1; num < 2; ++num) {
       cudaError_t e = cudaFuncSetAttribute(small_kernel<V>(bin, num), cudaFuncAttributeMaxDynamicSharedMemorySize,
                                            (int)small_smem<V>(bin, num));
       if (e != cudaSuccess) return e;

@@ -136,12 +136,37 @@ __device__ __forceinline__ void merge_row(const Prob<V>& P, const int i, const G
     g.sync();
   }
 
-  // 3. expand: product j of run r -> keyX[j] = colB, valX[j] = a_r * valB (coalesced per run)
-  for (int j = g.rank; j < f; j += G) {
-    const int r = upper_idx(seg, nr, j);
-    const int q = keyY[r] + (j - seg[r]);
-    keyX[j] = P.colB[q];
-    if (NUM) valX[j] = valY[r] * P.valB[q];
+  // 3. expand: product j of run r -> keyX[j] = colB, valX[j] = a_r * valB (coalesced per run).
+  //    EU products per thread per step: run lookups first, then all loads, then the stores, so
+  //    one L2 round trip covers EU products.
+  constexpr int EU = 8;
+  for (int j0 = g.rank; j0 < f; j0 += G * EU) {
+    int q[EU], r[EU];
+#pragma unroll
+    for (int u = 0; u < EU; ++u) {
+      const int j = j0 + u * G;
+      r[u] = 0;
+      q[u] = -1;
+      if (j < f) {
+        r[u] = upper_idx(seg, nr, j);
+        q[u] = keyY[r[u]] + (j - seg[r[u]]);
+      }
+    }
+    int kk[EU];
+    V bb[EU];
+#pragma unroll
+    for (int u = 0; u < EU; ++u) {
+      kk[u] = q[u] >= 0 ? P.colB[q[u]] : 0;
+      if (NUM) bb[u] = q[u] >= 0 ? P.valB[q[u]] : V(0);
+    }
+#pragma unroll
+    for (int u = 0; u < EU; ++u) {
+      const int j = j0 + u * G;
+      if (j < f) {
+        keyX[j] = kk[u];
+        if (NUM) valX[j] = valY[r[u]] * bb[u];
+      }
+    }
   }
   g.sync();
   const int nrs = hub ? nr - 1 : nr;
@@ -176,24 +201,27 @@ __device__ __forceinline__ void merge_row(const Prob<V>& P, const int i, const G
     V* tv = sv; sv = dv; dv = tv;
   }
 
-  // 5. like-tuples: head = first of each equal-column group; heads add their group and write
+  // 5. like-tuples: head = first of each equal-column group; each thread owns a contiguous
+  //    segment, counts its heads, one group scan gives output positions, heads add their group.
   const long long rowoff = NUM ? P.crow[i - P.row_begin] : 0;
-  int base = 0;
-  for (int j0 = 0; j0 < f; j0 += G) {
-    const int j = j0 + g.rank;
-    const int kj = j < f ? sk[j] : KEY_INF;
-    const bool head = j < f && (j == 0 || sk[j - 1] != kj);
-    int tot;
-    const int pos = g.excl_scan(head ? 1 : 0, tot);
-    if (NUM && head) {
+  const int vo = (f + G - 1) / G;
+  const int s0 = min(g.rank * vo, f), s1 = min(s0 + vo, f);
+  int heads = 0;
+  for (int j = s0; j < s1; ++j) heads += (j == 0 || sk[j - 1] != sk[j]);
+  int tot;
+  int pos = g.excl_scan(heads, tot);
+  if (NUM) {
+    for (int j = s0; j < s1; ++j) {
+      const int kj = sk[j];
+      if (j > 0 && sk[j - 1] == kj) continue;
       V s = sv[j];
-      for (int t = j + 1; t < f && sk[t] == kj; ++t) s += sv[t];
-      P.ccol[rowoff + base + pos] = kj;
-      P.cval[rowoff + base + pos] = s;
+      for (int t2 = j + 1; t2 < f && sk[t2] == kj; ++t2) s += sv[t2];
+      P.ccol[rowoff + pos] = kj;
+      P.cval[rowoff + pos] = s;
+      ++pos;
     }
-    base += tot;
   }
-  if (!NUM && g.rank == 0) P.crow[i - P.row_begin + 1] = base;
+  if (!NUM && g.rank == 0) P.crow[i - P.row_begin + 1] = tot;
   g.sync();
 }
 

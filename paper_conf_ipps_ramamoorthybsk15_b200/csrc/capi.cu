@@ -178,6 +178,8 @@ Prob<V> make_prob(spg_handle h, const spg_csr* A, const spg_csr* B, long long* c
   P.rpB = B->row_ptr; P.colB = B->col_idx; P.valB = (const V*)B->vals;
   P.sp = h->sp.as<int>(); P.frow = h->f.as<int>();
   P.row_begin = h->rb; P.crow = crow; P.ccol = ccol; P.cval = (V*)cval;
+  P.lgN = 0;
+  while (P.lgN < 31 && ((long long)1 << P.lgN) < (long long)B->ncols) ++P.lgN;
   return P;
 }
 

@@ -35,8 +35,9 @@ __host__ __device__ constexpr int class_first_bin(int c) {
 // Class-kernel geometry.
 constexpr int TINY_MAX = 32;          // one product per lane of a 4/8/16/32-lane group
 constexpr int LIGHT_CAP = 256;        // warp merge, per-warp shared memory
-constexpr int LIGHT_WARPS = 8;        // warps per block in the light kernel
-constexpr int MEDIUM_NT = 128;
+constexpr int LIGHT_WARPS = 7;        // warps per block in the light kernel (4 blocks / SM fit in smem)
+constexpr int MED1_NT = 128;          // MEDIUM rows f <= 1024: 128-thread blocks
+constexpr int MEDIUM_NT = 256;        // MEDIUM rows f <= 2048: 256-thread blocks (occupancy)
 constexpr int MED1_CAP = 1024;        // MEDIUM rows split by shared-memory footprint
 constexpr int MEDIUM_CAP = 2048;
 constexpr int HEAVY_CAP = 8192;       // largest f of the register-cached bitmap mode

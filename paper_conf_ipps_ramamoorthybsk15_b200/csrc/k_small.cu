@@ -182,7 +182,7 @@ __global__ void __launch_bounds__(LIGHT_WARPS * 32) k_light(Prob<V> P, const int
   char* my = smem + warp * PER;
   const int n = *count;
   for (int t = blockIdx.x * LIGHT_WARPS + warp; t < n; t += gridDim.x * LIGHT_WARPS)
-    merge_row<32, LIGHT_CAP, NUM, V>(P, list[t], g, my);
+    esc_row<32, LIGHT_CAP, NUM, V>(P, list[t], g, my);
 }
 
 // ================================ MEDIUM (block merge) ==========================================
@@ -192,7 +192,7 @@ __global__ void __launch_bounds__(NT) k_block(Prob<V> P, const int* __restrict__
   __shared__ int scratch[NT / 32 + 1];
   const Group<NT> g{(int)threadIdx.x, scratch};
   const int n = *count;
-  for (int t = blockIdx.x; t < n; t += gridDim.x) merge_row<NT, CAP, NUM, V>(P, list[t], g, smem);
+  for (int t = blockIdx.x; t < n; t += gridDim.x) esc_row<NT, CAP, NUM, V>(P, list[t], g, smem);
 }
 
 // ================================ hash-set symbolic (LIGHT, MEDIUM) ==============================
@@ -290,7 +290,9 @@ size_t small_smem(int bin, bool numeric) {
 }
 
 template <typename V>
-int small_threads(int bin) { return (bin == BIN_MED1 || bin == BIN_MED2) ? MEDIUM_NT : 256; }
+int small_threads(int bin) {
+  return bin == BIN_MED1 ? MED1_NT : bin == BIN_MED2 ? MEDIUM_NT : bin == BIN_LIGHT ? LIGHT_WARPS * 32 : 256;
+}
 
 template <typename V>
 int small_rows_per_block(int bin) {
@@ -316,8 +318,8 @@ static const void* small_kernel(int bin, bool numeric) {
     case BIN_LIGHT:
       return numeric ? (const void*)k_light<true, V> : (const void*)k_hsym_warp<V, 2 * LIGHT_CAP>;
     case BIN_MED1:
-      return numeric ? (const void*)k_block<MEDIUM_NT, MED1_CAP, true, V>
-                     : (const void*)k_hsym_block<V, MEDIUM_NT, 2 * MED1_CAP>;
+      return numeric ? (const void*)k_block<MED1_NT, MED1_CAP, true, V>
+                     : (const void*)k_hsym_block<V, MED1_NT, 2 * MED1_CAP>;
     case BIN_MED2:
       return numeric ? (const void*)k_block<MEDIUM_NT, MEDIUM_CAP, true, V>
                      : (const void*)k_hsym_block<V, MEDIUM_NT, 2 * MEDIUM_CAP>;

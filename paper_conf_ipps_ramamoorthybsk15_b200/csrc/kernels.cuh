@@ -29,6 +29,7 @@ struct Prob {
   const int* sp;    // per row: index of one A entry whose B row is non-empty (row analysis)
   const int* frow;  // per row: f_i (row analysis)
   int row_begin;
+  int lgN;          // ceil(log2(N)), N = columns of B (>= 0)
   long long* crow;
   int* ccol;
   V* cval;

@@ -225,4 +225,164 @@ __device__ __forceinline__ void merge_row(const Prob<V>& P, const int i, const G
   g.sync();
 }
 
+// Bucketed ESC for one row (LIGHT / MEDIUM): expand the products, histogram them by the column's
+// high bits into NB buckets (ATOMS.ADD returns each product's slot), scan, scatter into bucket
+// order, then every thread insertion-sorts its own few buckets (random columns: ~CAP/NB
+// products per bucket), counts heads and writes the compacted row.  A fixed number of barriers
+// per row — no log2(#runs) merge rounds.  Rows whose buckets turn out skewed (clustered
+// columns, > MAXB in one bucket) fall back to merge_row.  Same shared-memory footprint as
+// merge_row: the run table's space (seg) holds the slots and bucket counts after the expand.
+template <int G, int CAP, bool NUM, typename V>
+__device__ __forceinline__ void esc_row(const Prob<V>& P, const int i, const Group<G>& g, char* smem) {
+  constexpr int NB = CAP / 4, MAXB = 48;
+  V* valX = reinterpret_cast<V*>(smem);
+  V* valY = valX + CAP;
+  int* keyX = reinterpret_cast<int*>(smem + (NUM ? 2 * CAP * sizeof(V) : 0));
+  int* keyY = keyX + CAP;
+  int* seg = keyY + CAP;
+  const int pa0 = P.rpA[i], pa1 = P.rpA[i + 1];
+  // runs (no hub handling needed)
+  int nr = 0, f = 0;
+  for (int p0 = pa0; p0 < pa1; p0 += G) {
+    const int p = p0 + g.rank;
+    int L = 0, bs = 0;
+    V a = V(0);
+    if (p < pa1) {
+      const int k = P.colA[p];
+      bs = P.rpB[k];
+      L = P.rpB[k + 1] - bs;
+      if (NUM) a = P.valA[p];
+    }
+    int tot;
+    const int ex = g.excl_scan((L << 16) | (L > 0 ? 1 : 0), tot);
+    const int slot = nr + (ex & 0xffff);
+    if (L > 0) {
+      seg[slot] = f + (ex >> 16);
+      keyY[slot] = bs;
+      if (NUM) valY[slot] = a;
+    }
+    nr += tot & 0xffff;
+    f += tot >> 16;
+  }
+  if (g.rank == 0) seg[nr] = f;
+  g.sync();
+  constexpr int EU = 8;
+  for (int j0 = g.rank; j0 < f; j0 += G * EU) {
+    int q[EU], r[EU];
+#pragma unroll
+    for (int u = 0; u < EU; ++u) {
+      const int j = j0 + u * G;
+      r[u] = 0;
+      q[u] = -1;
+      if (j < f) {
+        r[u] = upper_idx(seg, nr, j);
+        q[u] = keyY[r[u]] + (j - seg[r[u]]);
+      }
+    }
+    int kk[EU];
+    V bb[EU];
+#pragma unroll
+    for (int u = 0; u < EU; ++u) {
+      kk[u] = q[u] >= 0 ? P.colB[q[u]] : 0;
+      if (NUM) bb[u] = q[u] >= 0 ? P.valB[q[u]] : V(0);
+    }
+#pragma unroll
+    for (int u = 0; u < EU; ++u) {
+      const int j = j0 + u * G;
+      if (j < f) {
+        keyX[j] = kk[u];
+        if (NUM) valX[j] = valY[r[u]] * bb[u];
+      }
+    }
+  }
+  g.sync();
+  // histogram (seg area reused: cnt[NB + 1] then 16-bit slots)
+  int* cnt = seg;
+  unsigned short* slot = reinterpret_cast<unsigned short*>(seg + NB + 1);
+  const int lgNB = 31 - __clz(NB);
+  const int shift = P.lgN > lgNB ? P.lgN - lgNB : 0;
+  for (int b = g.rank; b <= NB; b += G) cnt[b] = 0;
+  g.sync();
+  for (int j = g.rank; j < f; j += G) slot[j] = (unsigned short)atomicAdd(&cnt[keyX[j] >> shift], 1);
+  g.sync();
+  // exclusive scan of the bucket counts, NB / G contiguous buckets per thread
+  constexpr int BPT = NB / G > 0 ? NB / G : 1;
+  int mine = 0, mx = 0;
+  int c8[BPT];
+#pragma unroll
+  for (int k = 0; k < BPT; ++k) {
+    const int b = g.rank * BPT + k;
+    c8[k] = b < NB ? cnt[b] : 0;
+    mine += c8[k];
+    mx = max(mx, c8[k]);
+  }
+  int tot;
+  int run = g.excl_scan(mine, tot);
+  const int mxall = g.max(mx);
+  if (mxall > MAXB) {  // clustered columns: merge instead (re-gathers the runs)
+    merge_row<G, CAP, NUM, V>(P, i, g, smem);
+    return;
+  }
+#pragma unroll
+  for (int k = 0; k < BPT; ++k) {
+    const int b = g.rank * BPT + k;
+    if (b < NB) cnt[b] = run;
+    run += c8[k];
+  }
+  if (g.rank == 0) cnt[NB] = f;
+  g.sync();
+  for (int j = g.rank; j < f; j += G) {
+    const int d = cnt[keyX[j] >> shift] + slot[j];
+    keyY[d] = keyX[j];
+    if (NUM) valY[d] = valX[j];
+  }
+  g.sync();
+  // sort each of my buckets (insertion sort), count heads
+  int heads = 0;
+#pragma unroll
+  for (int k = 0; k < BPT; ++k) {
+    const int b = g.rank * BPT + k;
+    if (b >= NB) break;
+    const int s0 = cnt[b], s1 = cnt[b + 1];
+    for (int x = s0 + 1; x < s1; ++x) {
+      const int kx = keyY[x];
+      V vx = V(0);
+      if (NUM) vx = valY[x];
+      int y = x - 1;
+      while (y >= s0 && keyY[y] > kx) {
+        keyY[y + 1] = keyY[y];
+        if (NUM) valY[y + 1] = valY[y];
+        --y;
+      }
+      keyY[y + 1] = kx;
+      if (NUM) valY[y + 1] = vx;
+    }
+    for (int x = s0; x < s1; ++x) heads += (x == s0 || keyY[x - 1] != keyY[x]);
+  }
+  int htot;
+  int pos = g.excl_scan(heads, htot);
+  if (NUM) {
+    const long long rowoff = P.crow[i - P.row_begin];
+#pragma unroll
+    for (int k = 0; k < BPT; ++k) {
+      const int b = g.rank * BPT + k;
+      if (b >= NB) break;
+      const int s0 = cnt[b], s1 = cnt[b + 1];
+      for (int x = s0; x < s1;) {
+        const int kx = keyY[x];
+        V s = valY[x];
+        int y = x + 1;
+        for (; y < s1 && keyY[y] == kx; ++y) s += valY[y];
+        P.ccol[rowoff + pos] = kx;
+        P.cval[rowoff + pos] = s;
+        ++pos;
+        x = y;
+      }
+    }
+  } else if (g.rank == 0) {
+    P.crow[i - P.row_begin + 1] = htot;
+  }
+  g.sync();
+}
+
 }  // namespace spg

@@ -103,8 +103,8 @@ __device__ __forceinline__ int classify_bin(int f, int nz, const ClassParams& p)
   else if (f <= 8) b = BIN_T8;
   else if (f <= 16) b = BIN_T16;
   else if (f <= TINY_MAX) b = BIN_T32;
-  else if (f <= p.light_max) b = BIN_LIGHT;
-  else if (f <= p.medium_max) b = f <= MED1_CAP ? BIN_MED1 : BIN_MED2;
+  else if (f <= p.light_max) b = f <= 64 ? BIN_L64 : (f <= 128 ? BIN_L128 : BIN_L256);
+  else if (f <= p.medium_max) b = f <= 512 ? BIN_M512 : (f <= 1024 ? BIN_M1024 : BIN_M2048);
   else if (f <= p.heavy_max) b = f <= HEAVY1_CAP ? BIN_HEAVY : BIN_HEAVY2;
   else b = BIN_HUGE;
   if (p.force > CLS_TINY) {  // forced class: smallest bin of that class at least

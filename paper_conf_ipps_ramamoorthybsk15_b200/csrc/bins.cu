@@ -15,7 +15,7 @@ template <typename V> int bitmap_occupancy(int, bool);
 template <typename V>
 cudaError_t bitmap_launch(int, cudaStream_t, int, bool, const Prob<V>&, const int*, const int*, long long);
 
-static bool is_bitmap(int bin) { return bin == BIN_HEAVY || bin == BIN_HEAVY2 || bin == BIN_HUGE; }
+static bool is_bitmap(int bin) { return bin_is_bitmap(bin); }
 
 template <typename V>
 cudaError_t BinLaunch<V>::launch(int bin, cudaStream_t st, int grid, bool numeric, const Prob<V>& P, const int* list,

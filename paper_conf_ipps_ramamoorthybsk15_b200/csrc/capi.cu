@@ -200,8 +200,8 @@ spg_status run_bins(spg_handle h, const spg_csr* A, const spg_csr* B, bool numer
   const bool conc = h->concurrent != 0;
   CK(cudaMemsetAsync(ds->qhead, 0, sizeof(ds->qhead), h->stream));
   if (conc) CK(cudaEventRecord(h->ev_fork, h->stream));
-  const int order[] = {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY, BIN_MED2, BIN_MED1, BIN_LIGHT, BIN_T32, BIN_T16, BIN_T8,
-                       BIN_T4, BIN_SINGLE};
+  const int order[] = {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY, BIN_M2048, BIN_M1024, BIN_M512, BIN_L256, BIN_L128,
+                       BIN_L64, BIN_T32, BIN_T16, BIN_T8, BIN_T4, BIN_SINGLE};
   for (int b : order) {
     if (b == BIN_SINGLE && !numeric) continue;  // c_i = f_i written by classify
     if (numeric && h->counts[b] == 0) continue;
@@ -210,7 +210,7 @@ spg_status run_bins(spg_handle h, const spg_csr* A, const spg_csr* B, bool numer
     const int* list = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
     const int rpb = BinLaunch<V>::rows_per_block(b);
     long long grid = (long long)h->max_bpsm[numeric][b] * h->sms;
-    if ((b == BIN_HEAVY || b == BIN_HEAVY2 || b == BIN_HUGE) && h->huge_slots_opt > 0 && h->huge_slots_opt < grid)
+    if (bin_is_bitmap(b) && h->huge_slots_opt > 0 && h->huge_slots_opt < grid)
       grid = h->huge_slots_opt;
     if (numeric) {
       const long long need = (h->counts[b] + rpb - 1) / rpb;

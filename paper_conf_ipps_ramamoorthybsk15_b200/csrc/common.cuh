@@ -14,23 +14,27 @@ enum : int { CLS_EMPTY = 0, CLS_SINGLE, CLS_TINY, CLS_LIGHT, CLS_MEDIUM, CLS_HEA
 
 // Internal work lists ("bins"): a class may be split by kernel geometry (TINY by sub-warp width).
 enum : int {
-  BIN_SINGLE = 0, BIN_T4, BIN_T8, BIN_T16, BIN_T32, BIN_LIGHT, BIN_MED1, BIN_MED2, BIN_HEAVY, BIN_HEAVY2, BIN_HUGE,
+  BIN_SINGLE = 0, BIN_T4, BIN_T8, BIN_T16, BIN_T32,   // TINY: one W-lane group per row
+  BIN_L64, BIN_L128, BIN_L256,                        // LIGHT: one warp per row, CAP = 64/128/256
+  BIN_M512, BIN_M1024, BIN_M2048,                     // MEDIUM: one block per row, CAP = 512/1024/2048
+  BIN_HEAVY, BIN_HEAVY2, BIN_HUGE,                    // HEAVY / HUGE: column-bitmap blocks
   NUM_BINS
 };
 __host__ __device__ constexpr int bin_class(int b) {
   return b == BIN_SINGLE ? CLS_SINGLE
        : b <= BIN_T32   ? CLS_TINY
-       : b == BIN_LIGHT ? CLS_LIGHT
-       : b <= BIN_MED2  ? CLS_MEDIUM
+       : b <= BIN_L256  ? CLS_LIGHT
+       : b <= BIN_M2048 ? CLS_MEDIUM
        : b <= BIN_HEAVY2 ? CLS_HEAVY : CLS_HUGE;
 }
 __host__ __device__ constexpr int class_first_bin(int c) {
   return c == CLS_SINGLE ? BIN_SINGLE
        : c == CLS_TINY   ? BIN_T4
-       : c == CLS_LIGHT  ? BIN_LIGHT
-       : c == CLS_MEDIUM ? BIN_MED1
+       : c == CLS_LIGHT  ? BIN_L64
+       : c == CLS_MEDIUM ? BIN_M512
        : c == CLS_HEAVY  ? BIN_HEAVY : BIN_HUGE;
 }
+__host__ __device__ constexpr bool bin_is_bitmap(int b) { return b >= BIN_HEAVY; }
 
 // Class-kernel geometry.
 constexpr int TINY_MAX = 32;          // one product per lane of a 4/8/16/32-lane group

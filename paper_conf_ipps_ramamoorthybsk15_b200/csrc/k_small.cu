@@ -172,17 +172,17 @@ __global__ void __launch_bounds__(256) k_tiny(Prob<V> P, const int* __restrict__
 }
 
 // ================================ LIGHT (warp merge) ============================================
-template <bool NUM, typename V>
+template <int CAP, bool NUM, typename V>
 __global__ void __launch_bounds__(LIGHT_WARPS * 32) k_light(Prob<V> P, const int* __restrict__ list,
                                                            const int* __restrict__ count) {
   extern __shared__ __align__(16) char smem[];
-  constexpr int PER = msmem_aligned<V, NUM>(LIGHT_CAP);
+  constexpr int PER = msmem_aligned<V, NUM>(CAP);
   const int warp = threadIdx.x >> 5;
   const Group<32> g{lane_id(), nullptr};
   char* my = smem + warp * PER;
   const int n = *count;
   for (int t = blockIdx.x * LIGHT_WARPS + warp; t < n; t += gridDim.x * LIGHT_WARPS)
-    esc_row<32, LIGHT_CAP, NUM, V>(P, list[t], g, my);
+    esc_row<32, CAP, NUM, V>(P, list[t], g, my);
 }
 
 // ================================ MEDIUM (block merge) ==========================================
@@ -280,18 +280,26 @@ __global__ void __launch_bounds__(NT) k_hsym_block(Prob<V> P, const int* __restr
 }
 
 // ================================ launch glue ====================================================
+// Merge-class geometry per bin: (threads per row, capacity); warp bins run LIGHT_WARPS rows per block.
+__host__ __device__ constexpr int merge_cap(int bin) {
+  return bin == BIN_L64 ? 64 : bin == BIN_L128 ? 128 : bin == BIN_L256 ? 256
+       : bin == BIN_M512 ? 512 : bin == BIN_M1024 ? 1024 : 2048;
+}
+constexpr int M512_NT = 64;
+
 template <typename V>
 size_t small_smem(int bin, bool numeric) {
-  if (!numeric && (bin == BIN_LIGHT || bin == BIN_MED1 || bin == BIN_MED2)) return 0;  // hash symbolic: static
-  if (bin == BIN_LIGHT) return LIGHT_WARPS * (numeric ? msmem_aligned<V, true>(LIGHT_CAP) : msmem_aligned<V, false>(LIGHT_CAP));
-  if (bin == BIN_MED1) return numeric ? msmem_aligned<V, true>(MED1_CAP) : msmem_aligned<V, false>(MED1_CAP);
-  if (bin == BIN_MED2) return numeric ? msmem_aligned<V, true>(MEDIUM_CAP) : msmem_aligned<V, false>(MEDIUM_CAP);
+  if (!numeric && bin >= BIN_L64 && bin <= BIN_M2048) return 0;  // hash symbolic: static shared memory
+  const int cap = merge_cap(bin);
+  if (bin >= BIN_L64 && bin <= BIN_L256) return (size_t)LIGHT_WARPS * msmem_aligned<V, true>(cap);
+  if (bin >= BIN_M512 && bin <= BIN_M2048) return msmem_aligned<V, true>(cap);
   return 0;
 }
 
 template <typename V>
 int small_threads(int bin) {
-  return bin == BIN_MED1 ? MED1_NT : bin == BIN_MED2 ? MEDIUM_NT : bin == BIN_LIGHT ? LIGHT_WARPS * 32 : 256;
+  return bin == BIN_M512 ? M512_NT : bin == BIN_M1024 ? MED1_NT : bin == BIN_M2048 ? MEDIUM_NT
+       : (bin >= BIN_L64 && bin <= BIN_L256) ? LIGHT_WARPS * 32 : 256;
 }
 
 template <typename V>
@@ -302,7 +310,7 @@ int small_rows_per_block(int bin) {
     case BIN_T8: return 8 * 4;
     case BIN_T16: return 8 * 2;
     case BIN_T32: return 8;
-    case BIN_LIGHT: return LIGHT_WARPS;
+    case BIN_L64: case BIN_L128: case BIN_L256: return LIGHT_WARPS;
     default: return 1;
   }
 }
@@ -315,26 +323,26 @@ static const void* small_kernel(int bin, bool numeric) {
     case BIN_T8: return numeric ? (const void*)k_tiny<8, true, V> : (const void*)k_tiny<8, false, V>;
     case BIN_T16: return numeric ? (const void*)k_tiny<16, true, V> : (const void*)k_tiny<16, false, V>;
     case BIN_T32: return numeric ? (const void*)k_tiny<32, true, V> : (const void*)k_tiny<32, false, V>;
-    case BIN_LIGHT:
-      return numeric ? (const void*)k_light<true, V> : (const void*)k_hsym_warp<V, 2 * LIGHT_CAP>;
-    case BIN_MED1:
-      return numeric ? (const void*)k_block<MED1_NT, MED1_CAP, true, V>
-                     : (const void*)k_hsym_block<V, MED1_NT, 2 * MED1_CAP>;
-    case BIN_MED2:
-      return numeric ? (const void*)k_block<MEDIUM_NT, MEDIUM_CAP, true, V>
-                     : (const void*)k_hsym_block<V, MEDIUM_NT, 2 * MEDIUM_CAP>;
+    case BIN_L64: return numeric ? (const void*)k_light<64, true, V> : (const void*)k_hsym_warp<V, 128>;
+    case BIN_L128: return numeric ? (const void*)k_light<128, true, V> : (const void*)k_hsym_warp<V, 256>;
+    case BIN_L256: return numeric ? (const void*)k_light<256, true, V> : (const void*)k_hsym_warp<V, 512>;
+    case BIN_M512:
+      return numeric ? (const void*)k_block<M512_NT, 512, true, V> : (const void*)k_hsym_block<V, M512_NT, 1024>;
+    case BIN_M1024:
+      return numeric ? (const void*)k_block<MED1_NT, 1024, true, V> : (const void*)k_hsym_block<V, MED1_NT, 2048>;
+    case BIN_M2048:
+      return numeric ? (const void*)k_block<MEDIUM_NT, 2048, true, V> : (const void*)k_hsym_block<V, MEDIUM_NT, 4096>;
   }
   return nullptr;
 }
 
 template <typename V>
 cudaError_t small_configure() {
-  for (int bin : {BIN_LIGHT, BIN_MED1, BIN_MED2})
-    for (int num = 1; num < 2; ++num) {
-      cudaError_t e = cudaFuncSetAttribute(small_kernel<V>(bin, num), cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                           (int)small_smem<V>(bin, num));
-      if (e != cudaSuccess) return e;
-    }
+  for (int bin = BIN_L64; bin <= BIN_M2048; ++bin) {
+    cudaError_t e = cudaFuncSetAttribute(small_kernel<V>(bin, true), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)small_smem<V>(bin, true));
+    if (e != cudaSuccess) return e;
+  }
   return cudaSuccess;
 }
 

@@ -41,6 +41,12 @@ cudaError_t BinLaunch<V>::configure() {
   return bitmap_configure<V>();
 }
 
+template <typename V>
+cudaError_t BinLaunch<V>::launch_general(cudaStream_t st, int grid, const Prob<V>& P, const int* list,
+                                         const int* count, long long N) {
+  return bitmap_launch<V>(BIN_HUGE, st, grid, true, P, list, count, N);
+}
+
 template struct BinLaunch<double>;
 template struct BinLaunch<float>;
 

@@ -43,6 +43,7 @@ struct DevBuf {
 struct Small {
   int counts[16];  // per bin
   int qhead[16];   // per bin: dynamic row-queue heads of the bitmap kernels (counts + 16)
+  int fb[32];      // fallback list: [0] rows, [16] queue head
   int err;
   int range[2];
   int amax;       // longest row of A
@@ -94,7 +95,7 @@ struct spg_ctx {
   int light_max = 256, medium_max = MEDIUM_CAP, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
   // workspace
-  DevBuf f, nz, sp, lists, small, scan_tmp, Pf, splits, canonB[4], iota, ones, crow_tmp;
+  DevBuf f, nz, sp, lists, small, scan_tmp, Pf, splits, canonB[4], iota, ones, crow_tmp, fblist;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
   long long iota_n = -1, ones_n = -1;
@@ -178,6 +179,8 @@ Prob<V> make_prob(spg_handle h, const spg_csr* A, const spg_csr* B, long long* c
   P.rpB = B->row_ptr; P.colB = B->col_idx; P.valB = (const V*)B->vals;
   P.sp = h->sp.as<int>(); P.frow = h->f.as<int>();
   P.row_begin = h->rb; P.crow = crow; P.ccol = ccol; P.cval = (V*)cval;
+  P.fb_list = h->fblist.as<int>();
+  P.fb_count = h->small.as<Small>()->fb;
   P.lgN = 0;
   while (P.lgN < 31 && ((long long)1 << P.lgN) < (long long)B->ncols) ++P.lgN;
   return P;
@@ -198,7 +201,7 @@ spg_status run_bins(spg_handle h, const spg_csr* A, const spg_csr* B, bool numer
   int* lists = h->lists.as<int>();
   const long long Mloc = h->re - h->rb;
   const bool conc = h->concurrent != 0;
-  CK(cudaMemsetAsync(ds->qhead, 0, sizeof(ds->qhead), h->stream));
+  CK(cudaMemsetAsync(ds->qhead, 0, sizeof(ds->qhead) + sizeof(ds->fb), h->stream));
   if (conc) CK(cudaEventRecord(h->ev_fork, h->stream));
   const int order[] = {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY, BIN_M2048, BIN_M1024, BIN_M512, BIN_L256, BIN_L128,
                        BIN_L64, BIN_T32, BIN_T16, BIN_T8, BIN_T4, BIN_SINGLE};
@@ -231,6 +234,13 @@ spg_status run_bins(spg_handle h, const spg_csr* A, const spg_csr* B, bool numer
       CK(cudaStreamWaitEvent(h->stream, h->ev_join[b], 0));
     }
   }
+  if (numeric) {  // rows the light/medium kernels handed over (many runs / clustered columns)
+    const long long grid = (long long)h->max_bpsm[1][BIN_HUGE] * h->sms;
+    const cudaError_t e = BinLaunch<V>::launch_general(h->stream, (int)grid, P, h->fblist.as<int>(), ds->fb,
+                                                       B->ncols);
+    if (e != cudaSuccess) return setf(h, SPG_ERR_CUDA, "fallback kernel launch failed: %s", cudaGetErrorString(e));
+    h->launches++;
+  }
   return SPG_OK;
 }
 
@@ -240,6 +250,7 @@ spg_status ensure_ws(spg_handle h, int M) {
   CK(h->nz.ensure(m));
   CK(h->sp.ensure(m * sizeof(int)));
   CK(h->lists.ensure(m * NUM_BINS * sizeof(int)));
+  CK(h->fblist.ensure(m * sizeof(int)));
   CK(h->small.ensure(sizeof(Small)));
   CK(h->scan_tmp.ensure(scan_tmp_elems((long long)m + 1) * sizeof(long long)));
   return SPG_OK;
@@ -497,7 +508,7 @@ spg_status spg_spgemm_free(spg_handle h) {
     DeviceGuard g(h->device);
     cudaStreamSynchronize(h->stream);
     DevBuf* bufs[] = {&h->f, &h->nz, &h->sp, &h->lists, &h->small, &h->scan_tmp, &h->Pf, &h->splits, &h->iota,
-                      &h->ones, &h->crow_tmp};
+                      &h->ones, &h->crow_tmp, &h->fblist};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
     if (h->canon) spg_spgemm_free(h->canon);

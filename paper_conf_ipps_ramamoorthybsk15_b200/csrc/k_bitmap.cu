@@ -29,6 +29,9 @@ namespace spg {
 constexpr int BMP_CTCAP = 2048;      // 32-product windows per chunk with a precomputed run index
 constexpr int BMP_SLOTS = 8;         // products per lane cached in registers (HEAVY: f <= 8192)
 constexpr int MODE_SYM = 0, MODE_HEAVY = 1, MODE_HUGE = 2;
+#ifndef SPG_HEAVY_SMALL
+#define SPG_HEAVY_SMALL 1  // HEAVY rows (f <= 4096): 512-thread / 112 KB blocks that co-reside
+#endif
 
 __host__ __device__ constexpr int al16(int x) { return (x + 15) & ~15; }
 
@@ -393,12 +396,15 @@ __global__ void __launch_bounds__(BMP_NT, BMP_SMEM > 120 * 1024 ? 1 : 2) k_bitma
 // ================================ launch glue ====================================================
 template <typename V>
 static const void* bitmap_kernel(int bin, bool numeric) {
+  if (bin == BIN_HEAVY && SPG_HEAVY_SMALL)
+    return numeric ? (const void*)k_bitmap<MODE_HEAVY, V, BMP_NT_S, BMP_SMEM_S>
+                   : (const void*)k_bitmap<MODE_SYM, V, BMP_NT_S, BMP_SMEM_S>;
   if (!numeric) return (const void*)k_bitmap<MODE_SYM, V, BMP_NT, BMP_SMEM_L>;
   return bin == BIN_HUGE ? (const void*)k_bitmap<MODE_HUGE, V, BMP_NT, BMP_SMEM_L>
                          : (const void*)k_bitmap<MODE_HEAVY, V, BMP_NT, BMP_SMEM_L>;
 }
-static int bitmap_threads(int) { return BMP_NT; }
-static int bitmap_smem(int) { return BMP_SMEM_L; }
+static int bitmap_threads(int bin) { return bin == BIN_HEAVY && SPG_HEAVY_SMALL ? BMP_NT_S : BMP_NT; }
+static int bitmap_smem(int bin) { return bin == BIN_HEAVY && SPG_HEAVY_SMALL ? BMP_SMEM_S : BMP_SMEM_L; }
 
 template <typename V>
 cudaError_t bitmap_configure() {

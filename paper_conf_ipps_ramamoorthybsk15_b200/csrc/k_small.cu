@@ -176,13 +176,14 @@ template <int CAP, bool NUM, typename V>
 __global__ void __launch_bounds__(LIGHT_WARPS * 32) k_light(Prob<V> P, const int* __restrict__ list,
                                                            const int* __restrict__ count) {
   extern __shared__ __align__(16) char smem[];
-  constexpr int PER = msmem_aligned<V, NUM>(CAP);
+  constexpr int PER = NUM ? esc2_smem_aligned<V, CAP>() : msmem_aligned<V, NUM>(CAP);
   const int warp = threadIdx.x >> 5;
   const Group<32> g{lane_id(), nullptr};
   char* my = smem + warp * PER;
   const int n = *count;
   for (int t = blockIdx.x * LIGHT_WARPS + warp; t < n; t += gridDim.x * LIGHT_WARPS)
-    esc_row<32, CAP, NUM, V>(P, list[t], g, my);
+    if constexpr (NUM) esc2_row<32, CAP, V>(P, list[t], g, my);
+    else esc_row<32, CAP, NUM, V>(P, list[t], g, my);
 }
 
 // ================================ MEDIUM (block merge) ==========================================
@@ -192,7 +193,10 @@ __global__ void __launch_bounds__(NT) k_block(Prob<V> P, const int* __restrict__
   __shared__ int scratch[NT / 32 + 1];
   const Group<NT> g{(int)threadIdx.x, scratch};
   const int n = *count;
-  for (int t = blockIdx.x; t < n; t += gridDim.x) esc_row<NT, CAP, NUM, V>(P, list[t], g, smem);
+  for (int t = blockIdx.x; t < n; t += gridDim.x) {
+    if constexpr (NUM) esc2_row<NT, CAP, V>(P, list[t], g, smem);
+    else esc_row<NT, CAP, NUM, V>(P, list[t], g, smem);
+  }
 }
 
 // ================================ hash-set symbolic (LIGHT, MEDIUM) ==============================
@@ -290,9 +294,14 @@ constexpr int M512_NT = 64;
 template <typename V>
 size_t small_smem(int bin, bool numeric) {
   if (!numeric && bin >= BIN_L64 && bin <= BIN_M2048) return 0;  // hash symbolic: static shared memory
-  const int cap = merge_cap(bin);
-  if (bin >= BIN_L64 && bin <= BIN_L256) return (size_t)LIGHT_WARPS * msmem_aligned<V, true>(cap);
-  if (bin >= BIN_M512 && bin <= BIN_M2048) return msmem_aligned<V, true>(cap);
+  switch (bin) {
+    case BIN_L64: return (size_t)LIGHT_WARPS * esc2_smem_aligned<V, 64>();
+    case BIN_L128: return (size_t)LIGHT_WARPS * esc2_smem_aligned<V, 128>();
+    case BIN_L256: return (size_t)LIGHT_WARPS * esc2_smem_aligned<V, 256>();
+    case BIN_M512: return esc2_smem_aligned<V, 512>();
+    case BIN_M1024: return esc2_smem_aligned<V, 1024>();
+    case BIN_M2048: return esc2_smem_aligned<V, 2048>();
+  }
   return 0;
 }
 

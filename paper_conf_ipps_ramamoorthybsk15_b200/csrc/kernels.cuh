@@ -33,6 +33,8 @@ struct Prob {
   long long* crow;
   int* ccol;
   V* cval;
+  int* fb_list;     // numeric: rows the light/medium kernels hand to the general kernel
+  int* fb_count;    // [0] = rows, [16] = queue head of the general kernel
 };
 
 // analysis.cu
@@ -63,6 +65,9 @@ struct BinLaunch {
   static int rows_per_block(int bin);
   static int max_blocks_per_sm(int bin, bool numeric);
   static cudaError_t configure();  // opt-in dynamic shared memory sizes (once per device)
+  // general (HUGE-tier) kernel over an explicit row list, e.g. the fallback list
+  static cudaError_t launch_general(cudaStream_t st, int grid, const Prob<V>& P, const int* list, const int* count,
+                                    long long N);
 };
 
 }  // namespace spg

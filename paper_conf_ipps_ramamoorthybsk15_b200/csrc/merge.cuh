@@ -385,4 +385,180 @@ __device__ __forceinline__ void esc_row(const Prob<V>& P, const int i, const Gro
   g.sync();
 }
 
+// ESC2 (numeric, LIGHT / MEDIUM): the bucketed ESC of esc_row with ~17 bytes of shared memory
+// per product instead of 28, so twice the rows are in flight per SM.  The runs go to a small
+// table (<= CAP/4 runs); the products are enumerated twice — a histogram pass, then a pass that
+// scatters (key, a*b) straight into its bucket slot (atomicAdd cursor) — so no expand buffer.
+// Rows with more runs or skewed buckets are appended to the fallback list (processed afterwards
+// by the general HUGE-tier kernel) and nothing of them is written here.
+template <int CAP>
+__host__ __device__ constexpr int esc2_rcap() { return CAP / 4; }
+template <typename V, int CAP>
+__host__ __device__ constexpr int esc2_smem() {
+  return CAP * (int)(sizeof(V) + 4) + (CAP / 4 + 1) * 4 + (esc2_rcap<CAP>() + 1) * 4 + esc2_rcap<CAP>() * 4 +
+         esc2_rcap<CAP>() * (int)sizeof(V) + 32;
+}
+template <typename V, int CAP>
+__host__ __device__ constexpr int esc2_smem_aligned() { return (esc2_smem<V, CAP>() + 15) & ~15; }
+
+template <int G, int CAP, typename V>
+__device__ __forceinline__ void esc2_row(const Prob<V>& P, const int i, const Group<G>& g, char* smem) {
+  constexpr int NB = CAP / 4, MAXB = 48, RC = esc2_rcap<CAP>();
+  V* vals = reinterpret_cast<V*>(smem);
+  int* keys = reinterpret_cast<int*>(smem + CAP * sizeof(V));
+  int* cnt = keys + CAP;                 // NB + 1
+  int* seg = cnt + NB + 1;               // RC + 1
+  int* sbs = seg + RC + 1;               // RC
+  V* sa = reinterpret_cast<V*>(reinterpret_cast<uintptr_t>(sbs + RC + 1) & ~(uintptr_t)7);  // RC (8-aligned)
+  const int pa0 = P.rpA[i], pa1 = P.rpA[i + 1];
+  int nr = 0, f = 0;
+  for (int p0 = pa0; p0 < pa1; p0 += G) {
+    const int p = p0 + g.rank;
+    int L = 0, bs = 0;
+    V a = V(0);
+    if (p < pa1) {
+      const int k = P.colA[p];
+      bs = P.rpB[k];
+      L = P.rpB[k + 1] - bs;
+      a = P.valA[p];
+    }
+    int tot;
+    const int ex = g.excl_scan((L << 16) | (L > 0 ? 1 : 0), tot);
+    const int slot = nr + (ex & 0xffff);
+    if (L > 0 && slot < RC) {
+      seg[slot] = f + (ex >> 16);
+      sbs[slot] = bs;
+      sa[slot] = a;
+    }
+    nr += tot & 0xffff;
+    f += tot >> 16;
+  }
+  if (nr > RC) {  // too many runs for the table: general kernel
+    if (g.rank == 0) P.fb_list[atomicAdd(P.fb_count, 1)] = i;
+    g.sync();
+    return;
+  }
+  if (g.rank == 0) seg[nr] = f;
+  const int lgNB = 31 - __clz(NB);
+  const int shift = P.lgN > lgNB ? P.lgN - lgNB : 0;
+  for (int b = g.rank; b <= NB; b += G) cnt[b] = 0;
+  g.sync();
+  // pass A: histogram of bucket sizes (columns only)
+  constexpr int EU = 8;
+  for (int j0 = g.rank; j0 < f; j0 += G * EU) {
+    int q[EU];
+#pragma unroll
+    for (int u = 0; u < EU; ++u) {
+      const int j = j0 + u * G;
+      q[u] = -1;
+      if (j < f) {
+        const int r = upper_idx(seg, nr, j);
+        q[u] = sbs[r] + (j - seg[r]);
+      }
+    }
+    int kk[EU];
+#pragma unroll
+    for (int u = 0; u < EU; ++u) kk[u] = q[u] >= 0 ? P.colB[q[u]] : 0;
+#pragma unroll
+    for (int u = 0; u < EU; ++u)
+      if (q[u] >= 0) atomicAdd(&cnt[kk[u] >> shift], 1);
+  }
+  g.sync();
+  // exclusive scan of the bucket sizes (NB / G contiguous buckets per thread) -> bucket bases
+  constexpr int BPT = NB / G > 0 ? NB / G : 1;
+  int mine = 0, mx = 0;
+  int c8[BPT];
+#pragma unroll
+  for (int k = 0; k < BPT; ++k) {
+    const int b = g.rank * BPT + k;
+    c8[k] = b < NB ? cnt[b] : 0;
+    mine += c8[k];
+    mx = max(mx, c8[k]);
+  }
+  int tot;
+  int run = g.excl_scan(mine, tot);
+  if (g.max(mx) > MAXB) {  // clustered columns: general kernel
+    if (g.rank == 0) P.fb_list[atomicAdd(P.fb_count, 1)] = i;
+    g.sync();
+    return;
+  }
+#pragma unroll
+  for (int k = 0; k < BPT; ++k) {
+    const int b = g.rank * BPT + k;
+    if (b < NB) cnt[b] = run;
+    run += c8[k];
+  }
+  g.sync();
+  // pass B: scatter (key, a*b) into bucket slots; afterwards cnt[b] = end of bucket b
+  for (int j0 = g.rank; j0 < f; j0 += G * EU) {
+    int q[EU], r[EU];
+#pragma unroll
+    for (int u = 0; u < EU; ++u) {
+      const int j = j0 + u * G;
+      q[u] = -1;
+      r[u] = 0;
+      if (j < f) {
+        r[u] = upper_idx(seg, nr, j);
+        q[u] = sbs[r[u]] + (j - seg[r[u]]);
+      }
+    }
+    int kk[EU];
+    V bb[EU];
+#pragma unroll
+    for (int u = 0; u < EU; ++u) {
+      kk[u] = q[u] >= 0 ? P.colB[q[u]] : 0;
+      bb[u] = q[u] >= 0 ? P.valB[q[u]] : V(0);
+    }
+#pragma unroll
+    for (int u = 0; u < EU; ++u)
+      if (q[u] >= 0) {
+        const int d = atomicAdd(&cnt[kk[u] >> shift], 1);
+        keys[d] = kk[u];
+        vals[d] = sa[r[u]] * bb[u];
+      }
+  }
+  g.sync();
+  // sort each of my buckets, count heads, write
+  int heads = 0;
+#pragma unroll
+  for (int k = 0; k < BPT; ++k) {
+    const int b = g.rank * BPT + k;
+    if (b >= NB) break;
+    const int s0 = b ? cnt[b - 1] : 0, s1 = cnt[b];
+    for (int x = s0 + 1; x < s1; ++x) {
+      const int kx = keys[x];
+      const V vx = vals[x];
+      int y = x - 1;
+      while (y >= s0 && keys[y] > kx) {
+        keys[y + 1] = keys[y];
+        vals[y + 1] = vals[y];
+        --y;
+      }
+      keys[y + 1] = kx;
+      vals[y + 1] = vx;
+    }
+    for (int x = s0; x < s1; ++x) heads += (x == s0 || keys[x - 1] != keys[x]);
+  }
+  int htot;
+  int pos = g.excl_scan(heads, htot);
+  const long long rowoff = P.crow[i - P.row_begin];
+#pragma unroll
+  for (int k = 0; k < BPT; ++k) {
+    const int b = g.rank * BPT + k;
+    if (b >= NB) break;
+    const int s0 = b ? cnt[b - 1] : 0, s1 = cnt[b];
+    for (int x = s0; x < s1;) {
+      const int kx = keys[x];
+      V s = vals[x];
+      int y = x + 1;
+      for (; y < s1 && keys[y] == kx; ++y) s += vals[y];
+      P.ccol[rowoff + pos] = kx;
+      P.cval[rowoff + pos] = s;
+      ++pos;
+      x = y;
+    }
+  }
+  g.sync();
+}
+
 }  // namespace spg

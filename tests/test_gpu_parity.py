@@ -343,3 +343,32 @@ def test_nccl_single_rank_broadcast_allgatherv():
         compare(A, B, (full.row_ptr.cpu().numpy(), full.col_idx.cpu().numpy(), full.vals.cpu().numpy()))
     finally:
         spg.spg_spgemm_free(h)
+
+
+# ---- light/medium kernels hand rows to the general kernel: many runs, clustered columns -----
+def test_fallback_many_short_runs():
+    """f ~ 100-1500 made of one-product runs: more runs than the ESC2 run table holds."""
+    rng = np.random.default_rng(21)
+    K, N = 5000, 200000
+    B = W.random_csr(K, N, 1.0 / N, 22, values="int")          # ~1 entry per B row
+    A = W.random_csr(400, K, 0.0, 23, values="int")
+    rows, cols = [], []
+    for i in range(A.nrows):
+        n = int(rng.integers(40, 1500))
+        rows += [i] * n
+        cols += list(rng.choice(K, n, replace=False))
+    D = np.zeros((A.nrows, K), np.float64)
+    D[rows, cols] = rng.integers(1, 5, len(rows))
+    A = dense_to_csr(D)
+    compare(A, B, run_gpu(A, B), exact_values=True)
+
+
+def test_fallback_clustered_columns():
+    """All products of a row land in a narrow column range of a wide matrix: skewed buckets."""
+    rng = np.random.default_rng(31)
+    K, N = 300, 1 << 20
+    rp = np.arange(0, K * 40 + 1, 40, dtype=np.int32)
+    col = np.concatenate([np.sort(rng.choice(256, 40, replace=False)) for _ in range(K)]).astype(np.int32)
+    B = W.CSR(K, N, rp, col, rng.integers(1, 5, K * 40).astype(np.float64))
+    A = W.random_csr(200, K, 0.05, 32, values="int")
+    compare(A, B, run_gpu(A, B), exact_values=True)

@@ -43,6 +43,8 @@ def parse():
     p.add_argument("--profile", action="store_true", help="short run for ncu (no baselines, no clocks)")
     p.add_argument("--opt", action="append", default=[], help="library option name=value")
     p.add_argument("--out", default=None, help="also append the JSON line to this file")
+    p.add_argument("--sim-ranks-on-one-gpu", dest="virtual", action="store_true",
+                   help="N>1 on one GPU for testing: gloo process group, virtual-rank handles (no NCCL)")
     return p.parse_args()
 
 
@@ -202,10 +204,16 @@ def run_ours(args):
     import paper_conf_ipps_ramamoorthybsk15_b200 as spg
 
     ws, rank, local = dist_env()
+    if args.virtual:
+        local = 0
     torch.cuda.set_device(local)
     if ws > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.virtual:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    cdev = torch.device("cpu") if args.virtual else torch.device("cuda", local)  # collective tensors
     dev = torch.device("cuda", local)
     A, B = W.make(args.config)
     same = B is A
@@ -214,7 +222,9 @@ def run_ours(args):
     dA = spg.DeviceCSR.from_host(A, dev)
     dB = dA if same else spg.DeviceCSR.from_host(B, dev)
     stream = torch.cuda.current_stream()
-    if ws > 1:
+    if ws > 1 and args.virtual:
+        h = spg.spg_create_dist(local, stream, vdt, None, rank, ws)   # partitioned rows, no communicator
+    elif ws > 1:
         obj = [spg.spg_get_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         h = spg.spg_create_dist(local, stream, vdt, obj[0], rank, ws)
@@ -274,7 +284,7 @@ def run_ours(args):
     tot_ms = float(sym.sum() + num.sum())
     st = spg.spg_get_stats(h)
     if ws > 1:
-        t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
+        t = torch.tensor([tot_ms], dtype=torch.float64, device=cdev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         tot_ms = float(t.item())
     ms_step = tot_ms / K
@@ -319,7 +329,7 @@ def run_ours(args):
         spg.spg_spgemm_free(h2)
         e_ms = float(np.mean(times[1:])) * 1e3
         if ws > 1:
-            t = torch.tensor([e_ms], dtype=torch.float64, device=dev)
+            t = torch.tensor([e_ms], dtype=torch.float64, device=cdev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e_ms = float(t.item())
         h2d = csr_bytes(Ah.nrows, Ah.nnz, vb) + (0 if Bp is Ap else csr_bytes(B.nrows, B.nnz, vb))
@@ -351,7 +361,8 @@ def run_ours(args):
             "config": {"workload": args.config, "rows": A.nrows, "nnzA": A.nnz, "nnzB": B.nnz, "flops": F_total,
                        "nnzC": int(st["nnz_c"]) if ws == 1 else None,
                        "l2": "flushed between timed steps (256 MiB memset)" if not args.no_flush else "not flushed",
-                       "parallelism": f"rows flop-partitioned over {ws} GPU(s)" if ws > 1 else "1 GPU",
+                       "parallelism": (f"rows flop-partitioned over {ws} GPU(s)" + (" (virtual ranks on one GPU)"
+                                       if args.virtual else "")) if ws > 1 else "1 GPU",
                        "options": args.opt},
             "phases": {"symbolic_ms": float(np.mean(sym)), "numeric_ms": num_ms,
                        "numeric_gflops": 2.0 * int(st["flops"]) / (num_ms * 1e-3) / 1e9,

@@ -401,6 +401,18 @@ __host__ __device__ constexpr int esc2_smem() {
 template <typename V, int CAP>
 __host__ __device__ constexpr int esc2_smem_aligned() { return (esc2_smem<V, CAP>() + 15) & ~15; }
 
+// Run of product j for a window of 32 consecutive products starting at jw (warp-uniform): one
+// binary search for the window, then each lane's run = first run + popcount of the run starts
+// inside the window at or below it (REDUX.OR bitmask).  All 32 lanes must call.
+__device__ __forceinline__ int window_run(const int* seg, int nr, int jw) {
+  const int lane = lane_id();
+  const int rb = upper_idx(seg, nr, jw);
+  const int rs = rb + 1 + lane;
+  const int d = rs <= nr ? seg[rs] - jw : 32;
+  const unsigned M = __reduce_or_sync(FULL, (d >= 1 && d <= 31) ? (1u << d) : 0u);
+  return rb + __popc(M & ((2u << lane) - 1u));
+}
+
 template <int G, int CAP, typename V>
 __device__ __forceinline__ void esc2_row(const Prob<V>& P, const int i, const Group<G>& g, char* smem) {
   constexpr int NB = CAP / 4, MAXB = 48, RC = esc2_rcap<CAP>();
@@ -445,15 +457,16 @@ __device__ __forceinline__ void esc2_row(const Prob<V>& P, const int i, const Gr
   g.sync();
   // pass A: histogram of bucket sizes (columns only)
   constexpr int EU = 8;
-  for (int j0 = g.rank; j0 < f; j0 += G * EU) {
+  const int lane = lane_id(), wbase = g.rank - lane;  // windows of 32 consecutive products per warp
+  for (int j0 = wbase; j0 < f; j0 += G * EU) {
     int q[EU];
 #pragma unroll
     for (int u = 0; u < EU; ++u) {
-      const int j = j0 + u * G;
+      const int jw = j0 + u * G, j = jw + lane;
       q[u] = -1;
-      if (j < f) {
-        const int r = upper_idx(seg, nr, j);
-        q[u] = sbs[r] + (j - seg[r]);
+      if (jw < f) {
+        const int r = G >= 128 ? window_run(seg, nr, jw) : upper_idx(seg, nr, min(j, f - 1));
+        if (j < f) q[u] = sbs[r] + (j - seg[r]);
       }
     }
     int kk[EU];
@@ -490,16 +503,16 @@ __device__ __forceinline__ void esc2_row(const Prob<V>& P, const int i, const Gr
   }
   g.sync();
   // pass B: scatter (key, a*b) into bucket slots; afterwards cnt[b] = end of bucket b
-  for (int j0 = g.rank; j0 < f; j0 += G * EU) {
+  for (int j0 = wbase; j0 < f; j0 += G * EU) {
     int q[EU], r[EU];
 #pragma unroll
     for (int u = 0; u < EU; ++u) {
-      const int j = j0 + u * G;
+      const int jw = j0 + u * G, j = jw + lane;
       q[u] = -1;
       r[u] = 0;
-      if (j < f) {
-        r[u] = upper_idx(seg, nr, j);
-        q[u] = sbs[r[u]] + (j - seg[r[u]]);
+      if (jw < f) {
+        r[u] = G >= 128 ? window_run(seg, nr, jw) : upper_idx(seg, nr, min(j, f - 1));
+        if (j < f) q[u] = sbs[r[u]] + (j - seg[r[u]]);
       }
     }
     int kk[EU];

@@ -15,23 +15,24 @@ template <typename V> int bitmap_occupancy(int, bool);
 template <typename V>
 cudaError_t bitmap_launch(int, cudaStream_t, int, bool, const Prob<V>&, const int*, const int*, long long);
 
-static bool is_bitmap(int bin) { return bin_is_bitmap(bin); }
+// HEAVY rows (f <= 4096) take the ESC2 kernel for numeric, the bitmap tier for symbolic
+static bool is_bitmap(int bin, bool numeric) { return bin_is_bitmap(bin) && !(numeric && bin == BIN_HEAVY); }
 
 template <typename V>
 cudaError_t BinLaunch<V>::launch(int bin, cudaStream_t st, int grid, bool numeric, const Prob<V>& P, const int* list,
                                  const int* count, long long N) {
-  if (is_bitmap(bin)) return bitmap_launch<V>(bin, st, grid, numeric, P, list, count, N);
+  if (is_bitmap(bin, numeric)) return bitmap_launch<V>(bin, st, grid, numeric, P, list, count, N);
   return small_launch<V>(bin, st, grid, numeric, P, list, count);
 }
 
 template <typename V>
 int BinLaunch<V>::rows_per_block(int bin) {
-  return is_bitmap(bin) ? 1 : small_rows_per_block<V>(bin);
+  return bin_is_bitmap(bin) ? 1 : small_rows_per_block<V>(bin);
 }
 
 template <typename V>
 int BinLaunch<V>::max_blocks_per_sm(int bin, bool numeric) {
-  return is_bitmap(bin) ? bitmap_occupancy<V>(bin, numeric) : small_occupancy<V>(bin, numeric);
+  return is_bitmap(bin, numeric) ? bitmap_occupancy<V>(bin, numeric) : small_occupancy<V>(bin, numeric);
 }
 
 template <typename V>

@@ -295,6 +295,7 @@ template <typename V>
 size_t small_smem(int bin, bool numeric) {
   if (!numeric && bin >= BIN_L64 && bin <= BIN_M2048) return 0;  // hash symbolic: static shared memory
   switch (bin) {
+    case BIN_HEAVY: return esc2_smem_aligned<V, HEAVY1_CAP>();  // numeric HEAVY through ESC2
     case BIN_L64: return (size_t)LIGHT_WARPS * esc2_smem_aligned<V, 64>();
     case BIN_L128: return (size_t)LIGHT_WARPS * esc2_smem_aligned<V, 128>();
     case BIN_L256: return (size_t)LIGHT_WARPS * esc2_smem_aligned<V, 256>();
@@ -307,7 +308,7 @@ size_t small_smem(int bin, bool numeric) {
 
 template <typename V>
 int small_threads(int bin) {
-  return bin == BIN_M512 ? M512_NT : bin == BIN_M1024 ? MED1_NT : bin == BIN_M2048 ? MEDIUM_NT
+  return bin == BIN_M512 ? M512_NT : bin == BIN_M1024 ? MED1_NT : (bin == BIN_M2048 || bin == BIN_HEAVY) ? MEDIUM_NT
        : (bin >= BIN_L64 && bin <= BIN_L256) ? LIGHT_WARPS * 32 : 256;
 }
 
@@ -341,13 +342,15 @@ static const void* small_kernel(int bin, bool numeric) {
       return numeric ? (const void*)k_block<MED1_NT, 1024, true, V> : (const void*)k_hsym_block<V, MED1_NT, 2048>;
     case BIN_M2048:
       return numeric ? (const void*)k_block<MEDIUM_NT, 2048, true, V> : (const void*)k_hsym_block<V, MEDIUM_NT, 4096>;
+    case BIN_HEAVY:  // numeric only (symbolic HEAVY runs on the bitmap tier)
+      return (const void*)k_block<MEDIUM_NT, HEAVY1_CAP, true, V>;
   }
   return nullptr;
 }
 
 template <typename V>
 cudaError_t small_configure() {
-  for (int bin = BIN_L64; bin <= BIN_M2048; ++bin) {
+  for (int bin : {BIN_L64, BIN_L128, BIN_L256, BIN_M512, BIN_M1024, BIN_M2048, BIN_HEAVY}) {
     cudaError_t e = cudaFuncSetAttribute(small_kernel<V>(bin, true), cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)small_smem<V>(bin, true));
     if (e != cudaSuccess) return e;

@@ -413,6 +413,18 @@ __device__ __forceinline__ int window_run(const int* seg, int nr, int jw) {
   return rb + __popc(M & ((2u << lane) - 1u));
 }
 
+// Run of product jw + lane for a window starting inside run rb (warp-uniform); advances rb to
+// the run holding jw + 32.  All 32 lanes must call.
+__device__ __forceinline__ int esc2_walk(const int* seg, int nr, int jw, int& rb) {
+  const int lane = lane_id();
+  const int rs = rb + 1 + lane;
+  const int d = rs <= nr ? seg[rs] - jw : 64;
+  const unsigned M = __reduce_or_sync(FULL, (d >= 1 && d <= 31) ? (1u << d) : 0u);
+  const int r = rb + __popc(M & ((2u << lane) - 1u));
+  rb += __popc(M) + (__ballot_sync(FULL, d == 32) != 0u);
+  return r;
+}
+
 template <int G, int CAP, typename V>
 __device__ __forceinline__ void esc2_row(const Prob<V>& P, const int i, const Group<G>& g, char* smem) {
   constexpr int NB = CAP / 4, MAXB = 48, RC = esc2_rcap<CAP>();
@@ -455,18 +467,25 @@ __device__ __forceinline__ void esc2_row(const Prob<V>& P, const int i, const Gr
   const int shift = P.lgN > lgNB ? P.lgN - lgNB : 0;
   for (int b = g.rank; b <= NB; b += G) cnt[b] = 0;
   g.sync();
+  // Each warp enumerates one contiguous chunk of products in windows of 32; the run of every
+  // lane comes from the run-start bitmask of the window (REDUX.OR), and the first run of the
+  // next window from the current one (no search after the first window).
+  constexpr int EU = 8, NW = G / 32;
+  const int lane = lane_id(), w = g.rank >> 5;
+  const int chunk = (f + NW * 32 - 1) / (NW * 32) * 32;
+  const int jbeg = min(f, w * chunk), jend = min(f, jbeg + chunk);
+  const int rb0 = jbeg < jend ? upper_idx(seg, nr, jbeg) : 0;
   // pass A: histogram of bucket sizes (columns only)
-  constexpr int EU = 8;
-  const int lane = lane_id(), wbase = g.rank - lane;  // windows of 32 consecutive products per warp
-  for (int j0 = wbase; j0 < f; j0 += G * EU) {
+  int rb = rb0;
+  for (int j0 = jbeg; j0 < jend; j0 += 32 * EU) {
     int q[EU];
 #pragma unroll
     for (int u = 0; u < EU; ++u) {
-      const int jw = j0 + u * G, j = jw + lane;
+      const int jw = j0 + u * 32, j = jw + lane;
       q[u] = -1;
-      if (jw < f) {
-        const int r = G >= 128 ? window_run(seg, nr, jw) : upper_idx(seg, nr, min(j, f - 1));
-        if (j < f) q[u] = sbs[r] + (j - seg[r]);
+      if (jw < jend) {
+        const int r = esc2_walk(seg, nr, jw, rb);
+        if (j < jend) q[u] = sbs[r] + (j - seg[r]);
       }
     }
     int kk[EU];
@@ -503,16 +522,17 @@ __device__ __forceinline__ void esc2_row(const Prob<V>& P, const int i, const Gr
   }
   g.sync();
   // pass B: scatter (key, a*b) into bucket slots; afterwards cnt[b] = end of bucket b
-  for (int j0 = wbase; j0 < f; j0 += G * EU) {
+  rb = rb0;
+  for (int j0 = jbeg; j0 < jend; j0 += 32 * EU) {
     int q[EU], r[EU];
 #pragma unroll
     for (int u = 0; u < EU; ++u) {
-      const int jw = j0 + u * G, j = jw + lane;
+      const int jw = j0 + u * 32, j = jw + lane;
       q[u] = -1;
       r[u] = 0;
-      if (jw < f) {
-        r[u] = G >= 128 ? window_run(seg, nr, jw) : upper_idx(seg, nr, min(j, f - 1));
-        if (j < f) q[u] = sbs[r[u]] + (j - seg[r[u]]);
+      if (jw < jend) {
+        r[u] = esc2_walk(seg, nr, jw, rb);
+        if (j < jend) q[u] = sbs[r[u]] + (j - seg[r[u]]);
       }
     }
     int kk[EU];
@@ -531,45 +551,56 @@ __device__ __forceinline__ void esc2_row(const Prob<V>& P, const int i, const Gr
       }
   }
   g.sync();
-  // sort each of my buckets, count heads, write
-  int heads = 0;
-#pragma unroll
-  for (int k = 0; k < BPT; ++k) {
-    const int b = g.rank * BPT + k;
-    if (b >= NB) break;
-    const int s0 = b ? cnt[b - 1] : 0, s1 = cnt[b];
-    for (int x = s0 + 1; x < s1; ++x) {
-      const int kx = keys[x];
-      const V vx = vals[x];
-      int y = x - 1;
-      while (y >= s0 && keys[y] > kx) {
-        keys[y + 1] = keys[y];
-        vals[y + 1] = vals[y];
-        --y;
-      }
-      keys[y + 1] = kx;
-      vals[y + 1] = vx;
-    }
-    for (int x = s0; x < s1; ++x) heads += (x == s0 || keys[x - 1] != keys[x]);
+  // Per product x in bucket b: x is the head of its column if no earlier slot of b holds the
+  // same column (later duplicates get the sign bit); hc[b] counts the distinct columns of b.
+  int* hc = sbs;  // the run table is dead after pass B
+  for (int b = g.rank; b < NB; b += G) hc[b] = 0;
+  g.sync();
+  for (int x = g.rank; x < f; x += G) {
+    const int kx = keys[x], b = kx >> shift;
+    const int s0 = b ? cnt[b - 1] : 0;
+    bool head = true;
+    for (int y = s0; y < x; ++y)
+      if ((keys[y] & 0x7fffffff) == kx) { head = false; break; }
+    if (head) atomicAdd(&hc[b], 1);
+    else keys[x] = kx | int(0x80000000);
   }
-  int htot;
-  int pos = g.excl_scan(heads, htot);
-  const long long rowoff = P.crow[i - P.row_begin];
+  g.sync();
+  {  // bucket output bases (same contiguous ownership as the size scan)
+    int h8[BPT], hm = 0;
 #pragma unroll
-  for (int k = 0; k < BPT; ++k) {
-    const int b = g.rank * BPT + k;
-    if (b >= NB) break;
-    const int s0 = b ? cnt[b - 1] : 0, s1 = cnt[b];
-    for (int x = s0; x < s1;) {
-      const int kx = keys[x];
-      V s = vals[x];
-      int y = x + 1;
-      for (; y < s1 && keys[y] == kx; ++y) s += vals[y];
-      P.ccol[rowoff + pos] = kx;
-      P.cval[rowoff + pos] = s;
-      ++pos;
-      x = y;
+    for (int k = 0; k < BPT; ++k) {
+      const int b = g.rank * BPT + k;
+      h8[k] = b < NB ? hc[b] : 0;
+      hm += h8[k];
     }
+    int ht;
+    int hr = g.excl_scan(hm, ht);
+#pragma unroll
+    for (int k = 0; k < BPT; ++k) {
+      const int b = g.rank * BPT + k;
+      if (b < NB) hc[b] = hr;
+      hr += h8[k];
+    }
+  }
+  g.sync();
+  // each head: output slot = bucket base + number of distinct smaller columns in the bucket;
+  // value = sum of its column's products in slot order
+  const long long rowoff = P.crow[i - P.row_begin];
+  for (int x = g.rank; x < f; x += G) {
+    const int kx = keys[x];
+    if (kx < 0) continue;
+    const int b = kx >> shift;
+    const int s0 = b ? cnt[b - 1] : 0, s1 = cnt[b];
+    int u = 0;
+    V s = V(0);
+    for (int y = s0; y < s1; ++y) {
+      const int ky = keys[y];
+      u += (ky >= 0 && ky < kx);
+      if ((ky & 0x7fffffff) == kx) s += vals[y];
+    }
+    P.ccol[rowoff + hc[b] + u] = kx;
+    P.cval[rowoff + hc[b] + u] = s;
   }
   g.sync();
 }

@@ -25,8 +25,9 @@
  *
  * Ownership and threading
  *   - The caller owns A, B and C.  The handle owns all workspace (row flops, class lists,
- *     dense accumulators, the NCCL communicator) and caches the symbolic analysis that
- *     spg_spgemm_numeric consumes.  spg_spgemm_free releases everything.
+ *     the per-product rank array R of 4 bytes per intermediate product, the NCCL
+ *     communicator) and caches the symbolic analysis that spg_spgemm_numeric consumes.
+ *     spg_spgemm_free releases everything.
  *   - A handle is bound to one device and one CUDA stream and is not thread-safe;
  *     several handles may coexist.
  *   - All work is stream-ordered on the handle's stream.  spg_spgemm_symbolic blocks the
@@ -78,31 +79,35 @@ typedef struct {
 } spg_csr;
 
 /* Row classes (PAPER.md L104 logical reordering A = [A_H; A_L]).
- * f_i = number of intermediate products of row i. */
+ * f_i = number of intermediate products of row i.  The heavy/light threshold t of the paper
+ * (Phase I) is SPG_OPT_LIGHT_MAX_FLOPS: rows with f_i <= t are "light"
+ * (TINY / LIGHT / MEDIUM, one shared kernel that sorts whole tiles of rows per thread block),
+ * the rest "heavy" (one thread block and a shared-memory column bitmap per row). */
 typedef enum {
-  SPG_CLASS_EMPTY = 0,  /* f_i = 0: no work, c_i = 0                                        */
-  SPG_CLASS_SINGLE = 1, /* exactly one non-empty B row referenced: scaled copy, c_i = f_i   */
-  SPG_CLASS_TINY = 2,   /* f_i <= 32: one warp, register bitonic sort                       */
-  SPG_CLASS_LIGHT = 3,  /* f_i <= LIGHT_MAX_FLOPS: one warp, shared-memory run merge        */
-  SPG_CLASS_MEDIUM = 4, /* f_i <= MEDIUM_MAX_FLOPS: 256-thread block, shared-memory merge   */
-  SPG_CLASS_HEAVY = 5,  /* f_i <= HEAVY_MAX_FLOPS: 512-thread block, shared-memory merge    */
-  SPG_CLASS_HUGE = 6,   /* larger: 1024-thread block, dense accumulator + touched bitmap    */
+  SPG_CLASS_EMPTY = 0,  /* f_i = 0: no work, c_i = 0                                         */
+  SPG_CLASS_SINGLE = 1, /* exactly one non-empty B row referenced: scaled copy, c_i = f_i    */
+  SPG_CLASS_TINY = 2,   /* light, f_i <= 32                                                  */
+  SPG_CLASS_LIGHT = 3,  /* light, 32 < f_i <= 256                                            */
+  SPG_CLASS_MEDIUM = 4, /* light, 256 < f_i <= LIGHT_MAX_FLOPS                               */
+  SPG_CLASS_HEAVY = 5,  /* heavy, f_i <= HEAVY_MAX_FLOPS: products cached in registers       */
+  SPG_CLASS_HUGE = 6,   /* heavy, larger: products re-gathered per pass                      */
   SPG_NUM_CLASSES = 7
 } spg_row_class;
 
 typedef enum {
-  SPG_OPT_LIGHT_MAX_FLOPS = 0,  /* heavy/light threshold t: 32..256, default 256 */
-  SPG_OPT_MEDIUM_MAX_FLOPS = 1, /* default 2048 (max 2048)                                      */
-  SPG_OPT_HEAVY_MAX_FLOPS = 2,  /* default 8192 (max 8192); rows above go to the HUGE tier     */
-  SPG_OPT_FORCE_CLASS = 3,      /* -1 (default) or a class id c >= TINY: every non-empty row
-                                   runs on class max(natural, c) and the SINGLE shortcut is
-                                   off — the threshold extremes of PAPER.md L233              */
+  SPG_OPT_LIGHT_MAX_FLOPS = 0,  /* heavy/light threshold t: 0..3072-TILE_FLOPS,
+                                   default 1024; 0 sends every non-SINGLE row to the heavy path */
+  SPG_OPT_TILE_FLOPS = 1,       /* nominal products per light tile, default 2048               */
+  SPG_OPT_HEAVY_MAX_FLOPS = 2,  /* 0..8192, default 8192; heavy rows above are HUGE            */
+  SPG_OPT_FORCE_CLASS = 3,      /* -1 (default) or a class id c >= TINY: the SINGLE shortcut is
+                                   off, and c >= HEAVY sends every non-empty row to the heavy
+                                   path (HUGE: uncached) — the threshold extremes of PAPER.md L233 */
   SPG_OPT_VALIDATE = 4,         /* 1: check CSR indices/order on the device (extra sync)      */
   SPG_OPT_INPUT_CANONICAL = 5,  /* 1 (default): caller promises B rows strictly ascending;
                                    0: the library canonicalises a copy of B                   */
   SPG_OPT_TIMING = 6,           /* 1: record per-phase CUDA-event times into the stats        */
-  SPG_OPT_HUGE_SLOTS = 7,       /* max concurrent dense accumulators (0 = one per SM)         */
-  SPG_OPT_CONCURRENT = 8        /* 1 (default): class kernels on concurrent streams           */
+  SPG_OPT_HUGE_SLOTS = 7,       /* max concurrent heavy-row blocks per bin (0 = full occupancy) */
+  SPG_OPT_CONCURRENT = 8        /* 1 (default): light and heavy kernels on concurrent streams  */
 } spg_option;
 
 typedef struct {
@@ -115,11 +120,15 @@ typedef struct {
   int64_t class_flops[SPG_NUM_CLASSES];   /* products per class (this rank)              */
   int64_t bin_hist[65];                   /* rows with f = 0 (index 0) and with
                                              ceil(log2 f) = b (index b + 1), all rows    */
+  int64_t tiles;                          /* light tiles of the last symbolic call       */
+  int64_t fallback_rows;                  /* light rows moved to the heavy path (clustered
+                                             columns)                                    */
+  int64_t rank_bytes;                     /* bytes of the per-product rank array R       */
   float ms_analysis;                      /* SPG_OPT_TIMING: row analysis + classify     */
-  float ms_symbolic;                      /*   symbolic class kernels + row_ptr scan     */
-  float ms_numeric;                       /*   numeric class kernels (last numeric call) */
-  float ms_class_numeric[SPG_NUM_CLASSES];/*   per-class numeric kernel time (serialised
-                                               when SPG_OPT_CONCURRENT = 0)               */
+  float ms_symbolic;                      /*   symbolic kernels + row_ptr scan            */
+  float ms_numeric;                       /*   numeric (last numeric call)                */
+  float ms_light;                         /*   symbolic light-tile kernel                 */
+  float ms_heavy;                         /*   symbolic heavy-row kernels                 */
   int32_t launches_symbolic;              /* kernels launched by the last symbolic call  */
   int32_t launches_numeric;               /* kernels launched by the last numeric call   */
 } spg_stats;
@@ -144,7 +153,8 @@ const char* spg_version(void);
 spg_status spg_spgemm_symbolic(spg_handle h, const spg_csr* A, const spg_csr* B, int64_t* C_row_ptr,
                                int64_t* nnzC, int32_t* row_begin, int32_t* row_end);
 
-/* Numeric phase + in-row sort/compaction (fused).  Requires a preceding symbolic call on
+/* Numeric phase: every product is scattered into its output slot, found by symbolic (the rank
+ * of its column within its row of C), so C comes out sorted and compacted.  Requires a preceding symbolic call on
  * this handle with the same A/B structure pointers.  C_col_idx: device int32[nnzC];
  * C_vals: device fp32/fp64[nnzC].  Values of A and B may differ from the symbolic call
  * (re-run numeric on new values with the same structure).  Asynchronous. */

@@ -11,50 +11,66 @@
 
 namespace spg {
 
-// f_i = sum over stored A(i,k) of len_B(k); nz_i = #entries with len_B(k) > 0 (capped at 2);
-// sp_i = index of one entry with len_B > 0 (the only one when nz_i = 1).  One block owns ROWS
-// consecutive rows; its threads stride over the rows' A entries (coalesced), find the owning
-// row by binary search in the cached row_ptr tile, pre-reduce per warp and row, and add into
-// shared 32-bit accumulators.
+// f_i = sum over stored A(i,k) of len_B(k); nz_i = #entries with len_B(k) > 0 (capped at 2, plus
+// bits 6/7 for A rows longer than one 512- / 1024-thread bitmap chunk).  Per A entry e of row i:
+// rowA[e] = i and Pe[e] = sum of len_B over the entries of row i before e (the entry's first
+// product within the row — the numeric kernel's index into R).  One block owns ROWS consecutive
+// rows; its threads stride over the rows' A entries (coalesced), find the owning row by binary
+// search in the cached row_ptr tile, pre-reduce per warp and row, and add into shared 32-bit
+// accumulators.  Pe comes from a block scan of len_B (wrapping 32-bit arithmetic: the in-row
+// value itself is < 2^31, or the row is reported as overflowing).
 template <int ROWS>
 __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict__ rpA, const int* __restrict__ colA,
                                                     int K, const int* __restrict__ rpB, int* __restrict__ f_out,
-                                                    uint8_t* __restrict__ nz_out, int* __restrict__ sp_out,
-                                                    unsigned long long* __restrict__ hist, int* __restrict__ err,
-                                                    int* __restrict__ amax) {
+                                                    uint8_t* __restrict__ nz_out, int* __restrict__ rowA,
+                                                    int* __restrict__ Pe, unsigned long long* __restrict__ hist,
+                                                    int* __restrict__ err, int* __restrict__ amax) {
+  constexpr int NW = ROWS / 32;
   __shared__ int s_rp[ROWS + 1];
   __shared__ unsigned s_f[ROWS];
   __shared__ int s_nz[ROWS];
-  __shared__ int s_sp[ROWS];
+  __shared__ unsigned s_base[ROWS];
+  __shared__ unsigned s_ws[NW + 1];
   __shared__ unsigned s_hist[65];
   __shared__ int s_amax;
-  const int t = threadIdx.x, lane = t & 31;
+  const int t = threadIdx.x, lane = t & 31, w = t >> 5;
   const int r0 = blockIdx.x * ROWS;
   const int nr = min(ROWS, M - r0);
   if (t <= nr) s_rp[t] = rpA[r0 + t];
   if (t == 0 && nr == ROWS) s_rp[ROWS] = rpA[r0 + ROWS];
   s_f[t] = 0;
   s_nz[t] = 0;
-  s_sp[t] = -1;
   if (t < 65) s_hist[t] = 0;
   if (t == 0) s_amax = 0;
   __syncthreads();
   const int e0 = s_rp[0], e1 = s_rp[nr];
   int bad = 0;
+  unsigned carry = 0;  // wrapping prefix of len_B over this block's entries
   for (int base = e0; base < e1; base += ROWS) {  // uniform trip count: warp collectives below
     const int e = base + t;
     bool act = e < e1;
     int L = 0, r = -1;
     if (act) {
       const int k = colA[e];
-      if ((unsigned)k >= (unsigned)K) {
-        bad |= 1;
-      } else {
-        L = rpB[k + 1] - rpB[k];
-        r = upper_idx(s_rp, nr, e);
-      }
+      r = upper_idx(s_rp, nr, e);
+      if ((unsigned)k >= (unsigned)K) bad |= 1;
+      else L = rpB[k + 1] - rpB[k];
     }
     act = r >= 0;
+    // block exclusive scan of L -> S (wrapping); rows starting in this chunk record their base
+    const unsigned incl = warp_incl_scan((unsigned)L);
+    if (lane == 31) s_ws[w] = incl;
+    __syncthreads();
+    if (w == 0) {
+      const unsigned x = lane < NW ? s_ws[lane] : 0u;
+      const unsigned xi = warp_incl_scan(x);
+      if (lane < NW) s_ws[lane] = xi - x;
+      if (lane == NW - 1) s_ws[NW] = xi;
+    }
+    __syncthreads();
+    const unsigned S = carry + incl - (unsigned)L + s_ws[w];
+    if (act && e == s_rp[r]) s_base[r] = S;
+    carry += s_ws[NW];
     const unsigned nzb = __ballot_sync(FULL, act && L > 0);
     const unsigned grp = __match_any_sync(FULL, r);
     if (act) {
@@ -70,7 +86,11 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
         }
         atomicAdd(&s_nz[r], __popc(grp & nzb));
       }
-      if (L > 0) s_sp[r] = e;
+    }
+    __syncthreads();
+    if (act) {
+      rowA[e] = r0 + r;
+      Pe[e] = (int)(S - s_base[r]);
     }
   }
   __syncthreads();
@@ -79,13 +99,12 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
     if (f > (unsigned)INT_MAX) f = INT_MAX;
     f_out[r0 + t] = (int)f;
     // bits 6/7: the A row has more entries than a 512- / 1024-thread bitmap block gathers in one
-    // chunk (HEAVY kernels cache single-chunk rows' products in registers; longer rows move up)
+    // chunk (register-cached HEAVY kernels need single-chunk rows; longer rows move up)
     const int alen = s_rp[t + 1] - s_rp[t];
     nz_out[r0 + t] = (uint8_t)(min(s_nz[t], 2) | (alen > BMP_NT_S ? 0x40 : 0) | (alen > BMP_NT ? 0x80 : 0));
-    sp_out[r0 + t] = s_sp[t];
     const int b = f == 0 ? 0 : 1 + (f == 1 ? 0 : 32 - __clz((int)f - 1));
     atomicAdd(&s_hist[b], 1u);
-    atomicMax(&s_amax, s_rp[t + 1] - s_rp[t]);
+    atomicMax(&s_amax, alen);
   }
   if (bad) atomicOr(err, bad);
   __syncthreads();
@@ -93,103 +112,139 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
   if (t == 0) atomicMax(amax, s_amax);
 }
 
-__device__ __forceinline__ int classify_bin(int f, int nz, const ClassParams& p) {
-  if (f == 0) return -1;
+// Row path.  Returns the class (CLS_*) and, through `bin`, the bitmap bin (-1: none).
+__device__ __forceinline__ int classify_row(int f, int nz, const ClassParams& p, int& bin, bool& light) {
+  bin = -1;
+  light = false;
+  if (f == 0) return CLS_EMPTY;
   const bool long1 = nz & 0x40, long2 = nz & 0x80;
   nz &= 0x3f;
-  if (p.force < 0 && nz == 1 && p.single_ok) return BIN_SINGLE;
-  int b;
-  if (f <= 4) b = BIN_T4;
-  else if (f <= 8) b = BIN_T8;
-  else if (f <= 16) b = BIN_T16;
-  else if (f <= TINY_MAX) b = BIN_T32;
-  else if (f <= p.light_max) b = f <= 64 ? BIN_L64 : (f <= 128 ? BIN_L128 : BIN_L256);
-  else if (f <= p.medium_max) b = f <= 512 ? BIN_M512 : (f <= 1024 ? BIN_M1024 : BIN_M2048);
-  else if (f <= p.heavy_max) b = f <= HEAVY1_CAP ? BIN_HEAVY : BIN_HEAVY2;
-  else b = BIN_HUGE;
-  if (p.force > CLS_TINY) {  // forced class: smallest bin of that class at least
-    const int fb = class_first_bin(p.force);
-    if (fb > b) b = fb;
+  if (p.force < 0 && nz == 1 && p.single_ok) return CLS_SINGLE;
+  if (f <= p.light_max && p.force < CLS_HEAVY) {
+    light = true;
+    return f <= TINY_MAX ? CLS_TINY : (f <= LIGHTC_MAX ? CLS_LIGHT : CLS_MEDIUM);
   }
-  if (b == BIN_HEAVY && long1) b = BIN_HEAVY2;
-  if (b == BIN_HEAVY2 && long2) b = BIN_HUGE;
-  return b;
+  const int hm = min(p.heavy_max, HEAVY_CAP);
+  if (p.force == CLS_HUGE || f > hm) bin = BIN_HUGE;
+  else if (f <= HEAVY1_CAP && !long1) bin = BIN_HEAVY;
+  else if (!long2) bin = BIN_HEAVY2;
+  else bin = BIN_HUGE;
+  return bin == BIN_HUGE ? CLS_HUGE : CLS_HEAVY;
 }
 
-// Classify this rank's rows [rb, re): append every row with work to its bin list, write c_i for
-// rows whose nnz(C) needs no work (EMPTY: 0; SINGLE: f_i, B canonical), accumulate per-class
-// statistics.  List positions come from shared counters (warp-aggregated) and ONE global
-// atomic per bin per 2048-row tile; statistics are flushed per tile.
-constexpr int CL_NT = 256, CL_IPT = 8, CL_TILE = CL_NT * CL_IPT;
+// Classify this rank's rows [rb, re) (local index li = i - rb): cls[li] = class | light-path bit;
+// fl[li] = f_i for light rows (scanned into the light-product prefix PL); heavy rows are
+// appended to their bitmap bin's list and get R offsets (relative to the end of the light
+// region) from one 64-bit atomic per warp; c_i is written for rows needing no symbolic work
+// (EMPTY: 0; SINGLE: f_i — B canonical, one run).  Per-class statistics are pre-reduced per
+// warp (MATCH.ANY + REDUX, 16-bit halves) and flushed once per block.
+constexpr int CL_NT = 256;
 
-__global__ void __launch_bounds__(CL_NT) k_classify(const int* __restrict__ f, const uint8_t* __restrict__ nz,
-                                                    int rb, int re, ClassParams prm, BinLists lists,
-                                                    int* __restrict__ counts,
-                                                    unsigned long long* __restrict__ cstats /* [2*NUM_CLS+2] */,
+__global__ void __launch_bounds__(CL_NT) k_classify(const int* __restrict__ f, const uint8_t* __restrict__ nz, int rb,
+                                                    int re, ClassParams prm, uint8_t* __restrict__ cls,
+                                                    int* __restrict__ fl, long long* __restrict__ Ro,
+                                                    HeavyLists lists, Small* __restrict__ sm,
                                                     long long* __restrict__ crow) {
-  __shared__ int s_cnt[NUM_BINS], s_base[NUM_BINS];
   __shared__ unsigned s_rows[NUM_CLS], s_flo[NUM_CLS], s_fhi[NUM_CLS], s_fmax;
   const int tid = threadIdx.x, lane = tid & 31;
-  if (tid < NUM_BINS) s_cnt[tid] = 0;
   if (tid < NUM_CLS) { s_rows[tid] = 0; s_flo[tid] = 0; s_fhi[tid] = 0; }
   if (tid == 0) s_fmax = 0;
   __syncthreads();
   const long long n = (long long)re - rb;
-  for (long long tile = (long long)blockIdx.x * CL_TILE; tile < n; tile += (long long)gridDim.x * CL_TILE) {
-    int mybin[CL_IPT], mypos[CL_IPT];
-#pragma unroll
-    for (int it = 0; it < CL_IPT; ++it) {
-      const long long li = tile + it * CL_NT + tid;
-      const bool act = li < n;
-      int fi = 0, bin = -1, cls = -1;
-      if (act) {
-        fi = f[rb + li];
-        bin = classify_bin(fi, nz[rb + li], prm);
-        cls = bin < 0 ? CLS_EMPTY : bin_class(bin);
-        if (bin < 0) crow[li + 1] = 0;
-        else if (bin == BIN_SINGLE) crow[li + 1] = fi;
+  const long long nup = (n + 31) & ~31LL;  // warp-uniform trip count
+  for (long long li = (long long)blockIdx.x * CL_NT + tid; li < nup; li += (long long)gridDim.x * CL_NT) {
+    const bool act = li < n;
+    int fi = 0, bin = -1, c = -1;
+    bool light = false;
+    if (act) {
+      fi = f[rb + li];
+      c = classify_row(fi, nz[rb + li], prm, bin, light);
+      cls[li] = (uint8_t)(c | (light ? CLS_LIGHT_PATH : 0));
+      fl[li] = light ? fi : 0;
+      if (c == CLS_EMPTY) crow[li + 1] = 0;
+      else if (c == CLS_SINGLE) crow[li + 1] = fi;
+      if (bin < 0) Ro[li] = -1;
+    }
+    const unsigned gc = __match_any_sync(FULL, c);
+    if (act) {
+      const unsigned lo = __reduce_add_sync(gc, (unsigned)fi & 0xffffu);
+      const unsigned hi = __reduce_add_sync(gc, (unsigned)fi >> 16);
+      if (lane == __ffs(gc) - 1) {
+        atomicAdd(&s_rows[c], (unsigned)__popc(gc));
+        atomicAdd(&s_flo[c], lo);
+        atomicAdd(&s_fhi[c], hi);
       }
-      const unsigned gc = __match_any_sync(FULL, cls);
-      if (act) {
-        const unsigned lo = __reduce_add_sync(gc, (unsigned)fi & 0xffffu);
-        const unsigned hi = __reduce_add_sync(gc, (unsigned)fi >> 16);
-        if (lane == __ffs(gc) - 1) {
-          atomicAdd(&s_rows[cls], (unsigned)__popc(gc));
-          atomicAdd(&s_flo[cls], lo);
-          atomicAdd(&s_fhi[cls], hi);
-        }
-      }
-      const unsigned fm = __reduce_max_sync(FULL, (unsigned)fi);
-      if (lane == 0 && fm) atomicMax(&s_fmax, fm);
+    }
+    const unsigned fm = __reduce_max_sync(FULL, (unsigned)fi);
+    if (lane == 0 && fm) atomicMax(&s_fmax, fm);
+    // heavy rows: list append + R offset (rare: one warp-level scan and atomic when present)
+    if (__ballot_sync(FULL, bin >= 0)) {
+      const long long hv = bin >= 0 ? fi : 0;
+      const long long incl = warp_incl_scan(hv);
+      unsigned long long hb = 0;
+      if (lane == 31) hb = atomicAdd(reinterpret_cast<unsigned long long*>(&sm->heavy_total), (unsigned long long)incl);
+      hb = __shfl_sync(FULL, hb, 31);
       const unsigned gb = __match_any_sync(FULL, bin);
-      int pos = 0;
       if (bin >= 0) {
+        Ro[li] = (long long)hb + incl - hv;
         const int leader = __ffs(gb) - 1;
-        if (lane == leader) pos = atomicAdd(&s_cnt[bin], __popc(gb));
+        int pos = 0;
+        if (lane == leader) pos = atomicAdd(&sm->counts[bin], __popc(gb));
         pos = __shfl_sync(gb, pos, leader) + __popc(gb & lanemask_lt());
+        lists.rows[bin][pos] = (int)li;
       }
-      mybin[it] = bin;
-      mypos[it] = pos;
     }
-    __syncthreads();
-    if (tid < NUM_BINS) {
-      const int c = s_cnt[tid];
-      s_base[tid] = c ? atomicAdd(&counts[tid], c) : 0;
-      s_cnt[tid] = 0;
-    }
-    if (tid < NUM_CLS) {
-      const unsigned long long fl = ((unsigned long long)s_fhi[tid] << 16) + s_flo[tid];
-      if (s_rows[tid]) atomicAdd(&cstats[tid], (unsigned long long)s_rows[tid]);
-      if (fl) atomicAdd(&cstats[NUM_CLS + tid], fl);
-      s_rows[tid] = 0; s_flo[tid] = 0; s_fhi[tid] = 0;
-    }
-    __syncthreads();
-#pragma unroll
-    for (int it = 0; it < CL_IPT; ++it)
-      if (mybin[it] >= 0) lists.rows[mybin[it]][s_base[mybin[it]] + mypos[it]] = rb + (int)(tile + it * CL_NT + tid);
-    __syncthreads();
   }
-  if (tid == 0 && s_fmax) atomicMax(&cstats[2 * NUM_CLS], (unsigned long long)s_fmax);
+  __syncthreads();
+  if (tid < NUM_CLS) {
+    const unsigned long long fl2 = ((unsigned long long)s_fhi[tid] << 16) + s_flo[tid];
+    if (s_rows[tid]) atomicAdd(&sm->cstats[tid], (unsigned long long)s_rows[tid]);
+    if (fl2) atomicAdd(&sm->cstats[NUM_CLS + tid], fl2);
+  }
+  if (tid == 0 && s_fmax) atomicMax(&sm->cstats[2 * NUM_CLS], (unsigned long long)s_fmax);
+}
+
+// Tiles of light rows.  PL = exclusive prefix of fl (light products, row order).  A light row
+// starts a tile when its product range [PL_i, PL_i + f_i) contains a multiple of `cap` (so a
+// tile holds < cap + light_max products).  Light rows get Ro = PL_i, heavy rows Ro += F_L.
+// r_ok = (F_L + F_H <= capacity of R): the symbolic kernels do nothing when R is too small and
+// the host re-runs them after growing R.
+__global__ void __launch_bounds__(256) k_tiles(const int* __restrict__ f, int rb, int re, int cap,
+                                               const uint8_t* __restrict__ cls, const long long* __restrict__ PL,
+                                               long long* __restrict__ Ro, uint8_t* __restrict__ tflag,
+                                               int* __restrict__ tiles, Small* __restrict__ sm, long long r_cap) {
+  const long long n = (long long)re - rb;
+  const long long FL = PL[n];
+  const int lane = threadIdx.x & 31;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    const long long fr = FL + sm->heavy_total;
+    sm->fr = fr;
+    sm->r_ok = fr <= r_cap ? 1 : 0;
+  }
+  const long long nup = (n + 31) & ~31LL;
+  for (long long li = (long long)blockIdx.x * blockDim.x + threadIdx.x; li < nup;
+       li += (long long)gridDim.x * blockDim.x) {
+    bool start = false;
+    if (li < n) {
+      const int c = cls[li];
+      if (c & CLS_LIGHT_PATH) {
+        const long long pl = PL[li];
+        const long long fi = f[rb + li];
+        Ro[li] = pl;
+        start = (pl % cap == 0) || (pl / cap != (pl + fi - 1) / cap);
+      } else if ((c & 7) == CLS_HEAVY || (c & 7) == CLS_HUGE) {
+        Ro[li] += FL;
+      }
+      tflag[li] = start ? 1 : 0;
+    }
+    const unsigned m = __ballot_sync(FULL, start);
+    if (m) {
+      int base = 0;
+      if (lane == 0) base = atomicAdd(&sm->ntiles, __popc(m));
+      base = __shfl_sync(FULL, base, 0);
+      if (start) tiles[base + __popc(m & lanemask_lt())] = (int)li;
+    }
+  }
 }
 
 // ---- inclusive scan to int64 (three passes: tile scan, tile-sum scan, add) -------------------
@@ -327,21 +382,32 @@ __global__ void k_narrow(const long long* __restrict__ in, int* __restrict__ out
 
 // ---- host launchers ------------------------------------------------------------------------
 cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB,
-                             int* f, uint8_t* nz, int* sp, unsigned long long* hist, int* err, int* amax) {
+                             int* f, uint8_t* nz, int* rowA, int* Pe, unsigned long long* hist, int* err, int* amax) {
   if (M <= 0) return cudaSuccess;
   constexpr int ROWS = 256;
-  k_row_flops<ROWS><<<(M + ROWS - 1) / ROWS, ROWS, 0, st>>>(M, rpA, colA, K, rpB, f, nz, sp, hist, err, amax);
+  k_row_flops<ROWS><<<(M + ROWS - 1) / ROWS, ROWS, 0, st>>>(M, rpA, colA, K, rpB, f, nz, rowA, Pe, hist, err, amax);
   return cudaGetLastError();
 }
 
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
-                            const ClassParams& prm, const BinLists& lists, int* counts, unsigned long long* cstats,
-                            long long* crow) {
+                            const ClassParams& prm, uint8_t* cls, int* fl, long long* Ro, const HeavyLists& lists,
+                            Small* small, long long* crow) {
   const long long n = (long long)re - rb;
   if (n <= 0) return cudaSuccess;
-  long long blocks = (n + CL_TILE - 1) / CL_TILE;
-  if (blocks > (long long)sms * 4) blocks = (long long)sms * 4;
-  k_classify<<<(int)blocks, CL_NT, 0, st>>>(f, nz, rb, re, prm, lists, counts, cstats, crow);
+  long long blocks = (n + CL_NT - 1) / CL_NT;
+  if (blocks > (long long)sms * 8) blocks = (long long)sms * 8;
+  k_classify<<<(int)blocks, CL_NT, 0, st>>>(f, nz, rb, re, prm, cls, fl, Ro, lists, small, crow);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tiles(cudaStream_t st, int sms, const int* f, int rb, int re, int tile_cap, const uint8_t* cls,
+                         const long long* PL, long long* Ro, uint8_t* tflag, int* tiles, Small* small,
+                         long long r_cap) {
+  const long long n = (long long)re - rb;
+  long long blocks = (n + 255) / 256;
+  if (blocks > (long long)sms * 8) blocks = (long long)sms * 8;
+  if (blocks < 1) blocks = 1;
+  k_tiles<<<(int)blocks, 256, 0, st>>>(f, rb, re, tile_cap, cls, PL, Ro, tflag, tiles, small, r_cap);
   return cudaGetLastError();
 }
 

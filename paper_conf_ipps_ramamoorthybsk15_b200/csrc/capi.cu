@@ -39,18 +39,6 @@ struct DevBuf {
   T* as() const { return reinterpret_cast<T*>(p); }
 };
 
-// Small per-call device scratch (zeroed at the start of every symbolic call).
-struct Small {
-  int counts[16];  // per bin
-  int qhead[16];   // per bin: dynamic row-queue heads of the bitmap kernels (counts + 16)
-  int fb[32];      // fallback list: [0] rows, [16] queue head
-  int err;
-  int range[2];
-  int amax;       // longest row of A
-  unsigned long long hist[65];
-  unsigned long long cstats[2 * NUM_CLS + 2];
-};
-
 struct HostRead {  // pinned readback area
   Small small;
   long long nnz;
@@ -77,11 +65,6 @@ struct DeviceGuard {
   }
 };
 
-const char* class_name(int c) {
-  static const char* n[] = {"empty", "single", "tiny", "light", "medium", "heavy", "huge"};
-  return (c >= 0 && c < NUM_CLS) ? n[c] : "?";
-}
-
 }  // namespace
 
 struct spg_ctx {
@@ -92,20 +75,20 @@ struct spg_ctx {
   int rank = 0, nranks = 1;
   ncclComm_t comm = nullptr;
   // options
-  int light_max = 256, medium_max = MEDIUM_CAP, heavy_max = HEAVY_CAP, force = -1;
+  int light_max = LIGHT_MAX_DEFAULT, tile_cap = TILE_CAP_DEFAULT, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
-  // workspace
-  DevBuf f, nz, sp, lists, small, scan_tmp, Pf, splits, canonB[4], iota, ones, crow_tmp, fblist;
+  // workspace: analysis (all rows / all A entries), classification (this rank's rows), R, windows
+  DevBuf f, nz, rowA, Pe, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, R, wrow, Pf, splits,
+      canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
   long long iota_n = -1, ones_n = -1;
   HostRead* hr = nullptr;
-  cudaStream_t aux[NUM_BINS] = {};
-  cudaEvent_t ev_fork = nullptr, ev_join[NUM_BINS] = {};
+  cudaStream_t aux[4] = {};
+  cudaEvent_t ev_fork = nullptr, ev_join[4] = {};
   cudaEvent_t ev_t[8] = {};
-  cudaEvent_t ev_c0[NUM_BINS] = {}, ev_c1[NUM_BINS] = {};
-  bool bin_timed[NUM_BINS] = {};
-  int max_bpsm[2][NUM_BINS] = {};
+  cudaEvent_t ev_p[4] = {};  // light path start/end, heavy path start/end
+  int occ_light = 1, occ_heavy[NUM_BINS] = {};
   // cached symbolic state
   bool sym_ok = false;
   SymKey key{};
@@ -113,7 +96,7 @@ struct spg_ctx {
   int64_t nnzC = 0;
   int counts[NUM_BINS] = {};
   spg_stats stats{};
-  bool num_timed = false;
+  bool num_timed = false, paths_timed = false;
   int launches = 0;  // kernels launched by the current phase
   // host (end-to-end) path buffers
   DevBuf hbuf[9];
@@ -172,83 +155,92 @@ SymKey make_key(const spg_csr* A, const spg_csr* B) {
   return k;
 }
 
-template <typename V>
-Prob<V> make_prob(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow, int* ccol, void* cval) {
-  Prob<V> P;
-  P.rpA = A->row_ptr; P.colA = A->col_idx; P.valA = (const V*)A->vals;
-  P.rpB = B->row_ptr; P.colB = B->col_idx; P.valB = (const V*)B->vals;
-  P.sp = h->sp.as<int>(); P.frow = h->f.as<int>();
-  P.row_begin = h->rb; P.crow = crow; P.ccol = ccol; P.cval = (V*)cval;
-  P.fb_list = h->fblist.as<int>();
-  P.fb_count = h->small.as<Small>()->fb;
-  P.lgN = 0;
-  while (P.lgN < 31 && ((long long)1 << P.lgN) < (long long)B->ncols) ++P.lgN;
+int ceil_log2(long long n) {
+  int l = 0;
+  while (l < 31 && ((long long)1 << l) < n) ++l;
+  return l;
+}
+
+SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
+  SymProb P;
+  P.rpA = A->row_ptr; P.colA = A->col_idx; P.rpB = B->row_ptr; P.colB = B->col_idx;
+  P.frow = h->f.as<int>();
+  P.cls = h->cls.as<uint8_t>();
+  P.Ro = h->Ro.as<long long>();
+  P.R = h->R.as<unsigned>();
+  P.crow = crow;
+  P.r_ok = &h->small.as<Small>()->r_ok;
+  P.row_begin = h->rb;
+  P.row_end = h->re;
+  P.lgN = ceil_log2(B->ncols);
   return P;
 }
 
-// Launch every bin's kernel for one phase.  Symbolic: bin sizes are not known on the host, so
-// each bin gets a full-occupancy persistent grid that exits at once when its list is empty.
-// Numeric: sizes known from the symbolic readback; empty bins are skipped.  Bins run on their
-// own streams (forked from / joined to the handle stream) so light and heavy rows overlap —
-// the paper's concurrent CPU and GPU legs of Phases II/III recast as
-// concurrent kernels on one GPU.
-template <typename V>
-spg_status run_bins(spg_handle h, const spg_csr* A, const spg_csr* B, bool numeric, long long* crow, int* ccol,
-                    void* cval) {
-  Prob<V> P = make_prob<V>(h, A, B, crow, ccol, cval);
+// Symbolic class kernels: light tiles and the heavy bitmap bins on concurrent streams (the
+// paper's concurrent CPU and GPU legs of Phases II/III, recast as
+// concurrent kernels on one GPU), then the rows the light kernel handed over.  Bin sizes are
+// device-side: every kernel is a persistent grid that exits at once when its list is empty.
+spg_status run_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
+  const SymProb P = make_sym(h, A, B, crow);
   Small* ds = h->small.as<Small>();
-  const int* cnt = ds->counts;
-  int* lists = h->lists.as<int>();
-  const long long Mloc = h->re - h->rb;
   const bool conc = h->concurrent != 0;
   CK(cudaMemsetAsync(ds->qhead, 0, sizeof(ds->qhead) + sizeof(ds->fb), h->stream));
   if (conc) CK(cudaEventRecord(h->ev_fork, h->stream));
-  const int order[] = {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY, BIN_M2048, BIN_M1024, BIN_M512, BIN_L256, BIN_L128,
-                       BIN_L64, BIN_T32, BIN_T16, BIN_T8, BIN_T4, BIN_SINGLE};
-  for (int b : order) {
-    if (b == BIN_SINGLE && !numeric) continue;  // c_i = f_i written by classify
-    if (numeric && h->counts[b] == 0) continue;
-    cudaStream_t st = conc ? h->aux[b] : h->stream;
+  const bool tm = h->timing != 0;
+  // light tiles
+  {
+    cudaStream_t st = conc ? h->aux[0] : h->stream;
     if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
-    const int* list = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
-    const int rpb = BinLaunch<V>::rows_per_block(b);
-    long long grid = (long long)h->max_bpsm[numeric][b] * h->sms;
-    if (bin_is_bitmap(b) && h->huge_slots_opt > 0 && h->huge_slots_opt < grid)
-      grid = h->huge_slots_opt;
-    if (numeric) {
-      const long long need = (h->counts[b] + rpb - 1) / rpb;
-      if (need < grid) grid = need;
-    }
-    if (grid < 1) grid = 1;
-    const bool tm = numeric && h->timing;
-    if (tm) CK(cudaEventRecord(h->ev_c0[b], st));
-    const cudaError_t e = BinLaunch<V>::launch(b, st, (int)grid, numeric, P, list, cnt + b, B->ncols);
-    if (e != cudaSuccess)
-      return setf(h, SPG_ERR_CUDA, "%s bin %d %s kernel launch failed: %s", class_name(bin_class(b)), b,
-                  numeric ? "numeric" : "symbolic", cudaGetErrorString(e));
+    if (tm) CK(cudaEventRecord(h->ev_p[0], st));
+    CK(launch_light_rank(st, h->occ_light * h->sms, P, h->tiles.as<int>(), &ds->ntiles, h->tflag.as<uint8_t>(),
+                         h->PL.as<long long>(), h->fblist.as<int>(), ds->fb));
     h->launches++;
-    if (tm) CK(cudaEventRecord(h->ev_c1[b], st));
-    h->bin_timed[b] = tm;
+    if (tm) CK(cudaEventRecord(h->ev_p[1], st));
     if (conc) {
-      CK(cudaEventRecord(h->ev_join[b], st));
-      CK(cudaStreamWaitEvent(h->stream, h->ev_join[b], 0));
+      CK(cudaEventRecord(h->ev_join[0], st));
+      CK(cudaStreamWaitEvent(h->stream, h->ev_join[0], 0));
     }
   }
-  if (numeric) {  // rows the light/medium kernels handed over (many runs / clustered columns)
-    const long long grid = (long long)h->max_bpsm[1][BIN_HUGE] * h->sms;
-    const cudaError_t e = BinLaunch<V>::launch_general(h->stream, (int)grid, P, h->fblist.as<int>(), ds->fb,
-                                                       B->ncols);
-    if (e != cudaSuccess) return setf(h, SPG_ERR_CUDA, "fallback kernel launch failed: %s", cudaGetErrorString(e));
-    h->launches++;
+  // heavy bins
+  {
+    cudaStream_t st = conc ? h->aux[1] : h->stream;
+    if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
+    if (tm) CK(cudaEventRecord(h->ev_p[2], st));
+    const long long Mloc = h->re - h->rb;
+    for (int b : {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY}) {
+      long long grid = (long long)h->occ_heavy[b] * h->sms;
+      if (h->huge_slots_opt > 0 && h->huge_slots_opt < grid) grid = h->huge_slots_opt;
+      const int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
+      CK(launch_heavy_rank(b, st, (int)grid, P, list, ds->counts + b, B->ncols));
+      h->launches++;
+    }
+    if (tm) CK(cudaEventRecord(h->ev_p[3], st));
+    if (conc) {
+      CK(cudaEventRecord(h->ev_join[1], st));
+      CK(cudaStreamWaitEvent(h->stream, h->ev_join[1], 0));
+    }
   }
+  h->paths_timed = tm;
+  // rows with clustered columns, handed over by the light kernel
+  long long grid = (long long)h->occ_heavy[BIN_HUGE] * h->sms;
+  CK(launch_heavy_rank(BIN_HUGE, h->stream, (int)grid, P, h->fblist.as<int>(), ds->fb, B->ncols));
+  h->launches++;
   return SPG_OK;
 }
 
-spg_status ensure_ws(spg_handle h, int M) {
+spg_status ensure_ws(spg_handle h, int M, long long nnzA) {
   size_t m = (size_t)(M > 0 ? M : 1);
+  size_t na = (size_t)(nnzA > 0 ? nnzA : 1);
   CK(h->f.ensure(m * sizeof(int)));
   CK(h->nz.ensure(m));
-  CK(h->sp.ensure(m * sizeof(int)));
+  CK(h->rowA.ensure(na * sizeof(int)));
+  CK(h->Pe.ensure(na * sizeof(int)));
+  CK(h->cls.ensure(m));
+  CK(h->fl.ensure(m * sizeof(int)));
+  CK(h->Ro.ensure(m * sizeof(long long)));
+  CK(h->PL.ensure((m + 1) * sizeof(long long)));
+  CK(h->tflag.ensure(m));
+  CK(h->tiles.ensure(m * sizeof(int)));
   CK(h->lists.ensure(m * NUM_BINS * sizeof(int)));
   CK(h->fblist.ensure(m * sizeof(int)));
   CK(h->small.ensure(sizeof(Small)));
@@ -256,12 +248,12 @@ spg_status ensure_ws(spg_handle h, int M) {
   return SPG_OK;
 }
 
-// Row analysis over all rows (f_i, non-empty-run flag, log2 histogram).
+// Row analysis over all rows (f_i, run flags, log2 histogram, per-entry row and offset).
 spg_status analysis(spg_handle h, const spg_csr* A, const spg_csr* B) {
   Small* ds = h->small.as<Small>();
   CK(cudaMemsetAsync(ds, 0, sizeof(Small), h->stream));
   CK(launch_row_flops(h->stream, A->nrows, A->row_ptr, A->col_idx, B->nrows, B->row_ptr, h->f.as<int>(),
-                      h->nz.as<uint8_t>(), h->sp.as<int>(), ds->hist, &ds->err, &ds->amax));
+                      h->nz.as<uint8_t>(), h->rowA.as<int>(), h->Pe.as<int>(), ds->hist, &ds->err, &ds->amax));
   h->launches += A->nrows > 0;
   return SPG_OK;
 }
@@ -287,8 +279,8 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
 // SPG_OPT_INPUT_CANONICAL = 0: B' = canonical B (rows sorted, duplicates summed), computed by
 // this library's own SpGEMM as A' x B'' with A' = pattern of B with unit values (columns =
 // positions 0..nnzB-1) and B'' = one row per stored entry of B — every stored entry becomes a
-// one-product run, so the row merge / bitmap kernels sort and add them.  values_only: reuse the
-// structure of the last call and recompute the values (numeric on new B values).
+// one-product run, so the symbolic kernels sort them and numeric adds them.  values_only: reuse
+// the structure of the last call and recompute the values (numeric on new B values).
 template <typename V>
 spg_status canonicalize(spg_handle h, const spg_csr* B, bool values_only) {
   const long long nnzB = B->nnz;
@@ -345,52 +337,69 @@ spg_status validate_device(spg_handle h, const spg_csr* A, const spg_csr* B) {
   return SPG_OK;
 }
 
-template <typename V>
+// a2 + symbolic classes: after analysis / classification (this rank's rows), the light and heavy
+// kernels compute R and c_i; scan of c_i -> C_row_ptr; one readback of nnz(C) and the stats.
 spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64_t* C_row_ptr, int64_t* nnzC,
                          int32_t* row_begin, int32_t* row_end) {
   const int M = A->nrows;
-  spg_status s = ensure_ws(h, M);
+  spg_status s = ensure_ws(h, M, A->nnz);
   if (s != SPG_OK) return s;
   h->launches = 0;
   if (h->validate && (s = validate_device(h, A, B)) != SPG_OK) return s;
   h->sym_ok = false;
   h->host_sym_ok = false;
-  if (h->timing) CK(cudaEventRecord(h->ev_t[0], h->stream));
-  if ((s = analysis(h, A, B)) != SPG_OK) return s;
   long long F_total = -1;
-  if (h->nranks > 1) {
-    if ((s = split_points(h, M, h->nranks)) != SPG_OK) return s;
-    h->rb = h->hr->splits[h->rank];
-    h->re = h->hr->splits[h->rank + 1];
-    F_total = h->hr->nnz;
-  } else {
-    h->rb = 0;
-    h->re = M;
-    h->hr->splits[0] = 0;
-    h->hr->splits[1] = M;
-  }
-  const long long Mloc = h->re - h->rb;
+  long long Mloc = 0;
   Small* ds = h->small.as<Small>();
-  ClassParams prm{h->light_max, h->medium_max, h->heavy_max, h->force, h->canonical ? 1 : 0};
-  BinLists L;
-  int* lists = h->lists.as<int>();
-  for (int b = 0; b < NUM_BINS; ++b) L.rows[b] = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
   long long* crow = reinterpret_cast<long long*>(C_row_ptr);
-  CK(cudaMemsetAsync(crow, 0, sizeof(long long), h->stream));
-  CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm, L, ds->counts,
-                     ds->cstats, crow));
-  h->launches += Mloc > 0;
-  if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));
-  if ((s = run_bins<V>(h, A, B, false, crow, nullptr, nullptr)) != SPG_OK) return s;
-  CK(launch_incl_scan<long long>(h->stream, crow + 1, crow + 1, Mloc, h->scan_tmp.as<long long>()));
-  h->launches += scan_launches(Mloc);
-  if (h->timing) CK(cudaEventRecord(h->ev_t[2], h->stream));
-  CK(cudaMemcpyAsync(&h->hr->small, ds, sizeof(Small), cudaMemcpyDeviceToHost, h->stream));
-  CK(cudaMemcpyAsync(&h->hr->nnz, crow + Mloc, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
-  CK(cudaStreamSynchronize(h->stream));
+  // Two attempts at most: the first call (or a larger product count) finds R too small — the
+  // kernels then skip their work, R is grown to the exact size read back, and the pass reruns.
+  for (int attempt = 0;; ++attempt) {
+    h->launches = 0;
+    if (h->timing) CK(cudaEventRecord(h->ev_t[0], h->stream));
+    if ((s = analysis(h, A, B)) != SPG_OK) return s;
+    if (h->nranks > 1) {
+      if ((s = split_points(h, M, h->nranks)) != SPG_OK) return s;
+      h->rb = h->hr->splits[h->rank];
+      h->re = h->hr->splits[h->rank + 1];
+      F_total = h->hr->nnz;
+    } else {
+      h->rb = 0;
+      h->re = M;
+      h->hr->splits[0] = 0;
+      h->hr->splits[1] = M;
+    }
+    Mloc = h->re - h->rb;
+    ClassParams prm{h->light_max, h->heavy_max, h->tile_cap, h->force, h->canonical ? 1 : 0};
+    int* lists = h->lists.as<int>();
+    HeavyLists L3;
+    for (int b = 0; b < NUM_BINS; ++b) L3.rows[b] = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
+    long long* PL = h->PL.as<long long>();
+    CK(cudaMemsetAsync(crow, 0, sizeof(long long), h->stream));
+    CK(cudaMemsetAsync(PL, 0, sizeof(long long), h->stream));
+    CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm,
+                       h->cls.as<uint8_t>(), h->fl.as<int>(), h->Ro.as<long long>(), L3, ds, crow));
+    CK(launch_incl_scan<int>(h->stream, h->fl.as<int>(), PL + 1, Mloc, h->scan_tmp.as<long long>()));
+    const long long r_cap = h->R.p ? (long long)(h->R.cap / sizeof(unsigned)) : 0;
+    CK(launch_tiles(h->stream, h->sms, h->f.as<int>(), h->rb, h->re, h->tile_cap, h->cls.as<uint8_t>(), PL,
+                    h->Ro.as<long long>(), h->tflag.as<uint8_t>(), h->tiles.as<int>(), ds, r_cap));
+    h->launches += (Mloc > 0) + scan_launches(Mloc) + 1;
+    if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));
+    if ((s = run_sym(h, A, B, crow)) != SPG_OK) return s;
+    CK(launch_incl_scan<long long>(h->stream, crow + 1, crow + 1, Mloc, h->scan_tmp.as<long long>()));
+    h->launches += scan_launches(Mloc);
+    if (h->timing) CK(cudaEventRecord(h->ev_t[2], h->stream));
+    CK(cudaMemcpyAsync(&h->hr->small, ds, sizeof(Small), cudaMemcpyDeviceToHost, h->stream));
+    CK(cudaMemcpyAsync(&h->hr->nnz, crow + Mloc, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
+    CK(cudaStreamSynchronize(h->stream));
+    const Small& hs = h->hr->small;
+    if (hs.err & 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "A has a column index outside [0, B.nrows)");
+    if (hs.err & 2) return setf(h, SPG_ERR_INDEX_OVERFLOW, "a row of A has >= 2^31 intermediate products");
+    if (hs.r_ok || attempt > 0) break;
+    CK(h->R.ensure((size_t)(hs.fr > 0 ? hs.fr : 1) * sizeof(unsigned)));
+  }
   const Small& hs = h->hr->small;
-  if (hs.err & 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "A has a column index outside [0, B.nrows)");
-  if (hs.err & 2) return setf(h, SPG_ERR_INDEX_OVERFLOW, "a row of A has >= 2^31 intermediate products");
+  if (!hs.r_ok && hs.fr > 0) return setf(h, SPG_ERR_OUT_OF_MEMORY, "rank array could not be sized");
   h->nnzC = h->hr->nnz;
   for (int b = 0; b < NUM_BINS; ++b) h->counts[b] = hs.counts[b];
   spg_stats& st = h->stats;
@@ -407,10 +416,17 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     st.class_flops[c] = (int64_t)hs.cstats[NUM_CLS + c];
   }
   for (int b = 0; b < 65; ++b) st.bin_hist[b] = (int64_t)hs.hist[b];
+  st.tiles = hs.ntiles;
+  st.fallback_rows = hs.fb[0];
+  st.rank_bytes = (int64_t)hs.fr * (int64_t)sizeof(unsigned);
   st.launches_symbolic = h->launches;
   if (h->timing) {
     cudaEventElapsedTime(&st.ms_analysis, h->ev_t[0], h->ev_t[1]);
     cudaEventElapsedTime(&st.ms_symbolic, h->ev_t[1], h->ev_t[2]);
+    if (h->paths_timed) {
+      cudaEventElapsedTime(&st.ms_light, h->ev_p[0], h->ev_p[1]);
+      cudaEventElapsedTime(&st.ms_heavy, h->ev_p[2], h->ev_p[3]);
+    }
   }
   h->key = make_key(A, B);
   h->sym_ok = true;
@@ -426,8 +442,22 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
                         void* C_val) {
   if (h->timing) CK(cudaEventRecord(h->ev_t[3], h->stream));
   h->launches = 0;
-  spg_status s = run_bins<V>(h, A, B, true, (long long*)C_row_ptr, C_col, C_val);
-  if (s != SPG_OK) return s;
+  const long long nwin = (h->nnzC + NUM_W - 1) / NUM_W;
+  if (nwin > INT_MAX) return setf(h, SPG_ERR_NOT_SUPPORTED, "nnz(C) too large for one rank (%lld windows)", nwin);
+  if (nwin > 0) {
+    CK(h->wrow.ensure((size_t)nwin * sizeof(int)));
+    const int mloc = h->re - h->rb;
+    CK(launch_window_rows(h->stream, (const long long*)C_row_ptr, mloc, h->wrow.as<int>(), (int)nwin));
+    NumProb<V> P;
+    P.rpA = A->row_ptr; P.colA = A->col_idx; P.valA = (const V*)A->vals;
+    P.rpB = B->row_ptr; P.colB = B->col_idx; P.valB = (const V*)B->vals;
+    P.rowA = h->rowA.as<int>(); P.Pe = h->Pe.as<int>(); P.Ro = h->Ro.as<long long>();
+    P.R = h->R.as<unsigned>(); P.crow = (const long long*)C_row_ptr; P.wrow = h->wrow.as<int>();
+    P.ccol = C_col; P.cval = (V*)C_val; P.nnzC = h->nnzC; P.nwin = (int)nwin;
+    P.row_begin = h->rb; P.mloc = mloc;
+    CK(launch_numeric<V>(h->stream, P));
+    h->launches += 2;
+  }
   h->stats.launches_numeric = h->launches;
   if (h->timing) {
     CK(cudaEventRecord(h->ev_t[4], h->stream));
@@ -461,13 +491,14 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     return SPG_ERR_CUDA;
   }
   cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, device);
-  e = dtype == SPG_FP64 ? BinLaunch<double>::configure() : BinLaunch<float>::configure();
+  e = light_configure();
+  if (e == cudaSuccess) e = heavy_configure();
+  if (e == cudaSuccess) e = dtype == SPG_FP64 ? numeric_configure<double>() : numeric_configure<float>();
   if (e == cudaSuccess) e = cudaHostAlloc((void**)&h->hr, sizeof(HostRead), cudaHostAllocDefault);
-  for (int c = 0; c < NUM_BINS && e == cudaSuccess; ++c) {
+  for (int c = 0; c < 4 && e == cudaSuccess; ++c) {
     e = cudaStreamCreateWithFlags(&h->aux[c], cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_join[c], cudaEventDisableTiming);
-    if (e == cudaSuccess) e = cudaEventCreate(&h->ev_c0[c]);
-    if (e == cudaSuccess) e = cudaEventCreate(&h->ev_c1[c]);
+    if (e == cudaSuccess) e = cudaEventCreate(&h->ev_p[c]);
   }
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming);
   for (int k = 0; k < 8 && e == cudaSuccess; ++k) e = cudaEventCreate(&h->ev_t[k]);
@@ -476,10 +507,8 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     spg_spgemm_free(h);
     return SPG_ERR_CUDA;
   }
-  for (int num = 0; num < 2; ++num)
-    for (int b = 0; b < NUM_BINS; ++b)
-      h->max_bpsm[num][b] = dtype == SPG_FP64 ? BinLaunch<double>::max_blocks_per_sm(b, num)
-                                              : BinLaunch<float>::max_blocks_per_sm(b, num);
+  h->occ_light = light_occupancy();
+  for (int b = 0; b < NUM_BINS; ++b) h->occ_heavy[b] = heavy_occupancy(b);
   cudaGetLastError();
   *out = h;
   return SPG_OK;
@@ -496,7 +525,7 @@ spg_status upload(spg_handle h, DevBuf& b, const void* src, size_t bytes) {
 // ===================================== ABI =====================================================
 extern "C" {
 
-const char* spg_version(void) { return "spg 0.1 (sm_100a, heavy/light-row Gustavson SpGEMM)"; }
+const char* spg_version(void) { return "spg 0.2 (sm_100a, heavy/light-row Gustavson SpGEMM, rank-scatter numeric)"; }
 
 spg_status spg_create(spg_handle* h, int device, void* cuda_stream, spg_dtype dtype) {
   return create_common(h, device, cuda_stream, dtype);
@@ -507,17 +536,17 @@ spg_status spg_spgemm_free(spg_handle h) {
   {
     DeviceGuard g(h->device);
     cudaStreamSynchronize(h->stream);
-    DevBuf* bufs[] = {&h->f, &h->nz, &h->sp, &h->lists, &h->small, &h->scan_tmp, &h->Pf, &h->splits, &h->iota,
-                      &h->ones, &h->crow_tmp, &h->fblist};
+    DevBuf* bufs[] = {&h->f,     &h->nz,    &h->rowA,   &h->Pe,    &h->cls,    &h->fl,  &h->Ro,
+                      &h->PL,    &h->tflag, &h->tiles,  &h->lists, &h->fblist, &h->small, &h->scan_tmp,
+                      &h->R,     &h->wrow,  &h->Pf,     &h->splits, &h->iota,  &h->ones, &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
     if (h->canon) spg_spgemm_free(h->canon);
     for (auto& b : h->hbuf) b.release();
-    for (int c = 0; c < NUM_BINS; ++c) {
+    for (int c = 0; c < 4; ++c) {
       if (h->aux[c]) cudaStreamDestroy(h->aux[c]);
       if (h->ev_join[c]) cudaEventDestroy(h->ev_join[c]);
-      if (h->ev_c0[c]) cudaEventDestroy(h->ev_c0[c]);
-      if (h->ev_c1[c]) cudaEventDestroy(h->ev_c1[c]);
+      if (h->ev_p[c]) cudaEventDestroy(h->ev_p[c]);
     }
     if (h->ev_fork) cudaEventDestroy(h->ev_fork);
     for (auto& e : h->ev_t)
@@ -536,15 +565,17 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
   if (!h) return SPG_ERR_INVALID_ARGUMENT;
   switch (opt) {
     case SPG_OPT_LIGHT_MAX_FLOPS:
-      if (v < TINY_MAX || v > LIGHT_CAP) return setf(h, SPG_ERR_INVALID_ARGUMENT, "LIGHT_MAX_FLOPS must be in [32, 256]");
+      if (v < 0 || v + h->tile_cap > TILE_PMAX)
+        return setf(h, SPG_ERR_INVALID_ARGUMENT, "LIGHT_MAX_FLOPS must be in [0, %d - TILE_FLOPS]", TILE_PMAX);
       h->light_max = (int)v;
       break;
-    case SPG_OPT_MEDIUM_MAX_FLOPS:
-      if (v < TINY_MAX || v > MEDIUM_CAP) return setf(h, SPG_ERR_INVALID_ARGUMENT, "MEDIUM_MAX_FLOPS must be in [32, 2048]");
-      h->medium_max = (int)v;
+    case SPG_OPT_TILE_FLOPS:
+      if (v < 1 || v + h->light_max > TILE_PMAX)
+        return setf(h, SPG_ERR_INVALID_ARGUMENT, "TILE_FLOPS must be in [1, %d - LIGHT_MAX_FLOPS]", TILE_PMAX);
+      h->tile_cap = (int)v;
       break;
     case SPG_OPT_HEAVY_MAX_FLOPS:
-      if (v < TINY_MAX || v > HEAVY_CAP) return setf(h, SPG_ERR_INVALID_ARGUMENT, "HEAVY_MAX_FLOPS must be in [32, 8192]");
+      if (v < 0 || v > HEAVY_CAP) return setf(h, SPG_ERR_INVALID_ARGUMENT, "HEAVY_MAX_FLOPS must be in [0, %d]", HEAVY_CAP);
       h->heavy_max = (int)v;
       break;
     case SPG_OPT_FORCE_CLASS:
@@ -570,7 +601,7 @@ spg_status spg_get_option(spg_handle h, spg_option opt, int64_t* v) {
   if (!h || !v) return SPG_ERR_INVALID_ARGUMENT;
   switch (opt) {
     case SPG_OPT_LIGHT_MAX_FLOPS: *v = h->light_max; break;
-    case SPG_OPT_MEDIUM_MAX_FLOPS: *v = h->medium_max; break;
+    case SPG_OPT_TILE_FLOPS: *v = h->tile_cap; break;
     case SPG_OPT_HEAVY_MAX_FLOPS: *v = h->heavy_max; break;
     case SPG_OPT_FORCE_CLASS: *v = h->force; break;
     case SPG_OPT_VALIDATE: *v = h->validate; break;
@@ -589,12 +620,6 @@ spg_status spg_get_stats(spg_handle h, spg_stats* out) {
   if (h->num_timed) {
     CK(cudaEventSynchronize(h->ev_t[4]));
     cudaEventElapsedTime(&h->stats.ms_numeric, h->ev_t[3], h->ev_t[4]);
-    for (int c = 0; c < NUM_CLS; ++c) h->stats.ms_class_numeric[c] = 0;
-    for (int b = 0; b < NUM_BINS; ++b) {
-      float ms = 0;
-      if (h->bin_timed[b] && cudaEventElapsedTime(&ms, h->ev_c0[b], h->ev_c1[b]) == cudaSuccess)
-        h->stats.ms_class_numeric[bin_class(b)] += ms;
-    }
   }
   *out = h->stats;
   return SPG_OK;
@@ -614,8 +639,7 @@ spg_status spg_spgemm_symbolic(spg_handle h, const spg_csr* A, const spg_csr* B,
     if (s != SPG_OK) return s;
     Bx = &h->Bc;
   }
-  s = h->dtype == SPG_FP64 ? symbolic_impl<double>(h, A, Bx, C_row_ptr, nnzC, row_begin, row_end)
-                           : symbolic_impl<float>(h, A, Bx, C_row_ptr, nnzC, row_begin, row_end);
+  s = symbolic_impl(h, A, Bx, C_row_ptr, nnzC, row_begin, row_end);
   if (s == SPG_OK) h->key = make_key(A, B);
   return s;
 }
@@ -708,7 +732,7 @@ spg_status spg_split_points(spg_handle h, const spg_csr* A, const spg_csr* B, in
   spg_status s = validate_pair(h, A, B, false);
   if (s != SPG_OK) return s;
   DeviceGuard g(h->device);
-  if ((s = ensure_ws(h, A->nrows)) != SPG_OK) return s;
+  if ((s = ensure_ws(h, A->nrows, A->nnz)) != SPG_OK) return s;
   if ((s = analysis(h, A, B)) != SPG_OK) return s;
   if ((s = split_points(h, A->nrows, P)) != SPG_OK) return s;
   std::memcpy(s_out, h->hr->splits, ((size_t)P + 1) * sizeof(int32_t));

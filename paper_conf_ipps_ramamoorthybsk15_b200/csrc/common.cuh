@@ -12,49 +12,33 @@ constexpr int KEY_INF = INT_MAX;  // sentinel column (> any valid column: N <= I
 // Row classes — must match spg_row_class in include/spg.h.
 enum : int { CLS_EMPTY = 0, CLS_SINGLE, CLS_TINY, CLS_LIGHT, CLS_MEDIUM, CLS_HEAVY, CLS_HUGE, NUM_CLS };
 
-// Internal work lists ("bins"): a class may be split by kernel geometry (TINY by sub-warp width).
-enum : int {
-  BIN_SINGLE = 0, BIN_T4, BIN_T8, BIN_T16, BIN_T32,   // TINY: one W-lane group per row
-  BIN_L64, BIN_L128, BIN_L256,                        // LIGHT: one warp per row, CAP = 64/128/256
-  BIN_M512, BIN_M1024, BIN_M2048,                     // MEDIUM: one block per row, CAP = 512/1024/2048
-  BIN_HEAVY, BIN_HEAVY2, BIN_HUGE,                    // HEAVY / HUGE: column-bitmap blocks
-  NUM_BINS
-};
-__host__ __device__ constexpr int bin_class(int b) {
-  return b == BIN_SINGLE ? CLS_SINGLE
-       : b <= BIN_T32   ? CLS_TINY
-       : b <= BIN_L256  ? CLS_LIGHT
-       : b <= BIN_M2048 ? CLS_MEDIUM
-       : b <= BIN_HEAVY2 ? CLS_HEAVY : CLS_HUGE;
-}
-__host__ __device__ constexpr int class_first_bin(int c) {
-  return c == CLS_SINGLE ? BIN_SINGLE
-       : c == CLS_TINY   ? BIN_T4
-       : c == CLS_LIGHT  ? BIN_L64
-       : c == CLS_MEDIUM ? BIN_M512
-       : c == CLS_HEAVY  ? BIN_HEAVY : BIN_HUGE;
-}
-__host__ __device__ constexpr bool bin_is_bitmap(int b) { return b >= BIN_HEAVY; }
+// Kernel paths ("bins").  TINY/LIGHT/MEDIUM rows all take the light (tile) kernel; HEAVY rows
+// the register-cached bitmap kernel (512 threads when f <= HEAVY1_CAP, else 1024); HUGE rows
+// (and rows the light kernel hands over) the uncached bitmap kernel.
+enum : int { BIN_HEAVY = 0, BIN_HEAVY2, BIN_HUGE, NUM_BINS };
 
-// Class-kernel geometry.
-constexpr int TINY_MAX = 32;          // one product per lane of a 4/8/16/32-lane group
-constexpr int LIGHT_CAP = 256;        // warp merge, per-warp shared memory
-constexpr int LIGHT_WARPS = 7;        // warps per block in the light kernel (4 blocks / SM fit in smem)
-constexpr int MED1_NT = 128;          // MEDIUM rows f <= 1024: 128-thread blocks
-constexpr int MEDIUM_NT = 256;        // MEDIUM rows f <= 2048: 256-thread blocks (occupancy)
-constexpr int MED1_CAP = 1024;        // MEDIUM rows split by shared-memory footprint
-constexpr int MEDIUM_CAP = 2048;
-constexpr int HEAVY_CAP = 8192;       // largest f of the register-cached bitmap mode
-constexpr int HEAVY1_CAP = 4096;      // HEAVY rows up to this f run as 512-thread blocks, 2 per SM
-constexpr int BMP_NT = 1024;          // bitmap kernel block size for HEAVY2 / HUGE (one block per SM)
-constexpr int BMP_NT_S = 512;         // ... for HEAVY (two blocks per SM)
-constexpr int MERGE_VT_MAX = 14;      // outputs per thread per merge round: min(ceil(f / G), 14) | 1
+// Per-row path code stored in the cls[] array (low 3 bits = class, bit 3 = light path).
+constexpr uint8_t CLS_LIGHT_PATH = 8;
 
-// Shared-memory bytes a merge of f products (nr <= f runs) needs: values x2, keys x2, seg.
-template <typename V>
-__host__ __device__ constexpr int merge_smem_bytes(int cap) {
-  return cap * (int)(2 * sizeof(V) + 2 * sizeof(int)) + (cap + 1) * (int)sizeof(int);
-}
+// Light (tile) kernel geometry.
+constexpr int TINY_MAX = 32;          // class boundaries for statistics only (same kernel)
+constexpr int LIGHTC_MAX = 256;
+constexpr int TILE_PMAX = 4096;       // products per tile: tile capacity + light threshold <= this
+constexpr int TILE_CAP_DEFAULT = 2048;
+constexpr int LIGHT_MAX_DEFAULT = 2048;
+constexpr int TILE_NT = 256;          // threads per tile block
+constexpr int TILE_RM = 512;          // light rows per batch
+constexpr int TILE_BK = 4;            // expected products per bucket
+constexpr int TILE_NBMAX = TILE_PMAX / TILE_BK + TILE_RM;  // buckets per batch (ceil per row)
+// Heavy (bitmap) kernel geometry.
+constexpr int HEAVY_CAP = 8192;       // largest f of the register-cached bitmap mode (1024 threads)
+constexpr int HEAVY1_CAP = 4096;      // ... 512-thread blocks, two per SM
+constexpr int BMP_NT = 1024;
+constexpr int BMP_NT_S = 512;
+// Numeric window kernel: outputs per window.
+constexpr int NUM_W = 4096;
+constexpr int NUM_NT = 256;
+constexpr unsigned RFLAG = 0x80000000u;  // R: first occurrence of its column in the row
 
 __device__ __forceinline__ unsigned lanemask_lt() {
   unsigned m;

@@ -1,0 +1,348 @@
+// k_heavy.cu — symbolic phase of the heavy rows (the paper's A_H: "good cache blocking
+// techniques can be used when multiplying A_H with B_H"): one 512- or 1024-thread
+// block per row, a column-tile bitmap in shared memory.
+//
+// The dense accumulator of [13] Alg. 1 (PartialOutput[N] + NonZeroIndices)
+// becomes a bitmap over a column tile of width Wt (TR_b of L88):
+//   pass 1  every product claims its column's bit with ATOMS.OR (on sm_100a as fast as a plain
+//           STS, tools/microbench_atomics.cu); the claimer that found the bit clear is the
+//           column's first occurrence.  A level-1 summary bit per bitmap word keeps every later
+//           step proportional to the touched words.
+//   build   rank prefixes: an int per 1024 columns and a u16 per 256 columns.
+//   pass 2  rank(col) = prefix + popcount of the <= 8 bitmap words below it in its 256-column
+//           block; R[Ro_i + j] = rank | RFLAG·first, written coalesced in product order.
+//   c_i     = claimed bits (summed over column tiles).
+// HEAVY rows (f <= 8192, one gather chunk) keep their products (column) in registers across
+// the passes and their first-occurrence flags in a shared bit array; other rows (HUGE, and rows
+// the light kernel handed over) re-gather columns per pass and keep the flag in R itself
+// between pass 1 and pass 2.  Products are visited in 32-product warp windows (coalesced within
+// a B row); the run of each lane comes from a REDUX.OR mask of run starts.
+#include "kernels.cuh"
+
+namespace spg {
+
+constexpr int BMP_CTCAP = 2048;      // 32-product windows per chunk with a precomputed run index
+constexpr int BMP_SLOTS = 8;         // products per lane cached in registers
+constexpr int MODE_CACHED = 0, MODE_PLAIN = 1;
+
+__host__ __device__ constexpr int al16(int x) { return (x + 15) & ~15; }
+
+template <int NT>
+__host__ __device__ constexpr int bmp_fixed_bytes() {
+  return 2 * al16((NT + 1) * 4) + al16(BMP_CTCAP * 2);
+}
+constexpr int BMP_SMEM_L = 226 * 1024;  // 1024-thread blocks, one per SM (static smem on top)
+constexpr int BMP_SMEM_S = 112 * 1024;  // 512-thread blocks, two per SM
+
+// Region bytes of a 2^lw column tile: bitmap, level-1 summary (one bit per bitmap word), rank
+// prefixes (int per 1024 columns, u16 per 256 columns) and — cached mode — f first-claim bits.
+template <int MODE>
+__device__ __forceinline__ int bmp_need(int lw, int f) {
+  const int words = 1 << (lw - 5), nl1 = 1 << (lw - 10);
+  int need = 4 * words + 4 * nl1 + 12 * nl1 + 16;
+  if (MODE == MODE_CACHED) need += 4 * ((f + 31) >> 5) + 16;
+  return need;
+}
+
+template <int MODE, int NT, int SMEM>
+__global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(SymProb P, const int* __restrict__ list,
+                                                                              const int* __restrict__ count, int lwmax,
+                                                                              int N) {
+  constexpr int RCAP = NT;
+  constexpr bool CACHED = MODE == MODE_CACHED;
+  extern __shared__ __align__(16) unsigned char sm[];
+  int* seg = reinterpret_cast<int*>(sm);                                   // run -> product offset
+  int* sbs = reinterpret_cast<int*>(sm + al16((RCAP + 1) * 4));            // run -> B row start
+  unsigned short* ctab = reinterpret_cast<unsigned short*>(sm + 2 * al16((RCAP + 1) * 4));  // window -> run
+  unsigned char* region = sm + bmp_fixed_bytes<NT>();
+  constexpr int REGION = SMEM - bmp_fixed_bytes<NT>();
+  __shared__ int scratch[NT / 32 + 1];
+  const Group<NT> g{(int)threadIdx.x, scratch};
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const unsigned upto = (2u << lane) - 1u;  // lanes <= me
+  if (!*P.r_ok) return;
+
+  // invariant between rows: the whole region is zero
+  for (int x = tid; x < REGION / 4; x += NT) reinterpret_cast<unsigned*>(region)[x] = 0;
+  __syncthreads();
+
+  // Rows are taken from a dynamic queue (one atomic per row): the bin's rows differ in size by
+  // up to an order of magnitude, so static striding would leave a long tail — the paper's work
+  // queue in its intra-GPU form.  count[0] = rows, count[8] = queue head.
+  const int n = count[0];
+  __shared__ int s_next;
+  for (;;) {
+    if (tid == 0) s_next = atomicAdd(const_cast<int*>(count) + 8, 1);
+    __syncthreads();
+    const int t = s_next;
+    __syncthreads();
+    if (t >= n) break;
+    const int li = list[t];
+    const int i = P.row_begin + li;
+    const int pa0 = P.rpA[i], pa1 = P.rpA[i + 1];
+    const int f = P.frow[i];
+    unsigned* Rrow = P.R + P.Ro[li];
+    // Column tile: the widest whose structures (and, cached, the flag bits) fit.
+    int lw = lwmax;
+    while (lw > 10 && bmp_need<MODE>(lw, f) > REGION) --lw;
+    const int Wt = 1 << lw, words = Wt >> 5, nl1 = 1 << (lw - 10);
+    unsigned* bm = reinterpret_cast<unsigned*>(region);
+    unsigned* l1 = bm + words;
+    int* sbp = reinterpret_cast<int*>(l1 + nl1);                           // rank prefix / 1024 columns
+    unsigned short* sbq = reinterpret_cast<unsigned short*>(sbp + nl1);   // .. / 256 columns (4 per 1024)
+    unsigned* flags = reinterpret_cast<unsigned*>(sbq + 4 * nl1);
+    const int nfw = CACHED ? (f + 31) >> 5 : 0;
+    const int ntiles = (int)(((long long)N + Wt - 1) >> lw);
+    const int nchunks = (pa1 - pa0 + RCAP - 1) / RCAP;
+    int out = 0;
+    int nz = 0, Lt = 0;  // current chunk: runs, products
+    int cc[BMP_SLOTS];   // cached mode: this lane's product columns
+
+    auto gather = [&](int c) {
+      const int p = pa0 + c * RCAP + tid;
+      const int pend = min(pa1, pa0 + (c + 1) * RCAP);
+      int L = 0, bs = 0;
+      if (p < pend) {
+        const int k = P.colA[p];
+        bs = P.rpB[k];
+        L = P.rpB[k + 1] - bs;
+      }
+      const int rk = g.excl_scan(L > 0 ? 1 : 0, nz);
+      const int off = g.excl_scan(L, Lt);  // f_i < 2^31 (checked in analysis)
+      if (L > 0) {
+        seg[rk] = off;
+        sbs[rk] = bs;
+      }
+      if (tid == 0) seg[nz] = Lt;
+      __syncthreads();
+      for (int x = tid; x < min((Lt + 31) >> 5, BMP_CTCAP); x += NT) ctab[x] = (unsigned short)upper_idx(seg, nz, x << 5);
+      __syncthreads();
+    };
+
+    // product window [j0, j0+32): run of each lane (runs starting inside the window form a
+    // bitmask, REDUX.OR; a lane's run = the window's first run + popcount of starts <= it)
+    auto lane_run = [&](int j0) {
+      const int rb = (j0 >> 5) < BMP_CTCAP ? (int)ctab[j0 >> 5] : upper_idx(seg, nz, j0);
+      const int rs = rb + 1 + lane;
+      const int d = rs <= nz ? seg[rs] - j0 : 32;
+      const unsigned M = __reduce_or_sync(FULL, (d >= 1 && d <= 31) ? (1u << d) : 0u);
+      return rb + __popc(M & upto);
+    };
+
+    // Visit the products of the current chunk: fn(j, col) with j the chunk product index.
+    // Cached: from the register cache.  Otherwise each warp takes 32-product windows, BATCH
+    // windows' loads issued together.
+    constexpr int BATCH = 4;
+    auto for_products = [&](auto&& fn) {
+      if constexpr (CACHED) {
+#pragma unroll
+        for (int s = 0; s < BMP_SLOTS; ++s) {
+          const int j = warp * 32 + s * NT + lane;
+          if (j < Lt) fn(j, cc[s]);
+        }
+      } else {
+        for (int j00 = warp * 32; j00 < Lt; j00 += BATCH * NT) {
+          int q[BATCH], col[BATCH];
+#pragma unroll
+          for (int u = 0; u < BATCH; ++u) {
+            const int j0 = j00 + u * NT;
+            q[u] = -1;
+            if (j0 < Lt) {
+              const int r = lane_run(j0);
+              if (j0 + lane < Lt) q[u] = sbs[r] + (j0 + lane - seg[r]);
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < BATCH; ++u) col[u] = q[u] >= 0 ? P.colB[q[u]] : -1;
+#pragma unroll
+          for (int u = 0; u < BATCH; ++u)
+            if (q[u] >= 0) fn(j00 + u * NT + lane, col[u]);
+        }
+      }
+    };
+    auto fill_cache = [&]() {
+      int q[BMP_SLOTS];
+#pragma unroll
+      for (int s = 0; s < BMP_SLOTS; ++s) {
+        const int j0 = warp * 32 + s * NT;
+        q[s] = -1;
+        if (j0 < Lt) {
+          const int r = lane_run(j0);
+          if (j0 + lane < Lt) q[s] = sbs[r] + (j0 + lane - seg[r]);
+        }
+      }
+#pragma unroll
+      for (int s = 0; s < BMP_SLOTS; ++s) cc[s] = q[s] >= 0 ? P.colB[q[s]] : -1;
+    };
+
+    // rank of a tile-local column among the tile's claimed columns: prefix of its 1024- and
+    // 256-column blocks + popcounts of the (<= 8) words of its 256-column block below it
+    auto rank_of = [&](unsigned lc) {
+      const int w = lc >> 5, v = w >> 3, k = w & 7;
+      const uint4 a = reinterpret_cast<const uint4*>(bm)[2 * v];
+      const uint4 b = reinterpret_cast<const uint4*>(bm)[2 * v + 1];
+      const unsigned wd[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+      int r = sbp[w >> 5] + sbq[v];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const unsigned m = q < k ? 0xffffffffu : (q == k ? (1u << (lc & 31)) - 1 : 0u);
+        r += __popc(wd[q] & m);
+      }
+      return r;
+    };
+
+    for (int tile = 0; tile < ntiles; ++tile) {
+      const int lo = tile << lw;
+      // ---- pass 1: claim bits; first claimers flagged -----------------------------------------
+      int cbase = 0;
+      for (int c = 0; c < nchunks; ++c) {
+        if (nchunks > 1 || tile == 0) {
+          gather(c);
+          if constexpr (CACHED) fill_cache();
+        }
+        if constexpr (CACHED) {
+          // cached windows start at multiples of 32: one ballot word of first-claim flags each
+#pragma unroll
+          for (int s = 0; s < BMP_SLOTS; ++s) {
+            const int j0 = warp * 32 + s * NT;
+            const unsigned lc = (unsigned)(cc[s] - lo);
+            bool first = false;
+            if (j0 + lane < Lt && lc < (unsigned)Wt) {
+              const int w = lc >> 5;
+              const unsigned b = 1u << (lc & 31);
+              const unsigned old = atomicOr(&bm[w], b);
+              first = !(old & b);
+              if (old == 0) atomicOr(&l1[w >> 5], 1u << (w & 31));
+            }
+            const unsigned fm = __ballot_sync(FULL, first);
+            if (lane == 0 && j0 < Lt) flags[j0 >> 5] = fm;
+          }
+        } else {
+          for_products([&](int j, int col) {
+            const unsigned lc = (unsigned)(col - lo);
+            if (lc < (unsigned)Wt) {
+              const int w = lc >> 5;
+              const unsigned b = 1u << (lc & 31);
+              const unsigned old = atomicOr(&bm[w], b);
+              if (old == 0) atomicOr(&l1[w >> 5], 1u << (w & 31));
+              Rrow[cbase + j] = (old & b) ? 0u : RFLAG;
+            }
+          });
+        }
+        cbase += Lt;
+        __syncthreads();
+      }
+      // ---- build: rank prefixes per 1024- and 256-column block (touched superblocks only) -----
+      int pcarry = 0;
+      for (int u0 = 0; u0 < nl1; u0 += NT) {
+        const int u = u0 + tid;
+        const unsigned x = u < nl1 ? l1[u] : 0u;
+        int pc = 0;
+        unsigned short q4[4] = {0, 0, 0, 0};
+        if (x) {
+          // all 32 words of the superblock; the 16-byte reads are rotated by lane so a warp's
+          // loads spread over all banks (a straight walk would be a 32-way conflict)
+          int sub[4] = {0, 0, 0, 0};
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            const int m = (k + tid) & 7;
+            const uint4 a = reinterpret_cast<const uint4*>(bm)[8 * u + m];
+            const int c4 = __popc(a.x) + __popc(a.y) + __popc(a.z) + __popc(a.w);
+#pragma unroll
+            for (int h = 0; h < 4; ++h) sub[h] += (m >> 1) == h ? c4 : 0;
+          }
+          q4[1] = (unsigned short)sub[0];
+          q4[2] = (unsigned short)(sub[0] + sub[1]);
+          q4[3] = (unsigned short)(sub[0] + sub[1] + sub[2]);
+          pc = sub[0] + sub[1] + sub[2] + sub[3];
+        }
+        int ptot;
+        const int pp = pcarry + g.excl_scan(pc, ptot);
+        if (x) {  // only touched superblocks are ever queried (and cleared)
+          sbp[u] = pp;
+          reinterpret_cast<unsigned long long*>(sbq)[u] =
+              (unsigned long long)q4[0] | ((unsigned long long)q4[1] << 16) | ((unsigned long long)q4[2] << 32) |
+              ((unsigned long long)q4[3] << 48);
+        }
+        pcarry += ptot;
+      }
+      const int ctile = pcarry;
+      __syncthreads();
+      // ---- pass 2: ranks -> R ---------------------------------------------------------------------
+      cbase = 0;
+      for (int c = 0; c < nchunks; ++c) {
+        if (nchunks > 1) gather(c);
+        for_products([&](int j, int col) {
+          const unsigned lc = (unsigned)(col - lo);
+          if (lc < (unsigned)Wt) {
+            const unsigned r = (unsigned)(out + rank_of(lc));
+            if constexpr (CACHED) {
+              const unsigned fl = (flags[j >> 5] >> (j & 31)) & 1u;
+              Rrow[j] = r | (fl << 31);
+            } else {
+              Rrow[cbase + j] = r | (Rrow[cbase + j] & RFLAG);
+            }
+          }
+        });
+        cbase += Lt;
+        __syncthreads();
+      }
+      out += ctile;
+      // ---- restore the zero invariant: touched bitmap words, summary, prefixes, flags ------------
+      for (int u = tid; u < nl1; u += NT) {
+        unsigned x = l1[u];
+        if (x) {
+          l1[u] = 0;
+          sbp[u] = 0;
+          reinterpret_cast<unsigned long long*>(sbq)[u] = 0ull;
+          while (x) {
+            const int b = __ffs(x) - 1;
+            x &= x - 1;
+            bm[(u << 5) + b] = 0;
+          }
+        }
+      }
+      if (CACHED)
+        for (int x = tid; x < nfw; x += NT) flags[x] = 0;
+      __syncthreads();
+    }
+    if (tid == 0) P.crow[li + 1] = out;
+  }
+}
+
+// ================================ launch glue ====================================================
+static const void* bitmap_kernel(int bin) {
+  switch (bin) {
+    case BIN_HEAVY: return (const void*)k_bitmap_rank<MODE_CACHED, BMP_NT_S, BMP_SMEM_S>;
+    case BIN_HEAVY2: return (const void*)k_bitmap_rank<MODE_CACHED, BMP_NT, BMP_SMEM_L>;
+    default: return (const void*)k_bitmap_rank<MODE_PLAIN, BMP_NT, BMP_SMEM_L>;
+  }
+}
+static int bitmap_threads(int bin) { return bin == BIN_HEAVY ? BMP_NT_S : BMP_NT; }
+static int bitmap_smem(int bin) { return bin == BIN_HEAVY ? BMP_SMEM_S : BMP_SMEM_L; }
+
+cudaError_t heavy_configure() {
+  for (int bin : {BIN_HEAVY, BIN_HEAVY2, BIN_HUGE}) {
+    cudaError_t e = cudaFuncSetAttribute(bitmap_kernel(bin), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         bitmap_smem(bin));
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+int heavy_occupancy(int bin) {
+  int nb = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, bitmap_kernel(bin), bitmap_threads(bin), bitmap_smem(bin));
+  return nb < 1 ? 1 : nb;
+}
+
+cudaError_t launch_heavy_rank(int bin, cudaStream_t st, int grid, const SymProb& P, const int* list,
+                              const int* count, long long N) {
+  int lwmax = 10;
+  while (lwmax < 20 && ((long long)1 << lwmax) < N) ++lwmax;
+  int n32 = (int)N;
+  void* args[] = {(void*)&P, (void*)&list, (void*)&count, (void*)&lwmax, (void*)&n32};
+  return cudaLaunchKernel(bitmap_kernel(bin), dim3(grid), dim3(bitmap_threads(bin)), args, bitmap_smem(bin), st);
+}
+
+}  // namespace spg

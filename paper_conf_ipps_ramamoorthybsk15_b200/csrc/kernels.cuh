@@ -1,48 +1,98 @@
 // kernels.cuh — declarations shared by the kernel translation units and the C-ABI layer.
+//
+// Pipeline:
+//   analysis   k_row_flops: f_i, run flags, log2 histogram, per-A-entry row and in-row product
+//              offset (rowA, Pe)
+//   classify   k_classify: row path (light tile kernel / heavy bitmap kernel / identity copy),
+//              heavy row lists and their R offsets; scan of light flops -> PL; k_tiles: tile
+//              cut points in light-product space, R offsets of light rows
+//   symbolic   k_light_rank (tiles of light rows) and k_bitmap_rank (heavy rows) compute, for
+//              every product of row i, its rank among the distinct columns of C(i,:) plus a
+//              first-occurrence flag: R[Ro_i + j] = rank | RFLAG·first.  c_i = #distinct.
+//   numeric    k_numeric: windows of NUM_W consecutive outputs of C; every product of the
+//              window's rows is scattered by its rank into shared memory and the window is
+//              written out coalesced (the Phase IV merge of PAPER.md L154-156, with the sort
+//              moved to the symbolic phase so numeric re-runs are a stream over R).
 #pragma once
 #include "common.cuh"
 
 namespace spg {
 
 struct ClassParams {
-  int light_max;   // f <= light_max -> LIGHT (warp merge), 32 < light_max <= LIGHT_CAP
-  int medium_max;  // f <= medium_max -> MEDIUM (256-thread block)
-  int heavy_max;   // f <= heavy_max -> HEAVY (512-thread block), else HUGE
+  int light_max;   // f <= light_max -> light (tile) kernel
+  int heavy_max;   // f <= heavy_max -> register-cached bitmap kernel, else HUGE (uncached)
+  int tile_cap;    // nominal products per tile (light_max + tile_cap <= TILE_PMAX)
   int force;       // -1 or a class id >= CLS_TINY
-  int single_ok;   // B rows canonical -> SINGLE shortcut allowed
+  int single_ok;   // B rows canonical -> SINGLE (identity) shortcut allowed
 };
 
-struct BinLists {
+struct HeavyLists {
   int* rows[NUM_BINS];
 };
 
-// Problem view passed to the class kernels.  crow is the int64 C row-offset array of this
-// rank's rows (index i - row_begin); symbolic writes counts at [i - row_begin + 1].
+// Small per-call device scratch (zeroed at the start of every symbolic call).
+struct Small {
+  int counts[8];            // per bitmap bin: rows
+  int qhead[8];             // per bitmap bin: dynamic row-queue heads (counts + 8)
+  int fb[16];               // fallback rows from the light kernel: [0] rows, [8] queue head
+  int ntiles;
+  int err;
+  int r_ok;                 // R capacity sufficient (written by k_tiles)
+  int amax;                 // longest row of A
+  long long heavy_total;    // products of heavy rows (R offsets of heavy rows, relative)
+  long long fr;             // products needing R (light + heavy)
+  unsigned long long hist[65];
+  unsigned long long cstats[2 * NUM_CLS + 2];
+};
+
+// Problem view passed to the symbolic kernels.  Row indices in lists / cls / Ro / crow are
+// local (i - row_begin).
+struct SymProb {
+  const int* __restrict__ rpA;
+  const int* __restrict__ colA;
+  const int* __restrict__ rpB;
+  const int* __restrict__ colB;
+  const int* frow;          // f_i (global row index)
+  const uint8_t* cls;       // path per local row
+  const long long* Ro;      // R offset per local row (-1: identity / empty)
+  unsigned* R;              // rank array
+  long long* crow;          // C row offsets (local); symbolic writes counts at [li + 1]
+  const int* r_ok;
+  int row_begin, row_end;
+  int lgN;                  // ceil(log2 N), N = columns of B
+};
+
+// Problem view of the numeric kernel.
 template <typename V>
-struct Prob {
+struct NumProb {
   const int* __restrict__ rpA;
   const int* __restrict__ colA;
   const V* __restrict__ valA;
   const int* __restrict__ rpB;
   const int* __restrict__ colB;
   const V* __restrict__ valB;
-  const int* sp;    // per row: index of one A entry whose B row is non-empty (row analysis)
-  const int* frow;  // per row: f_i (row analysis)
-  int row_begin;
-  int lgN;          // ceil(log2(N)), N = columns of B (>= 0)
-  long long* crow;
+  const int* __restrict__ rowA;   // global row of each A entry
+  const int* __restrict__ Pe;     // in-row product offset of each A entry
+  const long long* __restrict__ Ro;
+  const unsigned* __restrict__ R;
+  const long long* __restrict__ crow;
+  const int* __restrict__ wrow;   // first local row of each window
   int* ccol;
   V* cval;
-  int* fb_list;     // numeric: rows the light/medium kernels hand to the general kernel
-  int* fb_count;    // [0] = rows, [16] = queue head of the general kernel
+  long long nnzC;
+  int nwin;
+  int row_begin, mloc;
 };
 
 // analysis.cu
 cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB, int* f,
-                             uint8_t* nz, int* sp, unsigned long long* hist, int* err, int* amax);
+                             uint8_t* nz, int* rowA, int* Pe, unsigned long long* hist, int* err, int* amax);
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
-                            const ClassParams& prm, const BinLists& lists, int* counts, unsigned long long* cstats,
-                            long long* crow);
+                            const ClassParams& prm, uint8_t* cls, int* fl, long long* Ro, const HeavyLists& lists,
+                            Small* small, long long* crow);
+cudaError_t launch_tiles(cudaStream_t st, int sms, const int* f, int rb, int re, int tile_cap, const uint8_t* cls,
+                         const long long* PL, long long* Ro, uint8_t* tflag, int* tiles, Small* small,
+                         long long r_cap);
 size_t scan_tmp_elems(long long n);
 int scan_launches(long long n);
 template <typename Tin>
@@ -56,18 +106,23 @@ template <typename V>
 cudaError_t launch_fill(cudaStream_t st, V* p, long long n, V v);
 cudaError_t launch_narrow(cudaStream_t st, const long long* in, int* out, long long n);
 
-// Class kernels: one launcher per bin and phase.  `count` is the device-side bin size; `grid`
-// is chosen by the caller (persistent grid-stride loops inside).  N = columns of B.
+// k_light.cu — symbolic ranks of the light rows, one tile per block iteration.
+cudaError_t light_configure();
+int light_occupancy();
+cudaError_t launch_light_rank(cudaStream_t st, int grid, const SymProb& P, const int* tiles, const int* ntiles,
+                              const uint8_t* tflag, const long long* PL, int* fb_list, int* fb_count);
+
+// k_heavy.cu — symbolic ranks of heavy rows (column bitmap), per bin or over an explicit list.
+cudaError_t heavy_configure();
+int heavy_occupancy(int bin);
+cudaError_t launch_heavy_rank(int bin, cudaStream_t st, int grid, const SymProb& P, const int* list,
+                              const int* count, long long N);
+
+// k_numeric.cu — numeric phase.
 template <typename V>
-struct BinLaunch {
-  static cudaError_t launch(int bin, cudaStream_t st, int grid, bool numeric, const Prob<V>& P, const int* list,
-                            const int* count, long long N);
-  static int rows_per_block(int bin);
-  static int max_blocks_per_sm(int bin, bool numeric);
-  static cudaError_t configure();  // opt-in dynamic shared memory sizes (once per device)
-  // general (HUGE-tier) kernel over an explicit row list, e.g. the fallback list
-  static cudaError_t launch_general(cudaStream_t st, int grid, const Prob<V>& P, const int* list, const int* count,
-                                    long long N);
-};
+cudaError_t numeric_configure();
+cudaError_t launch_window_rows(cudaStream_t st, const long long* crow, int mloc, int* wrow, int nwin);
+template <typename V>
+cudaError_t launch_numeric(cudaStream_t st, const NumProb<V>& P);
 
 }  // namespace spg

@@ -19,7 +19,10 @@ def run_gpu(A, B, **opts):
     """Symbolic + numeric through the C ABI; returns host (row_ptr int64, col int32, val, stats)."""
     dA = to_dev(A)
     dB = dA if B is A else to_dev(B)
+    then = opts.pop("_then", {})
     plan = spg.SpGEMM(0, dA.vals.dtype, **opts)
+    for k, v in then.items():
+        plan.set_option(k, v)
     try:
         C = plan(dA, dB)
         torch.cuda.synchronize()

@@ -4,6 +4,7 @@
 #include <nccl.h>
 
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <new>
@@ -42,6 +43,7 @@ struct DevBuf {
 struct HostRead {  // pinned readback area
   Small small;
   long long nnz;
+  long long ncut;
   int splits[1025];
 };
 
@@ -78,22 +80,24 @@ struct spg_ctx {
   int light_max = LIGHT_MAX_DEFAULT, tile_cap = TILE_CAP_DEFAULT, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
   // workspace: analysis (all rows / all A entries), classification (this rank's rows), R, windows
-  DevBuf f, nz, rowA, Pe, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, R, wrow, Pf, splits,
-      canonB[4], iota, ones, crow_tmp;
+  DevBuf f, nz, rowA, Pe, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, R, cuts, wunits, lunits, rec0, rec1, gq, Pf,
+      splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
   long long iota_n = -1, ones_n = -1;
   HostRead* hr = nullptr;
-  cudaStream_t aux[4] = {};
-  cudaEvent_t ev_fork = nullptr, ev_join[4] = {};
+  cudaStream_t aux[6] = {};
+  cudaEvent_t ev_fork = nullptr, ev_join[6] = {};
   cudaEvent_t ev_t[8] = {};
   cudaEvent_t ev_p[4] = {};  // light path start/end, heavy path start/end
-  int occ_light = 1, occ_heavy[NUM_BINS] = {};
+  int occ_light = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1, occ_large[2] = {1, 1};
+  int large_cfg = 0;  // numeric large-row kernel configuration (SPG_LARGE_CFG=1: B)
   // cached symbolic state
   bool sym_ok = false;
   SymKey key{};
   int32_t rb = 0, re = 0;
   int64_t nnzC = 0;
+  int nwunits = 0, nlunits = 0, lcap = 0;
   int counts[NUM_BINS] = {};
   spg_stats stats{};
   bool num_timed = false, paths_timed = false;
@@ -201,24 +205,26 @@ spg_status run_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* 
       CK(cudaStreamWaitEvent(h->stream, h->ev_join[0], 0));
     }
   }
-  // heavy bins
+  // heavy bins, each on its own stream (the HUGE bin's long rows overlap the others' work)
   {
-    cudaStream_t st = conc ? h->aux[1] : h->stream;
-    if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
-    if (tm) CK(cudaEventRecord(h->ev_p[2], st));
     const long long Mloc = h->re - h->rb;
-    for (int b : {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY}) {
+    const int order[NUM_BINS] = {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY};
+    for (int x = 0; x < NUM_BINS; ++x) {
+      const int b = order[x];
+      cudaStream_t st = conc ? h->aux[1 + x] : h->stream;
+      if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
+      if (tm && x == 0) CK(cudaEventRecord(h->ev_p[2], st));
       long long grid = (long long)h->occ_heavy[b] * h->sms;
       if (h->huge_slots_opt > 0 && h->huge_slots_opt < grid) grid = h->huge_slots_opt;
       const int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
       CK(launch_heavy_rank(b, st, (int)grid, P, list, ds->counts + b, B->ncols));
       h->launches++;
+      if (conc) {
+        CK(cudaEventRecord(h->ev_join[1 + x], st));
+        CK(cudaStreamWaitEvent(h->stream, h->ev_join[1 + x], 0));
+      }
     }
-    if (tm) CK(cudaEventRecord(h->ev_p[3], st));
-    if (conc) {
-      CK(cudaEventRecord(h->ev_join[1], st));
-      CK(cudaStreamWaitEvent(h->stream, h->ev_join[1], 0));
-    }
+    if (tm) CK(cudaEventRecord(h->ev_p[3], h->stream));
   }
   h->paths_timed = tm;
   // rows with clustered columns, handed over by the light kernel
@@ -243,6 +249,10 @@ spg_status ensure_ws(spg_handle h, int M, long long nnzA) {
   CK(h->tiles.ensure(m * sizeof(int)));
   CK(h->lists.ensure(m * NUM_BINS * sizeof(int)));
   CK(h->fblist.ensure(m * sizeof(int)));
+  CK(h->cuts.ensure((2 * m + 2) * sizeof(Cut)));
+  CK(h->wunits.ensure((2 * m + 2) * sizeof(Unit)));
+  CK(h->rec0.ensure(na * sizeof(int4)));
+  CK(h->rec1.ensure(na * sizeof(int4)));
   CK(h->small.ensure(sizeof(Small)));
   CK(h->scan_tmp.ensure(scan_tmp_elems((long long)m + 1) * sizeof(long long)));
   return SPG_OK;
@@ -387,7 +397,17 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));
     if ((s = run_sym(h, A, B, crow)) != SPG_OK) return s;
     CK(launch_incl_scan<long long>(h->stream, crow + 1, crow + 1, Mloc, h->scan_tmp.as<long long>()));
-    h->launches += scan_launches(Mloc);
+    // numeric plan: row-aligned units and per-entry run records (cut counts in fl, their prefix in
+    // PL — both free now)
+    // segment units of long rows: capacity from the last call (the count is read back; a larger
+    // need reruns the plan below)
+    if (h->lcap < Mloc + 1) h->lcap = (int)(Mloc + 1);
+    CK(h->lunits.ensure((size_t)h->lcap * sizeof(Unit)));
+    CK(launch_plan(h->stream, h->sms, crow, (int)Mloc, A->row_ptr, A->col_idx, B->row_ptr, h->rowA.as<int>(),
+                   h->Pe.as<int>(), h->Ro.as<long long>(), h->R.as<unsigned>(), h->rb, h->re, A->nnz,
+                   h->fl.as<int>(), PL, h->scan_tmp.as<long long>(), h->cuts.as<Cut>(), h->wunits.as<Unit>(),
+                   h->lunits.as<Unit>(), h->lcap, h->rec0.as<int4>(), h->rec1.as<int4>(), ds));
+    h->launches += scan_launches(Mloc) + plan_launches(Mloc);
     if (h->timing) CK(cudaEventRecord(h->ev_t[2], h->stream));
     CK(cudaMemcpyAsync(&h->hr->small, ds, sizeof(Small), cudaMemcpyDeviceToHost, h->stream));
     CK(cudaMemcpyAsync(&h->hr->nnz, crow + Mloc, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
@@ -395,12 +415,26 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     const Small& hs = h->hr->small;
     if (hs.err & 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "A has a column index outside [0, B.nrows)");
     if (hs.err & 2) return setf(h, SPG_ERR_INDEX_OVERFLOW, "a row of A has >= 2^31 intermediate products");
+    if (hs.r_ok && hs.nlunits > h->lcap) {  // more long-row segments than room: grow, rerun the plan
+      h->lcap = hs.nlunits + 64;
+      CK(h->lunits.ensure((size_t)h->lcap * sizeof(Unit)));
+      CK(cudaMemsetAsync(&ds->nwunits, 0, 2 * sizeof(int), h->stream));
+      CK(launch_plan(h->stream, h->sms, crow, (int)Mloc, A->row_ptr, A->col_idx, B->row_ptr, h->rowA.as<int>(),
+                     h->Pe.as<int>(), h->Ro.as<long long>(), h->R.as<unsigned>(), h->rb, h->re, A->nnz,
+                     h->fl.as<int>(), PL, h->scan_tmp.as<long long>(), h->cuts.as<Cut>(), h->wunits.as<Unit>(),
+                     h->lunits.as<Unit>(), h->lcap, h->rec0.as<int4>(), h->rec1.as<int4>(), ds));
+      h->launches += plan_launches(Mloc);
+      CK(cudaMemcpyAsync(&h->hr->small, ds, sizeof(Small), cudaMemcpyDeviceToHost, h->stream));
+      CK(cudaStreamSynchronize(h->stream));
+    }
     if (hs.r_ok || attempt > 0) break;
     CK(h->R.ensure((size_t)(hs.fr > 0 ? hs.fr : 1) * sizeof(unsigned)));
   }
   const Small& hs = h->hr->small;
   if (!hs.r_ok && hs.fr > 0) return setf(h, SPG_ERR_OUT_OF_MEMORY, "rank array could not be sized");
   h->nnzC = h->hr->nnz;
+  h->nwunits = hs.nwunits;
+  h->nlunits = hs.nlunits;
   for (int b = 0; b < NUM_BINS; ++b) h->counts[b] = hs.counts[b];
   spg_stats& st = h->stats;
   std::memset(&st, 0, sizeof st);
@@ -440,23 +474,44 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
 template <typename V>
 spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const int64_t* C_row_ptr, int32_t* C_col,
                         void* C_val) {
+  (void)C_row_ptr;  // the symbolic plan already holds every row's C offset (run records)
   if (h->timing) CK(cudaEventRecord(h->ev_t[3], h->stream));
   h->launches = 0;
-  const long long nwin = (h->nnzC + NUM_W - 1) / NUM_W;
-  if (nwin > INT_MAX) return setf(h, SPG_ERR_NOT_SUPPORTED, "nnz(C) too large for one rank (%lld windows)", nwin);
-  if (nwin > 0) {
-    CK(h->wrow.ensure((size_t)nwin * sizeof(int)));
-    const int mloc = h->re - h->rb;
-    CK(launch_window_rows(h->stream, (const long long*)C_row_ptr, mloc, h->wrow.as<int>(), (int)nwin));
+  if (h->nnzC > 0) {
+    Small* ds = h->small.as<Small>();
     NumProb<V> P;
-    P.rpA = A->row_ptr; P.colA = A->col_idx; P.valA = (const V*)A->vals;
-    P.rpB = B->row_ptr; P.colB = B->col_idx; P.valB = (const V*)B->vals;
-    P.rowA = h->rowA.as<int>(); P.Pe = h->Pe.as<int>(); P.Ro = h->Ro.as<long long>();
-    P.R = h->R.as<unsigned>(); P.crow = (const long long*)C_row_ptr; P.wrow = h->wrow.as<int>();
-    P.ccol = C_col; P.cval = (V*)C_val; P.nnzC = h->nnzC; P.nwin = (int)nwin;
-    P.row_begin = h->rb; P.mloc = mloc;
-    CK(launch_numeric<V>(h->stream, P));
-    h->launches += 2;
+    P.valA = (const V*)A->vals;
+    P.colB = B->col_idx; P.valB = (const V*)B->vals;
+    P.R = h->R.as<unsigned>(); P.rec0 = h->rec0.as<int4>(); P.rec1 = h->rec1.as<int4>();
+    P.wunits = h->wunits.as<Unit>(); P.lunits = h->lunits.as<Unit>(); P.small = ds;
+    P.lqhead = &ds->lqhead; P.gq_pos = nullptr; P.gq_val = nullptr;
+    P.ccol = C_col; P.cval = (V*)C_val;
+    const bool conc = h->concurrent != 0 && h->nlunits > 0 && h->nwunits > 0;
+    if (h->nlunits > 0) {
+      const bool cfgB = h->large_cfg != 0;
+      int grid = h->occ_large[cfgB] * h->sms;
+      if (h->nlunits < grid) grid = h->nlunits;
+      CK(h->gq.ensure((size_t)grid * NUM_GDUP * (sizeof(int) + sizeof(V))));
+      P.gq_pos = h->gq.as<int>();
+      P.gq_val = reinterpret_cast<V*>(P.gq_pos + (size_t)grid * NUM_GDUP);
+      CK(cudaMemsetAsync(&ds->lqhead, 0, sizeof(int), h->stream));
+      if (conc) {
+        CK(cudaEventRecord(h->ev_fork, h->stream));
+        CK(cudaStreamWaitEvent(h->aux[4], h->ev_fork, 0));
+      }
+      CK(launch_num_large<V>(conc ? h->aux[4] : h->stream, grid, cfgB, P));
+      h->launches++;
+    }
+    if (h->nwunits > 0) {
+      int grid = h->occ_num * h->sms;
+      if (h->nwunits < grid) grid = h->nwunits;
+      CK(launch_num_windows<V>(h->stream, grid, P));
+      h->launches++;
+    }
+    if (conc) {
+      CK(cudaEventRecord(h->ev_join[4], h->aux[4]));
+      CK(cudaStreamWaitEvent(h->stream, h->ev_join[4], 0));
+    }
   }
   h->stats.launches_numeric = h->launches;
   if (h->timing) {
@@ -495,10 +550,10 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
   if (e == cudaSuccess) e = heavy_configure();
   if (e == cudaSuccess) e = dtype == SPG_FP64 ? numeric_configure<double>() : numeric_configure<float>();
   if (e == cudaSuccess) e = cudaHostAlloc((void**)&h->hr, sizeof(HostRead), cudaHostAllocDefault);
-  for (int c = 0; c < 4 && e == cudaSuccess; ++c) {
+  for (int c = 0; c < 6 && e == cudaSuccess; ++c) {
     e = cudaStreamCreateWithFlags(&h->aux[c], cudaStreamNonBlocking);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_join[c], cudaEventDisableTiming);
-    if (e == cudaSuccess) e = cudaEventCreate(&h->ev_p[c]);
+    if (e == cudaSuccess && c < 4) e = cudaEventCreate(&h->ev_p[c]);
   }
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming);
   for (int k = 0; k < 8 && e == cudaSuccess; ++k) e = cudaEventCreate(&h->ev_t[k]);
@@ -508,6 +563,10 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     return SPG_ERR_CUDA;
   }
   h->occ_light = light_occupancy();
+  h->occ_num = dtype == SPG_FP64 ? numeric_occupancy<double>(0) : numeric_occupancy<float>(0);
+  for (int x = 0; x < 2; ++x)
+    h->occ_large[x] = dtype == SPG_FP64 ? numeric_occupancy<double>(1 + x) : numeric_occupancy<float>(1 + x);
+  h->large_cfg = getenv("SPG_LARGE_CFG") != nullptr && getenv("SPG_LARGE_CFG")[0] == '1';
   for (int b = 0; b < NUM_BINS; ++b) h->occ_heavy[b] = heavy_occupancy(b);
   cudaGetLastError();
   *out = h;
@@ -538,15 +597,15 @@ spg_status spg_spgemm_free(spg_handle h) {
     cudaStreamSynchronize(h->stream);
     DevBuf* bufs[] = {&h->f,     &h->nz,    &h->rowA,   &h->Pe,    &h->cls,    &h->fl,  &h->Ro,
                       &h->PL,    &h->tflag, &h->tiles,  &h->lists, &h->fblist, &h->small, &h->scan_tmp,
-                      &h->R,     &h->wrow,  &h->Pf,     &h->splits, &h->iota,  &h->ones, &h->crow_tmp};
+                      &h->R,     &h->cuts,  &h->wunits, &h->lunits, &h->rec0, &h->rec1, &h->gq, &h->Pf,     &h->splits, &h->iota,  &h->ones, &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
     if (h->canon) spg_spgemm_free(h->canon);
     for (auto& b : h->hbuf) b.release();
-    for (int c = 0; c < 4; ++c) {
+    for (int c = 0; c < 6; ++c) {
       if (h->aux[c]) cudaStreamDestroy(h->aux[c]);
       if (h->ev_join[c]) cudaEventDestroy(h->ev_join[c]);
-      if (h->ev_p[c]) cudaEventDestroy(h->ev_p[c]);
+      if (c < 4 && h->ev_p[c]) cudaEventDestroy(h->ev_p[c]);
     }
     if (h->ev_fork) cudaEventDestroy(h->ev_fork);
     for (auto& e : h->ev_t)

@@ -23,9 +23,9 @@ constexpr uint8_t CLS_LIGHT_PATH = 8;
 // Light (tile) kernel geometry.
 constexpr int TINY_MAX = 32;          // class boundaries for statistics only (same kernel)
 constexpr int LIGHTC_MAX = 256;
-constexpr int TILE_PMAX = 4096;       // products per tile: tile capacity + light threshold <= this
+constexpr int TILE_PMAX = 3072;       // products per tile: tile capacity + light threshold <= this
 constexpr int TILE_CAP_DEFAULT = 2048;
-constexpr int LIGHT_MAX_DEFAULT = 2048;
+constexpr int LIGHT_MAX_DEFAULT = 1024;
 constexpr int TILE_NT = 256;          // threads per tile block
 constexpr int TILE_RM = 512;          // light rows per batch
 constexpr int TILE_BK = 4;            // expected products per bucket
@@ -35,9 +35,15 @@ constexpr int HEAVY_CAP = 8192;       // largest f of the register-cached bitmap
 constexpr int HEAVY1_CAP = 4096;      // ... 512-thread blocks, two per SM
 constexpr int BMP_NT = 1024;
 constexpr int BMP_NT_S = 512;
-// Numeric window kernel: outputs per window.
-constexpr int NUM_W = 4096;
+// Numeric kernel.  Rows of C with c_i <= NUM_CS are grouped into row-aligned windows of
+// < NUM_WS outputs (cut where a row crosses a multiple of NUM_WS - NUM_CS); longer rows are units
+// of NUM_WS outputs each (segments).
+constexpr int NUM_WS = 2048;
+constexpr int NUM_CS = 512;
 constexpr int NUM_NT = 256;
+constexpr int NUM_WDUP = 512;   // queued non-first products per window (more: a second pass)
+constexpr int NUM_LDUP = 512;   // ... per large-row pass in shared memory, then
+constexpr int NUM_GDUP = 1 << 16;  // ... in the block's global overflow queue
 constexpr unsigned RFLAG = 0x80000000u;  // R: first occurrence of its column in the row
 
 __device__ __forceinline__ unsigned lanemask_lt() {
@@ -135,6 +141,38 @@ struct Group {
     }
   }
 };
+
+// Predicated global loads that the compiler may not sink below later branches: a run of them is
+// issued back to back, so their latencies overlap (plain loads used only under a data-dependent
+// branch get moved under it, serialising R -> B-value -> B-column round trips).
+__device__ __forceinline__ int ldp_s32(const int* p, bool pred, int dflt = 0) {
+  int v = dflt;
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q ld.global.nc.b32 %0, [%1]; }" : "+r"(v) : "l"(p), "r"((int)pred));
+  return v;
+}
+__device__ __forceinline__ unsigned ldp_u32_stream(const unsigned* p, bool pred, unsigned dflt = 0) {
+  unsigned v = dflt;
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q ld.global.nc.L1::no_allocate.b32 %0, [%1]; }"
+               : "+r"(v) : "l"(p), "r"((int)pred));
+  return v;
+}
+__device__ __forceinline__ double ldp_val(const double* p, bool pred) {
+  double v = 0.0;
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q ld.global.nc.f64 %0, [%1]; }" : "+d"(v) : "l"(p), "r"((int)pred));
+  return v;
+}
+__device__ __forceinline__ float ldp_val(const float* p, bool pred) {
+  float v = 0.f;
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q ld.global.nc.f32 %0, [%1]; }" : "+f"(v) : "l"(p), "r"((int)pred));
+  return v;
+}
+
+__device__ __forceinline__ int4 ldp_v4(const int4* p, bool pred) {
+  int4 v = make_int4(0, 0, 0, 0);
+  asm volatile("{ .reg .pred q; setp.ne.b32 q, %4, 0; @q ld.global.nc.v4.s32 {%0, %1, %2, %3}, [%5]; }"
+               : "+r"(v.x), "+r"(v.y), "+r"(v.z), "+r"(v.w) : "r"((int)pred), "l"(p));
+  return v;
+}
 
 // Largest r in [0, n) with a[r] <= x, given a non-decreasing and a[0] <= x.
 __device__ __forceinline__ int upper_idx(const int* a, int n, int x) {

@@ -9,10 +9,11 @@
 //   symbolic   k_light_rank (tiles of light rows) and k_bitmap_rank (heavy rows) compute, for
 //              every product of row i, its rank among the distinct columns of C(i,:) plus a
 //              first-occurrence flag: R[Ro_i + j] = rank | RFLAG·first.  c_i = #distinct.
-//   numeric    k_numeric: windows of NUM_W consecutive outputs of C; every product of the
-//              window's rows is scattered by its rank into shared memory and the window is
-//              written out coalesced (the Phase IV merge of PAPER.md L154-156, with the sort
-//              moved to the symbolic phase so numeric re-runs are a stream over R).
+//   plan       k_cut_count / k_cut_write: row-aligned output windows of C (end of symbolic)
+//   numeric    k_num_windows / k_num_large: every product of a window's rows is scattered by
+//              its rank into shared memory and the window is written out coalesced (the
+//              Phase IV merge of PAPER.md L154-156, with the sort moved to the symbolic phase
+//              so numeric re-runs are a stream over R).
 #pragma once
 #include "common.cuh"
 
@@ -39,6 +40,10 @@ struct Small {
   int err;
   int r_ok;                 // R capacity sufficient (written by k_tiles)
   int amax;                 // longest row of A
+  int nwunits;              // numeric units: windows
+  int nlunits;              //   large rows
+  int ea0;                  // first A entry of this rank's rows
+  int lqhead;               // large-row numeric kernel: queue head
   long long heavy_total;    // products of heavy rows (R offsets of heavy rows, relative)
   long long fr;             // products needing R (light + heavy)
   unsigned long long hist[65];
@@ -62,26 +67,36 @@ struct SymProb {
   int lgN;                  // ceil(log2 N), N = columns of B
 };
 
+// Output window of the numeric phase: starts at C position pos (local), first row `row`.
+struct Cut {
+  long long pos;
+  int row;
+  int pad;
+};
+
+// Numeric work unit: outputs [lo, lo + c) of C (local positions) from local A entries [ea, eb).
+struct __align__(16) Unit {
+  long long lo;
+  int ea, eb, c, pad;
+};
+
 // Problem view of the numeric kernel.
 template <typename V>
 struct NumProb {
-  const int* __restrict__ rpA;
-  const int* __restrict__ colA;
   const V* __restrict__ valA;
-  const int* __restrict__ rpB;
   const int* __restrict__ colB;
   const V* __restrict__ valB;
-  const int* __restrict__ rowA;   // global row of each A entry
-  const int* __restrict__ Pe;     // in-row product offset of each A entry
-  const long long* __restrict__ Ro;
   const unsigned* __restrict__ R;
-  const long long* __restrict__ crow;
-  const int* __restrict__ wrow;   // first local row of each window
+  const int4* __restrict__ rec0;     // per local A entry: {B start, length, R index lo, hi}
+  const int4* __restrict__ rec1;     //   {C offset of its row lo, hi, first rank, last rank}
+  const Unit* __restrict__ wunits;
+  const Unit* __restrict__ lunits;
+  const Small* small;                // unit counts, ea0
+  int* lqhead;                       // large-row kernel: dynamic queue head
+  int* gq_pos;                       //   per-block overflow queues of non-first products
+  V* gq_val;                         //   (NUM_GDUP entries per block)
   int* ccol;
   V* cval;
-  long long nnzC;
-  int nwin;
-  int row_begin, mloc;
 };
 
 // analysis.cu
@@ -118,11 +133,19 @@ int heavy_occupancy(int bin);
 cudaError_t launch_heavy_rank(int bin, cudaStream_t st, int grid, const SymProb& P, const int* list,
                               const int* count, long long N);
 
-// k_numeric.cu — numeric phase.
+// k_numeric.cu — numeric plan (end of symbolic) and numeric phase.
+cudaError_t launch_plan(cudaStream_t st, int sms, const long long* crow, int mloc, const int* rpA, const int* colA,
+                        const int* rpB, const int* rowA, const int* Pe, const long long* Ro, const unsigned* R, int rb,
+                        int re, long long nnzA_upper, int* cnt, long long* coff, long long* scan_tmp, Cut* cuts,
+                        Unit* wunits, Unit* lunits, int lcap, int4* rec0, int4* rec1, Small* small);
+int plan_launches(long long mloc);
 template <typename V>
 cudaError_t numeric_configure();
-cudaError_t launch_window_rows(cudaStream_t st, const long long* crow, int mloc, int* wrow, int nwin);
 template <typename V>
-cudaError_t launch_numeric(cudaStream_t st, const NumProb<V>& P);
+int numeric_occupancy(int which);  // 0: windows, 1: large A, 2: large B
+template <typename V>
+cudaError_t launch_num_windows(cudaStream_t st, int grid, const NumProb<V>& P);
+template <typename V>
+cudaError_t launch_num_large(cudaStream_t st, int grid, bool cfgB, const NumProb<V>& P);
 
 }  // namespace spg

@@ -90,7 +90,7 @@ struct spg_ctx {
   cudaEvent_t ev_fork = nullptr, ev_join[6] = {};
   cudaEvent_t ev_t[8] = {};
   cudaEvent_t ev_p[4] = {};  // light path start/end, heavy path start/end
-  int occ_light = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1, occ_large[2] = {1, 1};
+  int occ_light = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1, occ_large[3] = {1, 1, 1};
   int large_cfg = 0;  // numeric large-row kernel configuration (SPG_LARGE_CFG=1: B)
   // cached symbolic state
   bool sym_ok = false;
@@ -488,8 +488,8 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
     P.ccol = C_col; P.cval = (V*)C_val;
     const bool conc = h->concurrent != 0 && h->nlunits > 0 && h->nwunits > 0;
     if (h->nlunits > 0) {
-      const bool cfgB = h->large_cfg != 0;
-      int grid = h->occ_large[cfgB] * h->sms;
+      const int cfg = h->large_cfg;
+      int grid = h->occ_large[cfg] * h->sms;
       if (h->nlunits < grid) grid = h->nlunits;
       CK(h->gq.ensure((size_t)grid * NUM_GDUP * (sizeof(int) + sizeof(V))));
       P.gq_pos = h->gq.as<int>();
@@ -499,7 +499,7 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
         CK(cudaEventRecord(h->ev_fork, h->stream));
         CK(cudaStreamWaitEvent(h->aux[4], h->ev_fork, 0));
       }
-      CK(launch_num_large<V>(conc ? h->aux[4] : h->stream, grid, cfgB, P));
+      CK(launch_num_large<V>(conc ? h->aux[4] : h->stream, grid, cfg, P));
       h->launches++;
     }
     if (h->nwunits > 0) {
@@ -564,9 +564,9 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
   }
   h->occ_light = light_occupancy();
   h->occ_num = dtype == SPG_FP64 ? numeric_occupancy<double>(0) : numeric_occupancy<float>(0);
-  for (int x = 0; x < 2; ++x)
+  for (int x = 0; x < 3; ++x)
     h->occ_large[x] = dtype == SPG_FP64 ? numeric_occupancy<double>(1 + x) : numeric_occupancy<float>(1 + x);
-  h->large_cfg = getenv("SPG_LARGE_CFG") != nullptr && getenv("SPG_LARGE_CFG")[0] == '1';
+  if (const char* lc = getenv("SPG_LARGE_CFG")) h->large_cfg = (lc[0] >= '0' && lc[0] <= '2') ? lc[0] - '0' : 0;
   for (int b = 0; b < NUM_BINS; ++b) h->occ_heavy[b] = heavy_occupancy(b);
   cudaGetLastError();
   *out = h;

@@ -337,7 +337,7 @@ __device__ __forceinline__ void num_chunk_products(const NumProb<V>& P, unsigned
       }
       const int* cb = P.colB + lc.x;
       const V* vb = P.valB + lc.x;
-      constexpr int U = 4;
+      constexpr int U = NT >= 1024 ? 2 : 4;
       for (int ob = o0; ob < o1; ob += 32 * U) {
         unsigned rv[U];
         int cB[U];
@@ -509,13 +509,17 @@ __global__ void __launch_bounds__(NT, MINB) k_num_large(NumProb<V> P) {
 
 // Large-row kernel configurations: A = one 512-thread block per SM staging NUM_LS_A outputs;
 // B = two per SM staging NUM_LS_B (more rows in flight, more multi-pass rows).
+// C = one 1024-thread block per SM staging NUM_LS_A outputs.
 constexpr int NUM_LS_A = 12288, NUM_LS_B = 5120;
 #define NUM_LARGE_A k_num_large<V, 512, NUM_LS_A, 1>
 #define NUM_LARGE_B k_num_large<V, 512, NUM_LS_B, 2>
+#define NUM_LARGE_C k_num_large<V, 1024, NUM_LS_A, 1>
 template <typename V>
-constexpr int large_smem(bool b) {
-  return b ? NumSmem<V, 512, NUM_LS_B, NUM_LDUP>::bytes : NumSmem<V, 512, NUM_LS_A, NUM_LDUP>::bytes;
+constexpr int large_smem(int cfg) {
+  return cfg == 1 ? NumSmem<V, 512, NUM_LS_B, NUM_LDUP>::bytes
+                  : cfg == 2 ? NumSmem<V, 1024, NUM_LS_A, NUM_LDUP>::bytes : NumSmem<V, 512, NUM_LS_A, NUM_LDUP>::bytes;
 }
+static_assert(NumSmem<double, 1024, NUM_LS_A, NUM_LDUP>::bytes + 2048 <= 227 * 1024, "large-row kernel C");
 
 static_assert(NumSmem<double, 512, NUM_LS_A, NUM_LDUP>::bytes + 1024 <= 227 * 1024, "large-row kernel A");
 static_assert(2 * (NumSmem<double, 512, NUM_LS_B, NUM_LDUP>::bytes + 1024) <= 228 * 1024, "large-row kernel B");
@@ -548,9 +552,11 @@ cudaError_t numeric_configure() {
   cudaError_t e = cudaFuncSetAttribute(k_num_windows<V>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        NumSmem<V, NUM_NT, NUM_WS, NUM_WDUP>::bytes);
   if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(NUM_LARGE_A, cudaFuncAttributeMaxDynamicSharedMemorySize, large_smem<V>(false));
+    e = cudaFuncSetAttribute(NUM_LARGE_A, cudaFuncAttributeMaxDynamicSharedMemorySize, large_smem<V>(0));
   if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(NUM_LARGE_B, cudaFuncAttributeMaxDynamicSharedMemorySize, large_smem<V>(true));
+    e = cudaFuncSetAttribute(NUM_LARGE_B, cudaFuncAttributeMaxDynamicSharedMemorySize, large_smem<V>(1));
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(NUM_LARGE_C, cudaFuncAttributeMaxDynamicSharedMemorySize, large_smem<V>(2));
   return e;
 }
 
@@ -560,9 +566,11 @@ int numeric_occupancy(int which) {
   if (which == 0)
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_num_windows<V>, NUM_NT, NumSmem<V, NUM_NT, NUM_WS, NUM_WDUP>::bytes);
   else if (which == 1)
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, NUM_LARGE_A, 512, large_smem<V>(false));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, NUM_LARGE_A, 512, large_smem<V>(0));
+  else if (which == 2)
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, NUM_LARGE_B, 512, large_smem<V>(1));
   else
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, NUM_LARGE_B, 512, large_smem<V>(true));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, NUM_LARGE_C, 1024, large_smem<V>(2));
   return nb < 1 ? 1 : nb;
 }
 
@@ -574,10 +582,11 @@ cudaError_t launch_num_windows(cudaStream_t st, int grid, const NumProb<V>& P) {
 }
 
 template <typename V>
-cudaError_t launch_num_large(cudaStream_t st, int grid, bool cfgB, const NumProb<V>& P) {
+cudaError_t launch_num_large(cudaStream_t st, int grid, int cfg, const NumProb<V>& P) {
   if (grid <= 0) return cudaSuccess;
-  if (cfgB) NUM_LARGE_B<<<grid, 512, large_smem<V>(true), st>>>(P);
-  else NUM_LARGE_A<<<grid, 512, large_smem<V>(false), st>>>(P);
+  if (cfg == 1) NUM_LARGE_B<<<grid, 512, large_smem<V>(1), st>>>(P);
+  else if (cfg == 2) NUM_LARGE_C<<<grid, 1024, large_smem<V>(2), st>>>(P);
+  else NUM_LARGE_A<<<grid, 512, large_smem<V>(0), st>>>(P);
   return cudaGetLastError();
 }
 
@@ -585,7 +594,7 @@ cudaError_t launch_num_large(cudaStream_t st, int grid, bool cfgB, const NumProb
   template cudaError_t numeric_configure<V>();                                               \
   template int numeric_occupancy<V>(int);                                                    \
   template cudaError_t launch_num_windows<V>(cudaStream_t, int, const NumProb<V>&);          \
-  template cudaError_t launch_num_large<V>(cudaStream_t, int, bool, const NumProb<V>&);
+  template cudaError_t launch_num_large<V>(cudaStream_t, int, int, const NumProb<V>&);
 INST(double)
 INST(float)
 #undef INST

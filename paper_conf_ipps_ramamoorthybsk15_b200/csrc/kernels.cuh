@@ -142,10 +142,10 @@ int plan_launches(long long mloc);
 template <typename V>
 cudaError_t numeric_configure();
 template <typename V>
-int numeric_occupancy(int which);  // 0: windows, 1: large A, 2: large B
+int numeric_occupancy(int which);  // 0: windows, 1..3: large-row kernel configuration 0..2
 template <typename V>
 cudaError_t launch_num_windows(cudaStream_t st, int grid, const NumProb<V>& P);
 template <typename V>
-cudaError_t launch_num_large(cudaStream_t st, int grid, bool cfgB, const NumProb<V>& P);
+cudaError_t launch_num_large(cudaStream_t st, int grid, int cfg, const NumProb<V>& P);
 
 }  // namespace spg

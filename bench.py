@@ -369,12 +369,12 @@ def run_ours(args):
                        "numeric_gflops": 2.0 * int(st["flops"]) / (num_ms * 1e-3) / 1e9,
                        "symbolic_path_ms": dict(zip(["analysis", "light", "heavy"], (path_ms / K).round(4).tolist())),
                        "tiles": int(st["tiles"]), "fallback_rows": int(st["fallback_rows"]),
-                       "rank_bytes": int(st["rank_bytes"]),
+                       "plan_bytes": int(st["rank_bytes"]),
                        "class_rows": dict(zip(spg.CLASS_NAMES, stl["class_rows"])),
                        "class_flops": dict(zip(spg.CLASS_NAMES, stl["class_flops"]))},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                         "kernel": "numeric phase (k_window_rows + k_numeric: rank-scatter windows)",
+                         "kernel": "numeric phase (k_numeric gather stream + k_numeric_dup)",
                          "algorithmic_bytes": int(alg_bytes)},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clocks,
         }

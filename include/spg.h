@@ -25,8 +25,8 @@
  *
  * Ownership and threading
  *   - The caller owns A, B and C.  The handle owns all workspace (row flops, class lists,
- *     the per-product rank array R of 4 bytes per intermediate product, the NCCL
- *     communicator) and caches the symbolic analysis that spg_spgemm_numeric consumes.
+ *     the gather plan — 8 bytes per intermediate product of the non-SINGLE rows plus a
+ *     16-byte dup entry per repeated column — and the NCCL communicator) and caches the symbolic analysis that spg_spgemm_numeric consumes.
  *     spg_spgemm_free releases everything.
  *   - A handle is bound to one device and one CUDA stream and is not thread-safe;
  *     several handles may coexist.
@@ -123,7 +123,7 @@ typedef struct {
   int64_t tiles;                          /* light tiles of the last symbolic call       */
   int64_t fallback_rows;                  /* light rows moved to the heavy path (clustered
                                              columns)                                    */
-  int64_t rank_bytes;                     /* bytes of the per-product rank array R       */
+  int64_t rank_bytes;                     /* bytes of the gather plan (EQ + dup list)    */
   float ms_analysis;                      /* SPG_OPT_TIMING: row analysis + classify     */
   float ms_symbolic;                      /*   symbolic kernels + row_ptr scan            */
   float ms_numeric;                       /*   numeric (last numeric call)                */
@@ -153,9 +153,11 @@ const char* spg_version(void);
 spg_status spg_spgemm_symbolic(spg_handle h, const spg_csr* A, const spg_csr* B, int64_t* C_row_ptr,
                                int64_t* nnzC, int32_t* row_begin, int32_t* row_end);
 
-/* Numeric phase: every product is scattered into its output slot, found by symbolic (the rank
- * of its column within its row of C), so C comes out sorted and compacted.  Requires a preceding symbolic call on
- * this handle with the same A/B structure pointers.  C_col_idx: device int32[nnzC];
+/* Numeric phase (Phase IV "add like-tuples, compact"): symbolic sorted every
+ * row's products and left, for each output of C, the A and B entry of its first product (plus a
+ * list of the repeated ones); numeric streams C in output order, C(i,r) = a·b, then adds the
+ * repeats — C comes out sorted and compacted.  Requires a preceding symbolic call on this handle
+ * with the same A/B structure pointers and the same C_row_ptr contents.  C_col_idx: device int32[nnzC];
  * C_vals: device fp32/fp64[nnzC].  Values of A and B may differ from the symbolic call
  * (re-run numeric on new values with the same structure).  Asynchronous. */
 spg_status spg_spgemm_numeric(spg_handle h, const spg_csr* A, const spg_csr* B, const int64_t* C_row_ptr,

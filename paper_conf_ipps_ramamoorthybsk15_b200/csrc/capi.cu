@@ -80,7 +80,7 @@ struct spg_ctx {
   int light_max = LIGHT_MAX_DEFAULT, tile_cap = TILE_CAP_DEFAULT, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
   // workspace: analysis (all rows / all A entries), classification (this rank's rows), R, windows
-  DevBuf f, nz, rowA, Pe, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, R, cuts, wunits, lunits, rec0, rec1, gq, Pf,
+  DevBuf f, nz, rowA, Pe, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, EQ, fl8, dup, nd, ne, chunk_row, Pf,
       splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
@@ -90,14 +90,14 @@ struct spg_ctx {
   cudaEvent_t ev_fork = nullptr, ev_join[6] = {};
   cudaEvent_t ev_t[8] = {};
   cudaEvent_t ev_p[4] = {};  // light path start/end, heavy path start/end
-  int occ_light = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1, occ_large[3] = {1, 1, 1};
-  int large_cfg = 0;  // numeric large-row kernel configuration (SPG_LARGE_CFG=1: B)
+  int occ_light = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1;
   // cached symbolic state
   bool sym_ok = false;
   SymKey key{};
   int32_t rb = 0, re = 0;
   int64_t nnzC = 0;
-  int nwunits = 0, nlunits = 0, lcap = 0;
+  long long ndup = 0, dupcap = 0;
+  int nch = 0, chcap = 0;
   int counts[NUM_BINS] = {};
   spg_stats stats{};
   bool num_timed = false, paths_timed = false;
@@ -171,7 +171,11 @@ SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* cr
   P.frow = h->f.as<int>();
   P.cls = h->cls.as<uint8_t>();
   P.Ro = h->Ro.as<long long>();
-  P.R = h->R.as<unsigned>();
+  P.EQ = h->EQ.as<int2>();
+  P.dup = h->dup.as<int4>();
+  P.dupn = &h->small.as<Small>()->dupn;
+  P.dupcap = h->dupcap;
+  P.fl8 = h->fl8.as<uint8_t>();
   P.crow = crow;
   P.r_ok = &h->small.as<Small>()->r_ok;
   P.row_begin = h->rb;
@@ -249,10 +253,8 @@ spg_status ensure_ws(spg_handle h, int M, long long nnzA) {
   CK(h->tiles.ensure(m * sizeof(int)));
   CK(h->lists.ensure(m * NUM_BINS * sizeof(int)));
   CK(h->fblist.ensure(m * sizeof(int)));
-  CK(h->cuts.ensure((2 * m + 2) * sizeof(Cut)));
-  CK(h->wunits.ensure((2 * m + 2) * sizeof(Unit)));
-  CK(h->rec0.ensure(na * sizeof(int4)));
-  CK(h->rec1.ensure(na * sizeof(int4)));
+  CK(h->nd.ensure(m * sizeof(long long)));
+  CK(h->ne.ensure(m * sizeof(int)));
   CK(h->small.ensure(sizeof(Small)));
   CK(h->scan_tmp.ensure(scan_tmp_elems((long long)m + 1) * sizeof(long long)));
   return SPG_OK;
@@ -362,8 +364,9 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   long long Mloc = 0;
   Small* ds = h->small.as<Small>();
   long long* crow = reinterpret_cast<long long*>(C_row_ptr);
-  // Two attempts at most: the first call (or a larger product count) finds R too small — the
-  // kernels then skip their work, R is grown to the exact size read back, and the pass reruns.
+  // The first call (or a larger product count) finds the gather plan too small — the kernels then
+  // skip their work, EQ is grown to the exact size read back, and the pass reruns; likewise a dup
+  // list that overflowed.
   for (int attempt = 0;; ++attempt) {
     h->launches = 0;
     if (h->timing) CK(cudaEventRecord(h->ev_t[0], h->stream));
@@ -390,24 +393,22 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm,
                        h->cls.as<uint8_t>(), h->fl.as<int>(), h->Ro.as<long long>(), L3, ds, crow));
     CK(launch_incl_scan<int>(h->stream, h->fl.as<int>(), PL + 1, Mloc, h->scan_tmp.as<long long>()));
-    const long long r_cap = h->R.p ? (long long)(h->R.cap / sizeof(unsigned)) : 0;
+    long long r_cap = h->EQ.p && h->fl8.p ? (long long)(h->EQ.cap / sizeof(int2)) : 0;
+    if (r_cap > (long long)h->fl8.cap) r_cap = (long long)h->fl8.cap;
     CK(launch_tiles(h->stream, h->sms, h->f.as<int>(), h->rb, h->re, h->tile_cap, h->cls.as<uint8_t>(), PL,
                     h->Ro.as<long long>(), h->tflag.as<uint8_t>(), h->tiles.as<int>(), ds, r_cap));
     h->launches += (Mloc > 0) + scan_launches(Mloc) + 1;
     if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));
     if ((s = run_sym(h, A, B, crow)) != SPG_OK) return s;
     CK(launch_incl_scan<long long>(h->stream, crow + 1, crow + 1, Mloc, h->scan_tmp.as<long long>()));
-    // numeric plan: row-aligned units and per-entry run records (cut counts in fl, their prefix in
-    // PL — both free now)
-    // segment units of long rows: capacity from the last call (the count is read back; a larger
-    // need reruns the plan below)
-    if (h->lcap < Mloc + 1) h->lcap = (int)(Mloc + 1);
-    CK(h->lunits.ensure((size_t)h->lcap * sizeof(Unit)));
-    CK(launch_plan(h->stream, h->sms, crow, (int)Mloc, A->row_ptr, A->col_idx, B->row_ptr, h->rowA.as<int>(),
-                   h->Pe.as<int>(), h->Ro.as<long long>(), h->R.as<unsigned>(), h->rb, h->re, A->nnz,
-                   h->fl.as<int>(), PL, h->scan_tmp.as<long long>(), h->cuts.as<Cut>(), h->wunits.as<Unit>(),
-                   h->lunits.as<Unit>(), h->lcap, h->rec0.as<int4>(), h->rec1.as<int4>(), ds));
-    h->launches += scan_launches(Mloc) + plan_launches(Mloc);
+    // numeric plan: per-row EQ-to-C offsets and chunk -> row (capacity from the last call; a
+    // larger need reruns the plan below)
+    if (h->chcap < 2) h->chcap = 2;
+    CK(h->chunk_row.ensure((size_t)h->chcap * sizeof(int)));
+    CK(launch_plan(h->stream, h->sms, crow, (int)Mloc, A->row_ptr, A->col_idx, B->row_ptr, h->cls.as<uint8_t>(),
+                   h->Ro.as<long long>(), h->rb, h->nd.as<long long>(), h->ne.as<int>(), h->chunk_row.as<int>(),
+                   h->chcap, ds));
+    h->launches += scan_launches(Mloc) + (Mloc > 0);
     if (h->timing) CK(cudaEventRecord(h->ev_t[2], h->stream));
     CK(cudaMemcpyAsync(&h->hr->small, ds, sizeof(Small), cudaMemcpyDeviceToHost, h->stream));
     CK(cudaMemcpyAsync(&h->hr->nnz, crow + Mloc, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
@@ -415,26 +416,38 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     const Small& hs = h->hr->small;
     if (hs.err & 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "A has a column index outside [0, B.nrows)");
     if (hs.err & 2) return setf(h, SPG_ERR_INDEX_OVERFLOW, "a row of A has >= 2^31 intermediate products");
-    if (hs.r_ok && hs.nlunits > h->lcap) {  // more long-row segments than room: grow, rerun the plan
-      h->lcap = hs.nlunits + 64;
-      CK(h->lunits.ensure((size_t)h->lcap * sizeof(Unit)));
-      CK(cudaMemsetAsync(&ds->nwunits, 0, 2 * sizeof(int), h->stream));
-      CK(launch_plan(h->stream, h->sms, crow, (int)Mloc, A->row_ptr, A->col_idx, B->row_ptr, h->rowA.as<int>(),
-                     h->Pe.as<int>(), h->Ro.as<long long>(), h->R.as<unsigned>(), h->rb, h->re, A->nnz,
-                     h->fl.as<int>(), PL, h->scan_tmp.as<long long>(), h->cuts.as<Cut>(), h->wunits.as<Unit>(),
-                     h->lunits.as<Unit>(), h->lcap, h->rec0.as<int4>(), h->rec1.as<int4>(), ds));
-      h->launches += plan_launches(Mloc);
-      CK(cudaMemcpyAsync(&h->hr->small, ds, sizeof(Small), cudaMemcpyDeviceToHost, h->stream));
+    const bool dup_ok = (long long)hs.dupn <= h->dupcap;
+    if (hs.r_ok && dup_ok && hs.nch_need > h->chcap) {  // more chunks than room: grow, rerun the plan
+      h->chcap = hs.nch_need + 64;
+      CK(h->chunk_row.ensure((size_t)h->chcap * sizeof(int)));
+      CK(launch_plan(h->stream, h->sms, crow, (int)Mloc, A->row_ptr, A->col_idx, B->row_ptr, h->cls.as<uint8_t>(),
+                     h->Ro.as<long long>(), h->rb, h->nd.as<long long>(), h->ne.as<int>(), h->chunk_row.as<int>(),
+                     h->chcap, ds));
+      h->launches += (Mloc > 0);
       CK(cudaStreamSynchronize(h->stream));
     }
+    if (hs.r_ok && !dup_ok && attempt < 3) {  // dup list too small: grow to the exact need, rerun
+      h->dupcap = (long long)hs.dupn + 1024;
+      CK(h->dup.ensure((size_t)h->dupcap * sizeof(int4)));
+      continue;
+    }
+    if (!dup_ok && hs.r_ok) return setf(h, SPG_ERR_OUT_OF_MEMORY, "dup list could not be sized");
     if (hs.r_ok || attempt > 0) break;
-    CK(h->R.ensure((size_t)(hs.fr > 0 ? hs.fr : 1) * sizeof(unsigned)));
+    {  // gather plan, first-claim flags and a first dup list sized from the product count
+      const size_t fr = (size_t)(hs.fr > 0 ? hs.fr : 1);
+      CK(h->EQ.ensure(fr * sizeof(int2)));
+      CK(h->fl8.ensure(fr));
+      if (h->dupcap < (long long)(fr / 8 + 1024)) {
+        h->dupcap = (long long)(fr / 8 + 1024);
+        CK(h->dup.ensure((size_t)h->dupcap * sizeof(int4)));
+      }
+    }
   }
   const Small& hs = h->hr->small;
-  if (!hs.r_ok && hs.fr > 0) return setf(h, SPG_ERR_OUT_OF_MEMORY, "rank array could not be sized");
+  if (!hs.r_ok && hs.fr > 0) return setf(h, SPG_ERR_OUT_OF_MEMORY, "gather plan could not be sized");
   h->nnzC = h->hr->nnz;
-  h->nwunits = hs.nwunits;
-  h->nlunits = hs.nlunits;
+  h->ndup = (long long)hs.dupn;
+  h->nch = (int)((h->nnzC + NUM_CH - 1) / NUM_CH);
   for (int b = 0; b < NUM_BINS; ++b) h->counts[b] = hs.counts[b];
   spg_stats& st = h->stats;
   std::memset(&st, 0, sizeof st);
@@ -452,7 +465,7 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   for (int b = 0; b < 65; ++b) st.bin_hist[b] = (int64_t)hs.hist[b];
   st.tiles = hs.ntiles;
   st.fallback_rows = hs.fb[0];
-  st.rank_bytes = (int64_t)hs.fr * (int64_t)sizeof(unsigned);
+  st.rank_bytes = (int64_t)h->nnzC * (int64_t)sizeof(int2) + h->ndup * (int64_t)sizeof(int4);
   st.launches_symbolic = h->launches;
   if (h->timing) {
     cudaEventElapsedTime(&st.ms_analysis, h->ev_t[0], h->ev_t[1]);
@@ -474,44 +487,29 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
 template <typename V>
 spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const int64_t* C_row_ptr, int32_t* C_col,
                         void* C_val) {
-  (void)C_row_ptr;  // the symbolic plan already holds every row's C offset (run records)
   if (h->timing) CK(cudaEventRecord(h->ev_t[3], h->stream));
   h->launches = 0;
   if (h->nnzC > 0) {
-    Small* ds = h->small.as<Small>();
     NumProb<V> P;
     P.valA = (const V*)A->vals;
-    P.colB = B->col_idx; P.valB = (const V*)B->vals;
-    P.R = h->R.as<unsigned>(); P.rec0 = h->rec0.as<int4>(); P.rec1 = h->rec1.as<int4>();
-    P.wunits = h->wunits.as<Unit>(); P.lunits = h->lunits.as<Unit>(); P.small = ds;
-    P.lqhead = &ds->lqhead; P.gq_pos = nullptr; P.gq_val = nullptr;
-    P.ccol = C_col; P.cval = (V*)C_val;
-    const bool conc = h->concurrent != 0 && h->nlunits > 0 && h->nwunits > 0;
-    if (h->nlunits > 0) {
-      const int cfg = h->large_cfg;
-      int grid = h->occ_large[cfg] * h->sms;
-      if (h->nlunits < grid) grid = h->nlunits;
-      CK(h->gq.ensure((size_t)grid * NUM_GDUP * (sizeof(int) + sizeof(V))));
-      P.gq_pos = h->gq.as<int>();
-      P.gq_val = reinterpret_cast<V*>(P.gq_pos + (size_t)grid * NUM_GDUP);
-      CK(cudaMemsetAsync(&ds->lqhead, 0, sizeof(int), h->stream));
-      if (conc) {
-        CK(cudaEventRecord(h->ev_fork, h->stream));
-        CK(cudaStreamWaitEvent(h->aux[4], h->ev_fork, 0));
-      }
-      CK(launch_num_large<V>(conc ? h->aux[4] : h->stream, grid, cfg, P));
-      h->launches++;
-    }
-    if (h->nwunits > 0) {
-      int grid = h->occ_num * h->sms;
-      if (h->nwunits < grid) grid = h->nwunits;
-      CK(launch_num_windows<V>(h->stream, grid, P));
-      h->launches++;
-    }
-    if (conc) {
-      CK(cudaEventRecord(h->ev_join[4], h->aux[4]));
-      CK(cudaStreamWaitEvent(h->stream, h->ev_join[4], 0));
-    }
+    P.colB = B->col_idx;
+    P.valB = (const V*)B->vals;
+    P.EQ = h->EQ.as<int2>();
+    P.dup = h->dup.as<int4>();
+    P.crow = reinterpret_cast<const long long*>(C_row_ptr);
+    P.nd = h->nd.as<long long>();
+    P.ne = h->ne.as<int>();
+    P.chunk_row = h->chunk_row.as<int>();
+    P.nnz = h->nnzC;
+    P.ndup = h->ndup;
+    P.nch = h->nch;
+    P.mloc = h->re - h->rb;
+    P.ccol = C_col;
+    P.cval = (V*)C_val;
+    int grid = h->occ_num * h->sms;
+    if (h->nch < grid) grid = h->nch;
+    CK(launch_numeric<V>(h->stream, grid, P));
+    h->launches += (h->nch > 0) + (h->ndup > 0);
   }
   h->stats.launches_numeric = h->launches;
   if (h->timing) {
@@ -563,10 +561,7 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     return SPG_ERR_CUDA;
   }
   h->occ_light = light_occupancy();
-  h->occ_num = dtype == SPG_FP64 ? numeric_occupancy<double>(0) : numeric_occupancy<float>(0);
-  for (int x = 0; x < 3; ++x)
-    h->occ_large[x] = dtype == SPG_FP64 ? numeric_occupancy<double>(1 + x) : numeric_occupancy<float>(1 + x);
-  if (const char* lc = getenv("SPG_LARGE_CFG")) h->large_cfg = (lc[0] >= '0' && lc[0] <= '2') ? lc[0] - '0' : 0;
+  h->occ_num = dtype == SPG_FP64 ? numeric_occupancy<double>() : numeric_occupancy<float>();
   for (int b = 0; b < NUM_BINS; ++b) h->occ_heavy[b] = heavy_occupancy(b);
   cudaGetLastError();
   *out = h;
@@ -584,7 +579,7 @@ spg_status upload(spg_handle h, DevBuf& b, const void* src, size_t bytes) {
 // ===================================== ABI =====================================================
 extern "C" {
 
-const char* spg_version(void) { return "spg 0.2 (sm_100a, heavy/light-row Gustavson SpGEMM, rank-scatter numeric)"; }
+const char* spg_version(void) { return "spg 0.2 (sm_100a, heavy/light-row Gustavson SpGEMM, gather-plan numeric)"; }
 
 spg_status spg_create(spg_handle* h, int device, void* cuda_stream, spg_dtype dtype) {
   return create_common(h, device, cuda_stream, dtype);
@@ -597,7 +592,7 @@ spg_status spg_spgemm_free(spg_handle h) {
     cudaStreamSynchronize(h->stream);
     DevBuf* bufs[] = {&h->f,     &h->nz,    &h->rowA,   &h->Pe,    &h->cls,    &h->fl,  &h->Ro,
                       &h->PL,    &h->tflag, &h->tiles,  &h->lists, &h->fblist, &h->small, &h->scan_tmp,
-                      &h->R,     &h->cuts,  &h->wunits, &h->lunits, &h->rec0, &h->rec1, &h->gq, &h->Pf,     &h->splits, &h->iota,  &h->ones, &h->crow_tmp};
+                      &h->EQ,    &h->fl8,   &h->dup,    &h->nd,     &h->ne,   &h->chunk_row, &h->Pf,     &h->splits, &h->iota,  &h->ones, &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
     if (h->canon) spg_spgemm_free(h->canon);

@@ -35,16 +35,6 @@ constexpr int HEAVY_CAP = 8192;       // largest f of the register-cached bitmap
 constexpr int HEAVY1_CAP = 4096;      // ... 512-thread blocks, two per SM
 constexpr int BMP_NT = 1024;
 constexpr int BMP_NT_S = 512;
-// Numeric kernel.  Rows of C with c_i <= NUM_CS are grouped into row-aligned windows of
-// < NUM_WS outputs (cut where a row crosses a multiple of NUM_WS - NUM_CS); longer rows are units
-// of NUM_WS outputs each (segments).
-constexpr int NUM_WS = 2048;
-constexpr int NUM_CS = 512;
-constexpr int NUM_NT = 256;
-constexpr int NUM_WDUP = 512;   // queued non-first products per window (more: a second pass)
-constexpr int NUM_LDUP = 512;   // ... per large-row pass in shared memory, then
-constexpr int NUM_GDUP = 1 << 16;  // ... in the block's global overflow queue
-constexpr unsigned RFLAG = 0x80000000u;  // R: first occurrence of its column in the row
 
 __device__ __forceinline__ unsigned lanemask_lt() {
   unsigned m;

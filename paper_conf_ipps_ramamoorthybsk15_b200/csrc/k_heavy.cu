@@ -10,12 +10,13 @@
 //           step proportional to the touched words.
 //   build   rank prefixes: an int per 1024 columns and a u16 per 256 columns.
 //   pass 2  rank(col) = prefix + popcount of the <= 8 bitmap words below it in its 256-column
-//           block; R[Ro_i + j] = rank | RFLAG·first, written coalesced in product order.
+//           block; the first claimer writes {A entry, B entry} to the gather plan at
+//           EQ[Ro_i + rank], every other product goes to the dup list.
 //   c_i     = claimed bits (summed over column tiles).
 // HEAVY rows (f <= 8192, one gather chunk) keep their products (column) in registers across
 // the passes and their first-occurrence flags in a shared bit array; other rows (HUGE, and rows
-// the light kernel handed over) re-gather columns per pass and keep the flag in R itself
-// between pass 1 and pass 2.  Products are visited in 32-product warp windows (coalesced within
+// the light kernel handed over) re-gather columns per pass and keep the flag in a global byte
+// per product (fl8) between pass 1 and pass 2.  Products are visited in 32-product warp windows (coalesced within
 // a B row); the run of each lane comes from a REDUX.OR mask of run starts.
 #include "kernels.cuh"
 
@@ -29,7 +30,7 @@ __host__ __device__ constexpr int al16(int x) { return (x + 15) & ~15; }
 
 template <int NT>
 __host__ __device__ constexpr int bmp_fixed_bytes() {
-  return 2 * al16((NT + 1) * 4) + al16(BMP_CTCAP * 2);
+  return 3 * al16((NT + 1) * 4) + al16(BMP_CTCAP * 2);
 }
 constexpr int BMP_SMEM_L = 226 * 1024;  // 1024-thread blocks, one per SM (static smem on top)
 constexpr int BMP_SMEM_S = 112 * 1024;  // 512-thread blocks, two per SM
@@ -53,7 +54,8 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
   extern __shared__ __align__(16) unsigned char sm[];
   int* seg = reinterpret_cast<int*>(sm);                                   // run -> product offset
   int* sbs = reinterpret_cast<int*>(sm + al16((RCAP + 1) * 4));            // run -> B row start
-  unsigned short* ctab = reinterpret_cast<unsigned short*>(sm + 2 * al16((RCAP + 1) * 4));  // window -> run
+  int* sae = reinterpret_cast<int*>(sm + 2 * al16((RCAP + 1) * 4));      // run -> A entry
+  unsigned short* ctab = reinterpret_cast<unsigned short*>(sm + 3 * al16((RCAP + 1) * 4));  // window -> run
   unsigned char* region = sm + bmp_fixed_bytes<NT>();
   constexpr int REGION = SMEM - bmp_fixed_bytes<NT>();
   __shared__ int scratch[NT / 32 + 1];
@@ -81,7 +83,9 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
     const int i = P.row_begin + li;
     const int pa0 = P.rpA[i], pa1 = P.rpA[i + 1];
     const int f = P.frow[i];
-    unsigned* Rrow = P.R + P.Ro[li];
+    const long long ro = P.Ro[li];
+    int2* EQrow = P.EQ + ro;
+    uint8_t* frow8 = P.fl8 + ro;
     // Column tile: the widest whose structures (and, cached, the flag bits) fit.
     int lw = lwmax;
     while (lw > 10 && bmp_need<MODE>(lw, f) > REGION) --lw;
@@ -112,6 +116,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
       if (L > 0) {
         seg[rk] = off;
         sbs[rk] = bs;
+        sae[rk] = p;
       }
       if (tid == 0) seg[nz] = Lt;
       __syncthreads();
@@ -225,7 +230,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
               const unsigned b = 1u << (lc & 31);
               const unsigned old = atomicOr(&bm[w], b);
               if (old == 0) atomicOr(&l1[w >> 5], 1u << (w & 31));
-              Rrow[cbase + j] = (old & b) ? 0u : RFLAG;
+              frow8[cbase + j] = (old & b) ? 0 : 1;
             }
           });
         }
@@ -268,22 +273,66 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
       }
       const int ctile = pcarry;
       __syncthreads();
-      // ---- pass 2: ranks -> R ---------------------------------------------------------------------
+      // ---- pass 2: ranks -> gather plan (first claimers) and dup list (the others) ---------------
       cbase = 0;
       for (int c = 0; c < nchunks; ++c) {
         if (nchunks > 1) gather(c);
-        for_products([&](int j, int col) {
-          const unsigned lc = (unsigned)(col - lo);
-          if (lc < (unsigned)Wt) {
-            const unsigned r = (unsigned)(out + rank_of(lc));
-            if constexpr (CACHED) {
-              const unsigned fl = (flags[j >> 5] >> (j & 31)) & 1u;
-              Rrow[j] = r | (fl << 31);
-            } else {
-              Rrow[cbase + j] = r | (Rrow[cbase + j] & RFLAG);
+        if constexpr (CACHED) {
+#pragma unroll
+          for (int s = 0; s < BMP_SLOTS; ++s) {
+            const int j0 = warp * 32 + s * NT;
+            if (j0 < Lt) {  // warp-uniform
+              const int r = lane_run(j0);
+              const int j = j0 + lane;
+              const unsigned lc = (unsigned)(cc[s] - lo);
+              const bool in = j < Lt && lc < (unsigned)Wt;
+              bool first = false;
+              int rank = 0, e = 0, q = 0;
+              if (in) {
+                rank = out + rank_of(lc);
+                first = (flags[j >> 5] >> (j & 31)) & 1u;
+                q = sbs[r] + (j - seg[r]);
+                e = sae[r];
+                if (first) EQrow[rank] = make_int2(e, q);
+              }
+              dup_push(P, in && !first, li, rank, e, q);
             }
           }
-        });
+        } else {
+          for (int j00 = warp * 32; j00 < Lt; j00 += BATCH * NT) {
+            int q[BATCH], col[BATCH], rr[BATCH];
+#pragma unroll
+            for (int u = 0; u < BATCH; ++u) {
+              const int j0 = j00 + u * NT;
+              q[u] = -1;
+              rr[u] = 0;
+              if (j0 < Lt) {
+                rr[u] = lane_run(j0);
+                if (j0 + lane < Lt) q[u] = sbs[rr[u]] + (j0 + lane - seg[rr[u]]);
+              }
+            }
+            uint8_t fb[BATCH];
+#pragma unroll
+            for (int u = 0; u < BATCH; ++u) {
+              col[u] = q[u] >= 0 ? P.colB[q[u]] : -1;
+              fb[u] = q[u] >= 0 ? frow8[cbase + j00 + u * NT + lane] : 0;
+            }
+#pragma unroll
+            for (int u = 0; u < BATCH; ++u) {
+              if (j00 + u * NT < Lt) {  // warp-uniform
+                const unsigned lc = (unsigned)(col[u] - lo);
+                const bool in = q[u] >= 0 && lc < (unsigned)Wt;
+                int rank = 0;
+                const int e = sae[rr[u]];
+                if (in) {
+                  rank = out + rank_of(lc);
+                  if (fb[u]) EQrow[rank] = make_int2(e, q[u]);
+                }
+                dup_push(P, in && !fb[u], li, rank, e, q[u]);
+              }
+            }
+          }
+        }
         cbase += Lt;
         __syncthreads();
       }

@@ -16,12 +16,13 @@
 //   4. heads     a product is the head (first occurrence) of its column when no earlier slot of
 //                its bucket holds the same column; heads are counted per bucket and scanned.
 //   5. ranks     rank = heads of the row's earlier buckets + distinct smaller columns in the own
-//                bucket: R[PL + idx] = rank | RFLAG·head, written coalesced in product order;
-//                c_j = heads of the row's buckets (Phase IV "mark, scan, compact" of PAPER.md
-//                L154-156, done per tile in shared memory).
+//                bucket; a head writes its {A entry, B entry} to the gather plan at
+//                EQ[Ro_j + rank], every other product goes to the dup list; c_j = heads of the
+//                row's buckets (Phase IV "mark, scan, compact" of PAPER.md L154-156, done per
+//                tile in shared memory).
 //
 // Rows whose columns cluster (a bucket above TILE_MAXB) are handed to the bitmap kernel (the
-// fallback list); their R and c are written there.
+// fallback list); their plan and c are written there.
 #include "kernels.cuh"
 
 namespace spg {
@@ -75,8 +76,10 @@ __device__ __forceinline__ int2 block_scan2(int a, int b, int2& tot, int2* scrat
 // Shared-memory layout of one tile block (bytes).
 struct LightSmem {
   static constexpr int keys = 0;                                   // int[PMAX]    slot -> column (sign: not head)
-  static constexpr int rk = keys + TILE_PMAX * 4;                  // u32[PMAX]    idx -> column (expand), then R value
-  static constexpr int sidx = rk + TILE_PMAX * 4;                  // u16[PMAX]    slot -> product index
+  static constexpr int rk = keys + TILE_PMAX * 4;                  // u32[PMAX]    idx -> column
+  static constexpr int se = rk + TILE_PMAX * 4;                    // int[PMAX]    idx -> A entry
+  static constexpr int sq = se + TILE_PMAX * 4;                    // int[PMAX]    idx -> B entry
+  static constexpr int sidx = sq + TILE_PMAX * 4;                  // u16[PMAX]    slot -> product index
   static constexpr int sbk = sidx + TILE_PMAX * 2;                 // u16[PMAX]    slot -> bucket
   static constexpr int exb = sbk + TILE_PMAX * 2;                  // u16[PMAX]    idx -> bucket
   static constexpr int cnt = exb + TILE_PMAX * 2;                  // int[NBMAX+1] sizes -> starts -> ends
@@ -86,7 +89,9 @@ struct LightSmem {
   static constexpr int ae = row + (TILE_RM + 1) * 4;               // int[RM+1]    A-entry prefix
   static constexpr int bb = ae + (TILE_RM + 1) * 4;                // int[RM+1]    bucket base
   static constexpr int rpa = bb + (TILE_RM + 1) * 4;               // int[RM]      first A entry
-  static constexpr int seg = rpa + TILE_RM * 4;                    // int[NT+1]    chunk run -> product offset
+  static constexpr int ro = (rpa + TILE_RM * 4 + 15) & ~15;        // i64[RM]      EQ offset of the row
+  static constexpr int sae = ro + TILE_RM * 8;                     // int[NT]      chunk run -> A entry
+  static constexpr int seg = sae + TILE_NT * 4;                    // int[NT+1]    chunk run -> product offset
   static constexpr int sbs = seg + (TILE_NT + 1) * 4;              // int[NT]      chunk run -> B row start
   static constexpr int srw = sbs + TILE_NT * 4;                    // u16[NT]      chunk run -> batch row
   static constexpr int bad = srw + TILE_NT * 2;                    // u8[RM]
@@ -101,6 +106,10 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
   extern __shared__ __align__(16) unsigned char sm[];
   int* keys = reinterpret_cast<int*>(sm + LightSmem::keys);
   unsigned* rk = reinterpret_cast<unsigned*>(sm + LightSmem::rk);
+  int* se = reinterpret_cast<int*>(sm + LightSmem::se);
+  int* sq = reinterpret_cast<int*>(sm + LightSmem::sq);
+  long long* s_ro = reinterpret_cast<long long*>(sm + LightSmem::ro);
+  int* sae = reinterpret_cast<int*>(sm + LightSmem::sae);
   unsigned short* sidx = reinterpret_cast<unsigned short*>(sm + LightSmem::sidx);
   unsigned short* sbk = reinterpret_cast<unsigned short*>(sm + LightSmem::sbk);
   unsigned short* exb = reinterpret_cast<unsigned short*>(sm + LightSmem::exb);
@@ -167,6 +176,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
           const int i = P.row_begin + s_row[j0];
           const int pa = P.rpA[i];
           s_rpa[j0] = pa;
+          s_ro[j0] = P.Ro[s_row[j0]];
           a0 = P.rpA[i + 1] - pa;
           n0 = (P.frow[i] + TILE_BK - 1) / TILE_BK;
         }
@@ -174,6 +184,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
           const int i = P.row_begin + s_row[j1];
           const int pa = P.rpA[i];
           s_rpa[j1] = pa;
+          s_ro[j1] = P.Ro[s_row[j1]];
           a1 = P.rpA[i + 1] - pa;
           n1 = (P.frow[i] + TILE_BK - 1) / TILE_BK;
         }
@@ -185,7 +196,6 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       }
       __syncthreads();
       const int AE = s_ae[nr], NBt = s_bb[nr];
-      const long long pbase = PL[s_row[0]];
       for (int b = tid; b <= NBt; b += NT) {
         cnt[b] = 0;
         hc[b] = 0;
@@ -197,10 +207,10 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       int pc = 0;  // products before this chunk
       for (int u0 = 0; u0 < AE; u0 += NT) {
         const int u = u0 + tid;
-        int L = 0, bs = 0, j = 0;
+        int L = 0, bs = 0, j = 0, e = 0;
         if (u < AE) {
           j = upper_idx(s_ae, nr, u);
-          const int e = s_rpa[j] + (u - s_ae[j]);
+          e = s_rpa[j] + (u - s_ae[j]);
           const int k = P.colA[e];
           bs = P.rpB[k];
           L = P.rpB[k + 1] - bs;
@@ -211,6 +221,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
         if (L > 0) {
           seg[slot] = ex >> 16;
           sbs[slot] = bs;
+          sae[slot] = e;
           srw[slot] = (unsigned short)j;
         }
         if (tid == 0) seg[nrun] = Lt;
@@ -242,6 +253,8 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
               const int b = b0 + (int)(((unsigned long long)(unsigned)col[x] * (unsigned)nb) >> lgN);
               const int idx = pc + jw0 + x * 32 + lane;
               rk[idx] = (unsigned)col[x];
+              se[idx] = sae[rr[x]];
+              sq[idx] = q[x];
               exb[idx] = (unsigned short)b;
               atomicAdd(&cnt[b], 1);
             }
@@ -329,26 +342,35 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       }
       __syncthreads();
 
-      // ---- ranks: heads of the row's earlier buckets + distinct smaller columns in the bucket ---
-      for (int x = tid; x < Pg; x += NT) {
-        const int b = sbk[x];
-        const int s0 = b ? cnt[b - 1] : 0, s1 = cnt[b];
-        const int kx = keys[x];
-        const int k = kx & 0x7fffffff;
-        int u = 0;
-        for (int y = s0; y < s1; ++y) {
-          const int ky = keys[y];
-          u += (ky >= 0 && ky < k);
+      // ---- ranks: heads of the row's earlier buckets + distinct smaller columns in the bucket;
+      //      heads -> gather plan (slots are in (row, bucket) order: nearly coalesced), others
+      //      -> dup list --------------------------------------------------------------------
+      for (int x0 = warp * 32; x0 < Pg; x0 += NT) {  // warp-uniform trips (dup_push)
+        const int x = x0 + lane;
+        bool head = false, dup = false;
+        int rank = 0, jr = 0, idx = 0;
+        if (x < Pg) {
+          const int b = sbk[x];
+          const int s0 = b ? cnt[b - 1] : 0, s1 = cnt[b];
+          const int kx = keys[x];
+          const int k = kx & 0x7fffffff;
+          int u = 0;
+          for (int y = s0; y < s1; ++y) {
+            const int ky = keys[y];
+            u += (ky >= 0 && ky < k);
+          }
+          jr = brow[b];
+          rank = hc[b] - hc[s_bb[jr]] + u;
+          idx = sidx[x];
+          head = kx >= 0;
+          dup = !head;
         }
-        const int rank = hc[b] - hc[s_bb[brow[b]]] + u;
-        rk[sidx[x]] = (unsigned)rank | (kx >= 0 ? RFLAG : 0u);
+        const int e = se[idx], q = sq[idx];
+        if (head) P.EQ[s_ro[jr] + rank] = make_int2(e, q);
+        dup_push(P, dup, s_row[jr], rank, e, q);
       }
       for (int j = tid; j < nr; j += NT)
         if (!s_bad[j]) P.crow[s_row[j] + 1] = hc[s_bb[j + 1]] - hc[s_bb[j]];
-      __syncthreads();
-      // ---- R of the batch, in product order (bad rows: rewritten by the bitmap kernel) -------
-      unsigned* Rb = P.R + pbase;
-      for (int x = tid; x < Pb; x += NT) __stcs(Rb + x, rk[x]);
       __syncthreads();
     }
   }

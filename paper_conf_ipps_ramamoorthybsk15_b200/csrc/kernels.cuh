@@ -6,14 +6,14 @@
 //   classify   k_classify: row path (light tile kernel / heavy bitmap kernel / identity copy),
 //              heavy row lists and their R offsets; scan of light flops -> PL; k_tiles: tile
 //              cut points in light-product space, R offsets of light rows
-//   symbolic   k_light_rank (tiles of light rows) and k_bitmap_rank (heavy rows) compute, for
-//              every product of row i, its rank among the distinct columns of C(i,:) plus a
-//              first-occurrence flag: R[Ro_i + j] = rank | RFLAG·first.  c_i = #distinct.
-//   plan       k_cut_count / k_cut_write: row-aligned output windows of C (end of symbolic)
-//   numeric    k_num_windows / k_num_large: every product of a window's rows is scattered by
-//              its rank into shared memory and the window is written out coalesced (the
-//              Phase IV merge of PAPER.md L154-156, with the sort moved to the symbolic phase
-//              so numeric re-runs are a stream over R).
+//   symbolic   k_light_rank (tiles of light rows) and k_bitmap_rank (heavy rows) sort every row's
+//              products by column and emit the gather plan: for the first product of each
+//              distinct column of row i, EQ[Ro_i + rank] = {A entry, B entry}; every other
+//              product goes to the dup list.  c_i = #distinct.
+//   plan       k_plan: per-row EQ-to-C offset (or the SINGLE row's run), chunk -> first row
+//   numeric    k_numeric: C in chunks of NUM_CH outputs, one coalesced pass — C(i, r) =
+//              valA[e]·valB[q] from EQ (Phase IV of PAPER.md L154-156: the sort moved to the
+//              symbolic phase, so numeric re-runs are a stream); k_numeric_dup adds the dup list.
 #pragma once
 #include "common.cuh"
 
@@ -38,20 +38,26 @@ struct Small {
   int fb[16];               // fallback rows from the light kernel: [0] rows, [8] queue head
   int ntiles;
   int err;
-  int r_ok;                 // R capacity sufficient (written by k_tiles)
+  int r_ok;                 // EQ capacity sufficient (written by k_tiles)
   int amax;                 // longest row of A
-  int nwunits;              // numeric units: windows
-  int nlunits;              //   large rows
-  int ea0;                  // first A entry of this rank's rows
-  int lqhead;               // large-row numeric kernel: queue head
-  long long heavy_total;    // products of heavy rows (R offsets of heavy rows, relative)
-  long long fr;             // products needing R (light + heavy)
+  int nch_need;             // numeric chunks (+1) the plan needed
+  int pad0;
+  unsigned long long dupn;  // non-first products (dup list entries)
+  long long heavy_total;    // products of heavy rows (EQ offsets of heavy rows, relative)
+  long long fr;             // products of rows with a gather plan (light + heavy)
   unsigned long long hist[65];
   unsigned long long cstats[2 * NUM_CLS + 2];
 };
 
 // Problem view passed to the symbolic kernels.  Row indices in lists / cls / Ro / crow are
 // local (i - row_begin).
+//
+// Gather plan (the symbolic phase's output, consumed by numeric): row i's distinct columns, in
+// ascending order, are described by EQ[Ro_i + r] = {A entry e, B entry q} of the first product
+// (in the kernel's visiting order) that produced the column of rank r; every other product of
+// the column is a dup entry {li, r, e, q}.  Numeric is then C(i, r) = valA[e]·valB[q] (+ dups):
+// a coalesced stream in output order (Phase IV's "sort, mark, add like-tuples, compact" of
+// PAPER.md L154-156 with the sort moved to symbolic, so numeric re-runs on new values are cheap).
 struct SymProb {
   const int* __restrict__ rpA;
   const int* __restrict__ colA;
@@ -59,42 +65,48 @@ struct SymProb {
   const int* __restrict__ colB;
   const int* frow;          // f_i (global row index)
   const uint8_t* cls;       // path per local row
-  const long long* Ro;      // R offset per local row (-1: identity / empty)
-  unsigned* R;              // rank array
+  const long long* Ro;      // EQ offset per local row (-1: no plan: empty / SINGLE)
+  int2* EQ;                 // gather plan, indexed Ro_i + rank
+  int4* dup;                // dup list
+  unsigned long long* dupn; // its length (may exceed dupcap: then the host grows it and reruns)
+  long long dupcap;
+  uint8_t* fl8;             // uncached bitmap rows: first-claim flag per product (Ro_i + offset)
   long long* crow;          // C row offsets (local); symbolic writes counts at [li + 1]
   const int* r_ok;
   int row_begin, row_end;
   int lgN;                  // ceil(log2 N), N = columns of B
 };
 
-// Output window of the numeric phase: starts at C position pos (local), first row `row`.
-struct Cut {
-  long long pos;
-  int row;
-  int pad;
-};
+// Append a non-first product to the dup list (warp-aggregated; all 32 lanes must call).
+__device__ __forceinline__ void dup_push(const SymProb& P, bool d, int li, int rank, int e, int q) {
+  const unsigned m = __ballot_sync(FULL, d);
+  if (!m) return;
+  const int lane = threadIdx.x & 31, leader = __ffs(m) - 1;
+  unsigned long long b = 0;
+  if (lane == leader) b = atomicAdd(P.dupn, (unsigned long long)__popc(m));
+  b = __shfl_sync(FULL, b, leader) + __popc(m & lanemask_lt());
+  if (d && (long long)b < P.dupcap) P.dup[b] = make_int4(li, rank, e, q);
+}
 
-// Numeric work unit: outputs [lo, lo + c) of C (local positions) from local A entries [ea, eb).
-struct __align__(16) Unit {
-  long long lo;
-  int ea, eb, c, pad;
-};
+// Numeric phase: chunks of NUM_CH consecutive outputs of C.
+constexpr int NUM_CH = 2048;
+constexpr int NUM_NT = 256;
 
-// Problem view of the numeric kernel.
 template <typename V>
 struct NumProb {
   const V* __restrict__ valA;
   const int* __restrict__ colB;
   const V* __restrict__ valB;
-  const unsigned* __restrict__ R;
-  const int4* __restrict__ rec0;     // per local A entry: {B start, length, R index lo, hi}
-  const int4* __restrict__ rec1;     //   {C offset of its row lo, hi, first rank, last rank}
-  const Unit* __restrict__ wunits;
-  const Unit* __restrict__ lunits;
-  const Small* small;                // unit counts, ea0
-  int* lqhead;                       // large-row kernel: dynamic queue head
-  int* gq_pos;                       //   per-block overflow queues of non-first products
-  V* gq_val;                         //   (NUM_GDUP entries per block)
+  const int2* __restrict__ EQ;
+  const int4* __restrict__ dup;
+  const long long* __restrict__ crow;   // C row offsets (local)
+  const long long* __restrict__ nd;     // per local row: EQ index (or B index, SINGLE) minus C offset
+  const int* __restrict__ ne;           // per local row: -1, or the A entry of a SINGLE row
+  const int* __restrict__ chunk_row;    // row holding the first output of each chunk
+  long long nnz;                        // outputs (this rank)
+  long long ndup;
+  int nch;
+  int mloc;
   int* ccol;
   V* cval;
 };
@@ -135,17 +147,13 @@ cudaError_t launch_heavy_rank(int bin, cudaStream_t st, int grid, const SymProb&
 
 // k_numeric.cu — numeric plan (end of symbolic) and numeric phase.
 cudaError_t launch_plan(cudaStream_t st, int sms, const long long* crow, int mloc, const int* rpA, const int* colA,
-                        const int* rpB, const int* rowA, const int* Pe, const long long* Ro, const unsigned* R, int rb,
-                        int re, long long nnzA_upper, int* cnt, long long* coff, long long* scan_tmp, Cut* cuts,
-                        Unit* wunits, Unit* lunits, int lcap, int4* rec0, int4* rec1, Small* small);
-int plan_launches(long long mloc);
+                        const int* rpB, const uint8_t* cls, const long long* Ro, int rb, long long* nd, int* ne,
+                        int* chunk_row, int chcap, Small* small);
 template <typename V>
 cudaError_t numeric_configure();
 template <typename V>
-int numeric_occupancy(int which);  // 0: windows, 1..3: large-row kernel configuration 0..2
+int numeric_occupancy();
 template <typename V>
-cudaError_t launch_num_windows(cudaStream_t st, int grid, const NumProb<V>& P);
-template <typename V>
-cudaError_t launch_num_large(cudaStream_t st, int grid, int cfg, const NumProb<V>& P);
+cudaError_t launch_numeric(cudaStream_t st, int grid, const NumProb<V>& P);
 
 }  // namespace spg

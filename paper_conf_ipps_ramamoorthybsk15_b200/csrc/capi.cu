@@ -79,8 +79,9 @@ struct spg_ctx {
   // options
   int light_max = LIGHT_MAX_DEFAULT, tile_cap = TILE_CAP_DEFAULT, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
+  int pack_b = 0;  // numeric: gather B through a packed {column, value} copy (SPG_PACK_B=1)
   // workspace: analysis (all rows / all A entries), classification (this rank's rows), R, windows
-  DevBuf f, nz, rowA, Pe, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, EQ, fl8, dup, nd, ne, chunk_row, Pf,
+  DevBuf f, nz, rowA, Pe, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, EQ, fl8, dup, nd, ne, chunk_row, packB, Pf,
       splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
@@ -504,12 +505,18 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
     P.ndup = h->ndup;
     P.nch = h->nch;
     P.mloc = h->re - h->rb;
+    P.nB = B->nnz;
+    P.packB = nullptr;
+    if (h->pack_b && B->nnz > 0) {
+      CK(h->packB.ensure((size_t)B->nnz * (sizeof(V) == 8 ? 16 : 8)));
+      P.packB = h->packB.p;
+    }
     P.ccol = C_col;
     P.cval = (V*)C_val;
     int grid = h->occ_num * h->sms;
     if (h->nch < grid) grid = h->nch;
     CK(launch_numeric<V>(h->stream, grid, P));
-    h->launches += (h->nch > 0) + (h->ndup > 0);
+    h->launches += (h->nch > 0) + (h->ndup > 0) + (P.packB != nullptr);
   }
   h->stats.launches_numeric = h->launches;
   if (h->timing) {
@@ -562,6 +569,7 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
   }
   h->occ_light = light_occupancy();
   h->occ_num = dtype == SPG_FP64 ? numeric_occupancy<double>() : numeric_occupancy<float>();
+  if (const char* pb = getenv("SPG_PACK_B")) h->pack_b = atoi(pb);
   for (int b = 0; b < NUM_BINS; ++b) h->occ_heavy[b] = heavy_occupancy(b);
   cudaGetLastError();
   *out = h;
@@ -592,7 +600,7 @@ spg_status spg_spgemm_free(spg_handle h) {
     cudaStreamSynchronize(h->stream);
     DevBuf* bufs[] = {&h->f,     &h->nz,    &h->rowA,   &h->Pe,    &h->cls,    &h->fl,  &h->Ro,
                       &h->PL,    &h->tflag, &h->tiles,  &h->lists, &h->fblist, &h->small, &h->scan_tmp,
-                      &h->EQ,    &h->fl8,   &h->dup,    &h->nd,     &h->ne,   &h->chunk_row, &h->Pf,     &h->splits, &h->iota,  &h->ones, &h->crow_tmp};
+                      &h->EQ,    &h->fl8,   &h->dup,    &h->nd,     &h->ne,   &h->chunk_row, &h->packB, &h->Pf,     &h->splits, &h->iota,  &h->ones, &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
     if (h->canon) spg_spgemm_free(h->canon);

@@ -26,7 +26,7 @@ constexpr int LIGHTC_MAX = 256;
 constexpr int TILE_PMAX = 3072;       // products per tile: tile capacity + light threshold <= this
 constexpr int TILE_CAP_DEFAULT = 2048;
 constexpr int LIGHT_MAX_DEFAULT = 1024;
-constexpr int TILE_NT = 256;          // threads per tile block
+constexpr int TILE_NT = 512;          // threads per tile block
 constexpr int TILE_RM = 512;          // light rows per batch
 constexpr int TILE_BK = 4;            // expected products per bucket
 constexpr int TILE_NBMAX = TILE_PMAX / TILE_BK + TILE_RM;  // buckets per batch (ceil per row)

@@ -77,9 +77,9 @@ __device__ __forceinline__ int2 block_scan2(int a, int b, int2& tot, int2* scrat
 struct LightSmem {
   static constexpr int keys = 0;                                   // int[PMAX]    slot -> column (sign: not head)
   static constexpr int rk = keys + TILE_PMAX * 4;                  // u32[PMAX]    idx -> column
-  static constexpr int se = rk + TILE_PMAX * 4;                    // int[PMAX]    idx -> A entry
-  static constexpr int sq = se + TILE_PMAX * 4;                    // int[PMAX]    idx -> B entry
-  static constexpr int sidx = sq + TILE_PMAX * 4;                  // u16[PMAX]    slot -> product index
+  static constexpr int sq = rk + TILE_PMAX * 4;                    // int[PMAX]    idx -> B entry
+  static constexpr int se = sq + TILE_PMAX * 4;                    // u16[PMAX]    idx -> batch A entry
+  static constexpr int sidx = se + TILE_PMAX * 2;                  // u16[PMAX]    slot -> product index
   static constexpr int sbk = sidx + TILE_PMAX * 2;                 // u16[PMAX]    slot -> bucket
   static constexpr int exb = sbk + TILE_PMAX * 2;                  // u16[PMAX]    idx -> bucket
   static constexpr int cnt = exb + TILE_PMAX * 2;                  // int[NBMAX+1] sizes -> starts -> ends
@@ -90,7 +90,7 @@ struct LightSmem {
   static constexpr int bb = ae + (TILE_RM + 1) * 4;                // int[RM+1]    bucket base
   static constexpr int rpa = bb + (TILE_RM + 1) * 4;               // int[RM]      first A entry
   static constexpr int ro = (rpa + TILE_RM * 4 + 15) & ~15;        // i64[RM]      EQ offset of the row
-  static constexpr int sae = ro + TILE_RM * 8;                     // int[NT]      chunk run -> A entry
+  static constexpr int sae = ro + TILE_RM * 8;                     // int[NT]      chunk run -> batch A entry
   static constexpr int seg = sae + TILE_NT * 4;                    // int[NT+1]    chunk run -> product offset
   static constexpr int sbs = seg + (TILE_NT + 1) * 4;              // int[NT]      chunk run -> B row start
   static constexpr int srw = sbs + TILE_NT * 4;                    // u16[NT]      chunk run -> batch row
@@ -106,7 +106,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
   extern __shared__ __align__(16) unsigned char sm[];
   int* keys = reinterpret_cast<int*>(sm + LightSmem::keys);
   unsigned* rk = reinterpret_cast<unsigned*>(sm + LightSmem::rk);
-  int* se = reinterpret_cast<int*>(sm + LightSmem::se);
+  unsigned short* se = reinterpret_cast<unsigned short*>(sm + LightSmem::se);
   int* sq = reinterpret_cast<int*>(sm + LightSmem::sq);
   long long* s_ro = reinterpret_cast<long long*>(sm + LightSmem::ro);
   int* sae = reinterpret_cast<int*>(sm + LightSmem::sae);
@@ -196,6 +196,11 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       }
       __syncthreads();
       const int AE = s_ae[nr], NBt = s_bb[nr];
+      if (AE > 65535) {  // batch A entries do not fit the u16 index: hand the rows to the bitmap kernel
+        for (int j = tid; j < nr; j += NT) fb_list[atomicAdd(fb_count, 1)] = s_row[j];
+        __syncthreads();
+        continue;
+      }
       for (int b = tid; b <= NBt; b += NT) {
         cnt[b] = 0;
         hc[b] = 0;
@@ -221,7 +226,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
         if (L > 0) {
           seg[slot] = ex >> 16;
           sbs[slot] = bs;
-          sae[slot] = e;
+          sae[slot] = u;
           srw[slot] = (unsigned short)j;
         }
         if (tid == 0) seg[nrun] = Lt;
@@ -253,7 +258,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
               const int b = b0 + (int)(((unsigned long long)(unsigned)col[x] * (unsigned)nb) >> lgN);
               const int idx = pc + jw0 + x * 32 + lane;
               rk[idx] = (unsigned)col[x];
-              se[idx] = sae[rr[x]];
+              se[idx] = (unsigned short)sae[rr[x]];
               sq[idx] = q[x];
               exb[idx] = (unsigned short)b;
               atomicAdd(&cnt[b], 1);
@@ -365,7 +370,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
           head = kx >= 0;
           dup = !head;
         }
-        const int e = se[idx], q = sq[idx];
+        const int e = s_rpa[jr] + ((int)se[idx] - s_ae[jr]), q = sq[idx];
         if (head) P.EQ[s_ro[jr] + rank] = make_int2(e, q);
         dup_push(P, dup, s_row[jr], rank, e, q);
       }

@@ -77,8 +77,34 @@ cudaError_t launch_plan(cudaStream_t st, int sms, const long long* crow, int mlo
 constexpr int NUM_PT = NUM_CH / NUM_NT;  // outputs per thread and chunk
 static_assert(NUM_PT == 8, "slot ownership below assumes 8 slots per thread");
 
+// Packed B entry: column and value in one 16-byte (fp64) or 8-byte (fp32) word, so the gather of
+// an output's B entry is one load instead of two.
+template <typename V> struct PackB;
+template <> struct PackB<double> { using T = int4; };
+template <> struct PackB<float> { using T = int2; };
 template <typename V>
-__global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
+__device__ __forceinline__ typename PackB<V>::T pack_b(int c, V v);
+template <>
+__device__ __forceinline__ int4 pack_b<double>(int c, double v) {
+  const long long b = __double_as_longlong(v);
+  return make_int4(c, 0, (int)(unsigned)(b & 0xffffffffLL), (int)(b >> 32));
+}
+template <>
+__device__ __forceinline__ int2 pack_b<float>(int c, float v) { return make_int2(c, __float_as_int(v)); }
+__device__ __forceinline__ double unpack_v(const int4& t, double) {
+  return __longlong_as_double(((long long)t.w << 32) | (unsigned)t.z);
+}
+__device__ __forceinline__ float unpack_v(const int2& t, float) { return __int_as_float(t.y); }
+
+template <typename V>
+__global__ void __launch_bounds__(256) k_pack_b(const int* __restrict__ colB, const V* __restrict__ valB, long long n,
+                                                typename PackB<V>::T* __restrict__ out) {
+  for (long long x = blockIdx.x * (long long)blockDim.x + threadIdx.x; x < n; x += (long long)gridDim.x * blockDim.x)
+    out[x] = pack_b<V>(colB[x], valB[x]);
+}
+
+template <typename V, bool PACK>
+__global__ void __launch_bounds__(NUM_NT, 5) k_numeric(NumProb<V> P) {
   __shared__ __align__(16) int s_head[NUM_CH];   // slot -> 1 + slot of its row's first output in the chunk
   __shared__ long long s_nd[NUM_CH];             // head slot -> nd of its row
   __shared__ int s_ne[NUM_CH];                   // head slot -> ne of its row
@@ -153,8 +179,15 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
 #pragma unroll
     for (int k = 0; k < NUM_PT; ++k) {
       const bool ok = e[k] >= 0;
-      col[k] = ok ? __ldg(P.colB + q[k]) : 0;
-      vb[k] = ok ? __ldg(P.valB + q[k]) : V(0);
+      if constexpr (PACK) {
+        using T = typename PackB<V>::T;
+        const T t = ok ? __ldg(reinterpret_cast<const T*>(P.packB) + q[k]) : T{};
+        col[k] = t.x;
+        vb[k] = unpack_v(t, V(0));
+      } else {
+        col[k] = ok ? __ldg(P.colB + q[k]) : 0;
+        vb[k] = ok ? __ldg(P.valB + q[k]) : V(0);
+      }
       va[k] = ok ? __ldg(P.valA + e[k]) : V(0);
     }
 #pragma unroll
@@ -181,19 +214,28 @@ __global__ void __launch_bounds__(256) k_numeric_dup(NumProb<V> P) {
 
 template <typename V>
 cudaError_t numeric_configure() {
-  return cudaFuncSetAttribute(k_numeric<V>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  cudaError_t e = cudaFuncSetAttribute(k_numeric<V, false>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(k_numeric<V, true>, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+  return e;
 }
 
 template <typename V>
 int numeric_occupancy() {
   int nb = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_numeric<V>, NUM_NT, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_numeric<V, false>, NUM_NT, 0);
   return nb < 1 ? 1 : nb;
 }
 
 template <typename V>
 cudaError_t launch_numeric(cudaStream_t st, int grid, const NumProb<V>& P) {
-  if (P.nch > 0 && grid > 0) k_numeric<V><<<grid, NUM_NT, 0, st>>>(P);
+  if (P.packB) {
+    long long g = (P.nB + 255) / 256;
+    if (g > 148LL * 16) g = 148LL * 16;
+    if (P.nB > 0) k_pack_b<V><<<(int)g, 256, 0, st>>>(P.colB, P.valB, P.nB, reinterpret_cast<typename PackB<V>::T*>(P.packB));
+    if (P.nch > 0 && grid > 0) k_numeric<V, true><<<grid, NUM_NT, 0, st>>>(P);
+  } else if (P.nch > 0 && grid > 0) {
+    k_numeric<V, false><<<grid, NUM_NT, 0, st>>>(P);
+  }
   if (P.ndup > 0) {
     long long g = (P.ndup + 255) / 256;
     if (g > 148LL * 16) g = 148LL * 16;

@@ -88,7 +88,7 @@ __device__ __forceinline__ void dup_push(const SymProb& P, bool d, int li, int r
   if (d && (long long)b < P.dupcap) P.dup[b] = make_int4(li, rank, e, q);
 }
 
-// Numeric phase: chunks of NUM_CH consecutive outputs of C.
+// Numeric phase: chunks of NUM_CH consecutive outputs of C (one block each).
 constexpr int NUM_CH = 2048;
 constexpr int NUM_NT = 256;
 
@@ -105,6 +105,8 @@ struct NumProb {
   const int* __restrict__ chunk_row;    // row holding the first output of each chunk
   long long nnz;                        // outputs (this rank)
   long long ndup;
+  void* packB;                          // optional packed {column, value} copy of B (one gather)
+  long long nB;
   int nch;
   int mloc;
   int* ccol;

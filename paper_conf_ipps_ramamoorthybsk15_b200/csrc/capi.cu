@@ -182,6 +182,8 @@ SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* cr
   P.row_begin = h->rb;
   P.row_end = h->re;
   P.lgN = ceil_log2(B->ncols);
+  P.variant = 0;
+  if (const char* v = getenv("SPG_SYM_VARIANT")) P.variant = atoi(v);
   return P;
 }
 

@@ -73,6 +73,8 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
   // queue in its intra-GPU form.  count[0] = rows, count[8] = queue head.
   const int n = count[0];
   __shared__ int s_next;
+  __shared__ unsigned long long s_dbase;
+  __shared__ int s_dcnt;
   for (;;) {
     if (tid == 0) s_next = atomicAdd(const_cast<int*>(count) + 8, 1);
     __syncthreads();
@@ -200,6 +202,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
       const int lo = tile << lw;
       // ---- pass 1: claim bits; first claimers flagged -----------------------------------------
       int cbase = 0;
+      int npin = 0;  // this thread's products inside the tile
       for (int c = 0; c < nchunks; ++c) {
         if (nchunks > 1 || tile == 0) {
           gather(c);
@@ -213,6 +216,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
             const unsigned lc = (unsigned)(cc[s] - lo);
             bool first = false;
             if (j0 + lane < Lt && lc < (unsigned)Wt) {
+              ++npin;
               const int w = lc >> 5;
               const unsigned b = 1u << (lc & 31);
               const unsigned old = atomicOr(&bm[w], b);
@@ -226,6 +230,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
           for_products([&](int j, int col) {
             const unsigned lc = (unsigned)(col - lo);
             if (lc < (unsigned)Wt) {
+              ++npin;
               const int w = lc >> 5;
               const unsigned b = 1u << (lc & 31);
               const unsigned old = atomicOr(&bm[w], b);
@@ -272,6 +277,14 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
         pcarry += ptot;
       }
       const int ctile = pcarry;
+      {  // dup slots of the tile: its products minus its distinct columns (one global atomic)
+        const long long ptile = ntiles == 1 ? (long long)f : g.sum((long long)npin);
+        if (tid == 0) {
+          const long long nd = ptile - ctile;
+          s_dbase = nd > 0 ? atomicAdd(P.dupn, (unsigned long long)nd) : 0ull;
+          s_dcnt = 0;
+        }
+      }
       __syncthreads();
       // ---- pass 2: ranks -> gather plan (first claimers) and dup list (the others) ---------------
       cbase = 0;
@@ -293,9 +306,9 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
                 first = (flags[j >> 5] >> (j & 31)) & 1u;
                 q = sbs[r] + (j - seg[r]);
                 e = sae[r];
-                if (first) EQrow[rank] = make_int2(e, q);
+                if (first && !(P.variant & 1)) EQrow[rank] = make_int2(e, q);
               }
-              dup_push(P, in && !first, li, rank, e, q);
+              dup_push(P, in && !first && !(P.variant & 2), li, rank, e, q, s_dbase, &s_dcnt);
             }
           }
         } else {
@@ -326,9 +339,9 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
                 const int e = sae[rr[u]];
                 if (in) {
                   rank = out + rank_of(lc);
-                  if (fb[u]) EQrow[rank] = make_int2(e, q[u]);
+                  if (fb[u] && !(P.variant & 1)) EQrow[rank] = make_int2(e, q[u]);
                 }
-                dup_push(P, in && !fb[u], li, rank, e, q[u]);
+                dup_push(P, in && !fb[u] && !(P.variant & 2), li, rank, e, q[u], s_dbase, &s_dcnt);
               }
             }
           }

@@ -76,8 +76,7 @@ __device__ __forceinline__ int2 block_scan2(int a, int b, int2& tot, int2* scrat
 // Shared-memory layout of one tile block (bytes).
 struct LightSmem {
   static constexpr int keys = 0;                                   // int[PMAX]    slot -> column (sign: not head)
-  static constexpr int rk = keys + TILE_PMAX * 4;                  // u32[PMAX]    idx -> column
-  static constexpr int sq = rk + TILE_PMAX * 4;                    // int[PMAX]    idx -> B entry
+  static constexpr int sq = keys + TILE_PMAX * 4;                  // int[PMAX]    idx -> B entry
   static constexpr int se = sq + TILE_PMAX * 4;                    // u16[PMAX]    idx -> batch A entry
   static constexpr int sidx = se + TILE_PMAX * 2;                  // u16[PMAX]    slot -> product index
   static constexpr int sbk = sidx + TILE_PMAX * 2;                 // u16[PMAX]    slot -> bucket
@@ -105,7 +104,6 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
                                                         int* __restrict__ fb_count) {
   extern __shared__ __align__(16) unsigned char sm[];
   int* keys = reinterpret_cast<int*>(sm + LightSmem::keys);
-  unsigned* rk = reinterpret_cast<unsigned*>(sm + LightSmem::rk);
   unsigned short* se = reinterpret_cast<unsigned short*>(sm + LightSmem::se);
   int* sq = reinterpret_cast<int*>(sm + LightSmem::sq);
   long long* s_ro = reinterpret_cast<long long*>(sm + LightSmem::ro);
@@ -127,6 +125,8 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
   __shared__ int2 scratch2[TILE_NT / 32 + 1];
   __shared__ int scratch[TILE_NT / 32 + 1];
   __shared__ int s_misc[4];
+  __shared__ unsigned long long s_dbase;
+  __shared__ int s_dcnt;
   constexpr int NT = TILE_NT, NW = NT / 32;
   const Group<NT> g{(int)threadIdx.x, scratch};
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -257,7 +257,6 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
               const int b0 = s_bb[jr], nb = s_bb[jr + 1] - b0;
               const int b = b0 + (int)(((unsigned long long)(unsigned)col[x] * (unsigned)nb) >> lgN);
               const int idx = pc + jw0 + x * 32 + lane;
-              rk[idx] = (unsigned)col[x];
               se[idx] = (unsigned short)sae[rr[x]];
               sq[idx] = q[x];
               exb[idx] = (unsigned short)b;
@@ -304,13 +303,25 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       __syncthreads();
 
       // ---- pass 2: scatter into buckets; afterwards cnt[b] = end of bucket b -----------------
-      for (int idx = tid; idx < Pb; idx += NT) {
-        const int b = exb[idx];
-        if (s_bad[brow[b]]) continue;
-        const int slot = atomicAdd(&cnt[b], 1);
-        keys[slot] = (int)rk[idx];
-        sidx[slot] = (unsigned short)idx;
-        sbk[slot] = (unsigned short)b;
+      //      (columns re-gathered from B through L1/L2 rather than kept per product in shared
+      //      memory: that keeps two 512-thread blocks per SM at 4096 products per tile)
+      for (int i0 = tid; i0 < Pb; i0 += 4 * NT) {
+        int bk[4], cl[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int idx = i0 + u * NT;
+          bk[u] = idx < Pb ? (int)exb[idx] : -1;
+          cl[u] = idx < Pb ? __ldg(P.colB + sq[idx]) : 0;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int b = bk[u];
+          if (b < 0 || s_bad[brow[b]]) continue;
+          const int slot = atomicAdd(&cnt[b], 1);
+          keys[slot] = cl[u];
+          sidx[slot] = (unsigned short)(i0 + u * NT);
+          sbk[slot] = (unsigned short)b;
+        }
       }
       __syncthreads();
       const int Pg = NBt > 0 ? cnt[NBt - 1] : 0;
@@ -343,7 +354,13 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
           if (b < NBt) hc[b] = run;
           run += c8[k];
         }
-        if (tid == 0) hc[NBt] = tot;
+        if (tid == 0) {
+          hc[NBt] = tot;
+          // dup slots of the batch: products placed in buckets minus distinct columns
+          const int nd = (NBt > 0 ? cnt[NBt - 1] : 0) - tot;
+          s_dbase = nd > 0 ? atomicAdd(P.dupn, (unsigned long long)nd) : 0ull;
+          s_dcnt = 0;
+        }
       }
       __syncthreads();
 
@@ -371,8 +388,8 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
           dup = !head;
         }
         const int e = s_rpa[jr] + ((int)se[idx] - s_ae[jr]), q = sq[idx];
-        if (head) P.EQ[s_ro[jr] + rank] = make_int2(e, q);
-        dup_push(P, dup, s_row[jr], rank, e, q);
+        if (head && !(P.variant & 1)) P.EQ[s_ro[jr] + rank] = make_int2(e, q);
+        dup_push(P, dup && !(P.variant & 2), s_row[jr], rank, e, q, s_dbase, &s_dcnt);
       }
       for (int j = tid; j < nr; j += NT)
         if (!s_bad[j]) P.crow[s_row[j] + 1] = hc[s_bb[j + 1]] - hc[s_bb[j]];

@@ -75,16 +75,20 @@ struct SymProb {
   const int* r_ok;
   int row_begin, row_end;
   int lgN;                  // ceil(log2 N), N = columns of B
+  int variant;              // experiments only (SPG_SYM_VARIANT): bit 0 skips plan stores, bit 1 dup pushes
 };
 
-// Append a non-first product to the dup list (warp-aggregated; all 32 lanes must call).
-__device__ __forceinline__ void dup_push(const SymProb& P, bool d, int li, int rank, int e, int q) {
+// Append a non-first product to the dup list (all 32 lanes must call).  The caller reserved the
+// slots [base, base + n) of its row / tile / batch with one global atomic (the count is known before
+// the ranks are written: products - distinct columns); *s_cnt (shared) hands them out per warp.
+__device__ __forceinline__ void dup_push(const SymProb& P, bool d, int li, int rank, int e, int q,
+                                         unsigned long long base, int* s_cnt) {
   const unsigned m = __ballot_sync(FULL, d);
   if (!m) return;
   const int lane = threadIdx.x & 31, leader = __ffs(m) - 1;
-  unsigned long long b = 0;
-  if (lane == leader) b = atomicAdd(P.dupn, (unsigned long long)__popc(m));
-  b = __shfl_sync(FULL, b, leader) + __popc(m & lanemask_lt());
+  int o = 0;
+  if (lane == leader) o = atomicAdd(s_cnt, __popc(m));
+  const unsigned long long b = base + (unsigned long long)(__shfl_sync(FULL, o, leader) + __popc(m & lanemask_lt()));
   if (d && (long long)b < P.dupcap) P.dup[b] = make_int4(li, rank, e, q);
 }
 

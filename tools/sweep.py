@@ -48,6 +48,12 @@ def time_plan(dA, dB, steps, **opts):
     return float(np.median(ts)), float(np.median(tn)), st, digest
 
 
+LIGHT = [int(x) for x in os.environ.get("SWEEP_LIGHT", "0,256,512,1024,2048").split(",")]
+TILE = [int(x) for x in os.environ.get("SWEEP_TILE", "1024,2048").split(",")]
+HEAVY = [int(x) for x in os.environ.get("SWEEP_HEAVY", "4096,8192").split(",")]
+PMAX = int(os.environ.get("SWEEP_PMAX", "3072"))
+
+
 def main():
     p = argparse.ArgumentParser()
     p.add_argument("--config", default="webbase1m")
@@ -58,16 +64,16 @@ def main():
     A, B = W.make(a.config)
     dA = spg.DeviceCSR.from_host(A, "cuda")
     dB = dA if B is A else spg.DeviceCSR.from_host(B, "cuda")
-    grid = list(itertools.product([64, 128, 256], [512, 1024, 2048], [2048, 4096, 8192]))
+    # (light_max, tile_flops, heavy_max): light rows (f <= light_max) go to the tile kernel,
+    # light_max + tile_flops <= TILE_PMAX (3072); heavy rows up to heavy_max to the cached bitmap
+    grid = [(lm, tf, hm) for lm in LIGHT for tf in TILE for hm in HEAVY if lm + tf <= PMAX]
     ref = None
-    for lm, mm, hm in grid:
-        if mm < lm or hm < mm:
-            continue
-        ts, tn, st, dig = time_plan(dA, dB, a.steps, light_max_flops=lm, medium_max_flops=mm, heavy_max_flops=hm,
+    for lm, tf, hm in grid:
+        ts, tn, st, dig = time_plan(dA, dB, a.steps, tile_flops=tf, light_max_flops=lm, heavy_max_flops=hm,
                                     concurrent=a.concurrent)
         ref = ref or dig
         F = st["flops"]
-        line = {"config": a.config, "light_max": lm, "medium_max": mm, "heavy_max": hm, "symbolic_ms": ts,
+        line = {"config": a.config, "light_max": lm, "tile_flops": tf, "heavy_max": hm, "symbolic_ms": ts,
                 "numeric_ms": tn, "gflops": 2 * F / ((ts + tn) * 1e-3) / 1e9, "class_rows": st["class_rows"],
                 "same_result": dig[0] == ref[0] and dig[2] == ref[2] and abs(dig[1] - ref[1]) <= 1e-9 * abs(ref[1])}
         print(json.dumps(line), flush=True)

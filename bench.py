@@ -294,8 +294,12 @@ def run_ours(args):
 
     # roofline of the numeric phase (the dominant stage: class kernels forked on streams and joined)
     nnzA_loc = int(A.row_ptr[re]) - int(A.row_ptr[rb])
-    alg_bytes = (csr_bytes(re - rb, nnzA_loc, vb) + csr_bytes(B.nrows, B.nnz, vb)
+    # A + B + C + intermediate, the intermediate being the read of the symbolic
+    # phase's output (the gather plan: EQ entries of non-SINGLE outputs + the dup list)
+    abc_bytes = (csr_bytes(re - rb, nnzA_loc, vb) + csr_bytes(B.nrows, B.nnz, vb)
                  + csr_bytes(re - rb, nnz, vb, rp_bytes=8))
+    plan_bytes = int(st["rank_bytes"])
+    alg_bytes = abc_bytes + plan_bytes
     num_ms = float(np.mean(num))
     peak, peak_src = load_peaks()
     achieved = alg_bytes / (num_ms * 1e-3) / 1e9
@@ -375,7 +379,9 @@ def run_ours(args):
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                          "kernel": "numeric phase (k_numeric gather stream + k_numeric_dup)",
-                         "algorithmic_bytes": int(alg_bytes)},
+                         "algorithmic_bytes": int(alg_bytes), "abc_bytes": int(abc_bytes),
+                         "plan_bytes": plan_bytes,
+                         "abc_frac": abc_bytes / (num_ms * 1e-3) / 1e9 / peak},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clocks,
         }
         emit(line, args)

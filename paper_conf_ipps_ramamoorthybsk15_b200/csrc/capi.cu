@@ -182,8 +182,6 @@ SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* cr
   P.row_begin = h->rb;
   P.row_end = h->re;
   P.lgN = ceil_log2(B->ncols);
-  P.variant = 0;
-  if (const char* v = getenv("SPG_SYM_VARIANT")) P.variant = atoi(v);
   return P;
 }
 
@@ -468,7 +466,9 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   for (int b = 0; b < 65; ++b) st.bin_hist[b] = (int64_t)hs.hist[b];
   st.tiles = hs.ntiles;
   st.fallback_rows = hs.fb[0];
-  st.rank_bytes = (int64_t)h->nnzC * (int64_t)sizeof(int2) + h->ndup * (int64_t)sizeof(int4);
+  // gather-plan bytes numeric reads: an EQ entry per output of a non-SINGLE row (a SINGLE row's
+  // c_i = f_i outputs need none) and the dup list
+  st.rank_bytes = (h->nnzC - st.class_flops[CLS_SINGLE]) * (int64_t)sizeof(int2) + h->ndup * (int64_t)sizeof(int4);
   st.launches_symbolic = h->launches;
   if (h->timing) {
     cudaEventElapsedTime(&st.ms_analysis, h->ev_t[0], h->ev_t[1]);

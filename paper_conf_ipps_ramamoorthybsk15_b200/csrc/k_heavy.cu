@@ -306,9 +306,9 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
                 first = (flags[j >> 5] >> (j & 31)) & 1u;
                 q = sbs[r] + (j - seg[r]);
                 e = sae[r];
-                if (first && !(P.variant & 1)) EQrow[rank] = make_int2(e, q);
+                if (first) EQrow[rank] = make_int2(e, q);
               }
-              dup_push(P, in && !first && !(P.variant & 2), li, rank, e, q, s_dbase, &s_dcnt);
+              dup_push(P, in && !first, li, rank, e, q, s_dbase, &s_dcnt);
             }
           }
         } else {
@@ -339,9 +339,9 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
                 const int e = sae[rr[u]];
                 if (in) {
                   rank = out + rank_of(lc);
-                  if (fb[u] && !(P.variant & 1)) EQrow[rank] = make_int2(e, q[u]);
+                  if (fb[u]) EQrow[rank] = make_int2(e, q[u]);
                 }
-                dup_push(P, in && !fb[u] && !(P.variant & 2), li, rank, e, q[u], s_dbase, &s_dcnt);
+                dup_push(P, in && !fb[u], li, rank, e, q[u], s_dbase, &s_dcnt);
               }
             }
           }

@@ -388,8 +388,8 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
           dup = !head;
         }
         const int e = s_rpa[jr] + ((int)se[idx] - s_ae[jr]), q = sq[idx];
-        if (head && !(P.variant & 1)) P.EQ[s_ro[jr] + rank] = make_int2(e, q);
-        dup_push(P, dup && !(P.variant & 2), s_row[jr], rank, e, q, s_dbase, &s_dcnt);
+        if (head) P.EQ[s_ro[jr] + rank] = make_int2(e, q);
+        dup_push(P, dup, s_row[jr], rank, e, q, s_dbase, &s_dcnt);
       }
       for (int j = tid; j < nr; j += NT)
         if (!s_bad[j]) P.crow[s_row[j] + 1] = hc[s_bb[j + 1]] - hc[s_bb[j]];

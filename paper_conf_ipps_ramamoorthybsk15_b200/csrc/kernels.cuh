@@ -75,7 +75,6 @@ struct SymProb {
   const int* r_ok;
   int row_begin, row_end;
   int lgN;                  // ceil(log2 N), N = columns of B
-  int variant;              // experiments only (SPG_SYM_VARIANT): bit 0 skips plan stores, bit 1 dup pushes
 };
 
 // Append a non-first product to the dup list (all 32 lanes must call).  The caller reserved the

@@ -12,28 +12,21 @@
 namespace spg {
 
 // f_i = sum over stored A(i,k) of len_B(k); nz_i = #entries with len_B(k) > 0 (capped at 2, plus
-// bits 6/7 for A rows longer than one 512- / 1024-thread bitmap chunk).  Per A entry e of row i:
-// rowA[e] = i and Pe[e] = sum of len_B over the entries of row i before e (the entry's first
-// product within the row — the numeric kernel's index into R).  One block owns ROWS consecutive
-// rows; its threads stride over the rows' A entries (coalesced), find the owning row by binary
-// search in the cached row_ptr tile, pre-reduce per warp and row, and add into shared 32-bit
-// accumulators.  Pe comes from a block scan of len_B (wrapping 32-bit arithmetic: the in-row
-// value itself is < 2^31, or the row is reported as overflowing).
+// bits 6/7 for A rows longer than one 512- / 1024-thread bitmap chunk).  One block owns ROWS
+// consecutive rows; its threads stride over the rows' A entries (coalesced), find the owning row
+// by binary search in the cached row_ptr tile, pre-reduce per warp and row, and add into shared
+// 32-bit accumulators.
 template <int ROWS>
 __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict__ rpA, const int* __restrict__ colA,
                                                     int K, const int* __restrict__ rpB, int* __restrict__ f_out,
-                                                    uint8_t* __restrict__ nz_out, int* __restrict__ rowA,
-                                                    int* __restrict__ Pe, unsigned long long* __restrict__ hist,
+                                                    uint8_t* __restrict__ nz_out, unsigned long long* __restrict__ hist,
                                                     int* __restrict__ err, int* __restrict__ amax) {
-  constexpr int NW = ROWS / 32;
   __shared__ int s_rp[ROWS + 1];
   __shared__ unsigned s_f[ROWS];
   __shared__ int s_nz[ROWS];
-  __shared__ unsigned s_base[ROWS];
-  __shared__ unsigned s_ws[NW + 1];
   __shared__ unsigned s_hist[65];
   __shared__ int s_amax;
-  const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+  const int t = threadIdx.x, lane = t & 31;
   const int r0 = blockIdx.x * ROWS;
   const int nr = min(ROWS, M - r0);
   if (t <= nr) s_rp[t] = rpA[r0 + t];
@@ -45,7 +38,6 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
   __syncthreads();
   const int e0 = s_rp[0], e1 = s_rp[nr];
   int bad = 0;
-  unsigned carry = 0;  // wrapping prefix of len_B over this block's entries
   for (int base = e0; base < e1; base += ROWS) {  // uniform trip count: warp collectives below
     const int e = base + t;
     bool act = e < e1;
@@ -57,20 +49,6 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
       else L = rpB[k + 1] - rpB[k];
     }
     act = r >= 0;
-    // block exclusive scan of L -> S (wrapping); rows starting in this chunk record their base
-    const unsigned incl = warp_incl_scan((unsigned)L);
-    if (lane == 31) s_ws[w] = incl;
-    __syncthreads();
-    if (w == 0) {
-      const unsigned x = lane < NW ? s_ws[lane] : 0u;
-      const unsigned xi = warp_incl_scan(x);
-      if (lane < NW) s_ws[lane] = xi - x;
-      if (lane == NW - 1) s_ws[NW] = xi;
-    }
-    __syncthreads();
-    const unsigned S = carry + incl - (unsigned)L + s_ws[w];
-    if (act && e == s_rp[r]) s_base[r] = S;
-    carry += s_ws[NW];
     const unsigned nzb = __ballot_sync(FULL, act && L > 0);
     const unsigned grp = __match_any_sync(FULL, r);
     if (act) {
@@ -86,11 +64,6 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
         }
         atomicAdd(&s_nz[r], __popc(grp & nzb));
       }
-    }
-    __syncthreads();
-    if (act) {
-      rowA[e] = r0 + r;
-      Pe[e] = (int)(S - s_base[r]);
     }
   }
   __syncthreads();
@@ -382,10 +355,10 @@ __global__ void k_narrow(const long long* __restrict__ in, int* __restrict__ out
 
 // ---- host launchers ------------------------------------------------------------------------
 cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB,
-                             int* f, uint8_t* nz, int* rowA, int* Pe, unsigned long long* hist, int* err, int* amax) {
+                             int* f, uint8_t* nz, unsigned long long* hist, int* err, int* amax) {
   if (M <= 0) return cudaSuccess;
   constexpr int ROWS = 256;
-  k_row_flops<ROWS><<<(M + ROWS - 1) / ROWS, ROWS, 0, st>>>(M, rpA, colA, K, rpB, f, nz, rowA, Pe, hist, err, amax);
+  k_row_flops<ROWS><<<(M + ROWS - 1) / ROWS, ROWS, 0, st>>>(M, rpA, colA, K, rpB, f, nz, hist, err, amax);
   return cudaGetLastError();
 }
 
@@ -397,6 +370,54 @@ cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_
   long long blocks = (n + CL_NT - 1) / CL_NT;
   if (blocks > (long long)sms * 8) blocks = (long long)sms * 8;
   k_classify<<<(int)blocks, CL_NT, 0, st>>>(f, nz, rb, re, prm, cls, fl, Ro, lists, small, crow);
+  return cudaGetLastError();
+}
+
+// Largest rows first: each bitmap bin's row list is sorted by descending f_i (one block per bin,
+// bitonic sort of up to LPT_MAX (f, row) pairs in shared memory; longer lists keep their order).
+// The bins' blocks take rows from a dynamic queue, so this is longest-processing-time-first
+// scheduling: the biggest HUGE rows (up to ~9x the bin average on webbase1m) start first instead
+// of forming the kernel's tail.
+constexpr int LPT_MAX = 8192;
+__global__ void __launch_bounds__(1024) k_sort_lists(HeavyLists lists, const int* __restrict__ f, int rb,
+                                                     const Small* __restrict__ sm) {
+  extern __shared__ unsigned long long key[];  // LPT_MAX entries
+  const int b = blockIdx.x;
+  const int n = sm->counts[b];
+  if (n <= 1 || n > LPT_MAX) return;
+  int* list = lists.rows[b];
+  int np = 1;
+  while (np < n) np <<= 1;
+  for (int x = threadIdx.x; x < np; x += blockDim.x) {
+    unsigned long long k = 0;  // padding sorts last
+    if (x < n) {
+      const int li = list[x];
+      k = ((unsigned long long)(unsigned)f[rb + li] << 32) | (unsigned)li;
+    }
+    key[x] = k;
+  }
+  __syncthreads();
+  for (int size = 2; size <= np; size <<= 1)
+    for (int j = size >> 1; j > 0; j >>= 1) {
+      for (int x = threadIdx.x; x < np; x += blockDim.x) {
+        const int y = x ^ j;
+        if (y > x) {
+          const bool desc = (x & size) == 0;
+          const unsigned long long a = key[x], c = key[y];
+          if (desc ? a < c : a > c) { key[x] = c; key[y] = a; }
+        }
+      }
+      __syncthreads();
+    }
+  for (int x = threadIdx.x; x < n; x += blockDim.x) list[x] = (int)(unsigned)(key[x] & 0xffffffffu);
+}
+
+cudaError_t launch_sort_lists(cudaStream_t st, const HeavyLists& lists, const int* f, int rb, const Small* small) {
+  // (per call: the attribute is per device, and a process may drive several)
+  cudaError_t e = cudaFuncSetAttribute(k_sort_lists, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       LPT_MAX * (int)sizeof(unsigned long long));
+  if (e != cudaSuccess) return e;
+  k_sort_lists<<<NUM_BINS, 1024, LPT_MAX * sizeof(unsigned long long), st>>>(lists, f, rb, small);
   return cudaGetLastError();
 }
 

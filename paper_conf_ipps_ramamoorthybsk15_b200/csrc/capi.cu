@@ -81,7 +81,7 @@ struct spg_ctx {
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
   int pack_b = 0;  // numeric: gather B through a packed {column, value} copy (SPG_PACK_B=1)
   // workspace: analysis (all rows / all A entries), classification (this rank's rows), R, windows
-  DevBuf f, nz, rowA, Pe, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, EQ, fl8, dup, nd, ne, chunk_row, packB, Pf,
+  DevBuf f, nz, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, EQ, fl8, dup, nd, ne, chunk_row, packB, Pf,
       splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
@@ -244,8 +244,6 @@ spg_status ensure_ws(spg_handle h, int M, long long nnzA) {
   size_t na = (size_t)(nnzA > 0 ? nnzA : 1);
   CK(h->f.ensure(m * sizeof(int)));
   CK(h->nz.ensure(m));
-  CK(h->rowA.ensure(na * sizeof(int)));
-  CK(h->Pe.ensure(na * sizeof(int)));
   CK(h->cls.ensure(m));
   CK(h->fl.ensure(m * sizeof(int)));
   CK(h->Ro.ensure(m * sizeof(long long)));
@@ -266,7 +264,7 @@ spg_status analysis(spg_handle h, const spg_csr* A, const spg_csr* B) {
   Small* ds = h->small.as<Small>();
   CK(cudaMemsetAsync(ds, 0, sizeof(Small), h->stream));
   CK(launch_row_flops(h->stream, A->nrows, A->row_ptr, A->col_idx, B->nrows, B->row_ptr, h->f.as<int>(),
-                      h->nz.as<uint8_t>(), h->rowA.as<int>(), h->Pe.as<int>(), ds->hist, &ds->err, &ds->amax));
+                      h->nz.as<uint8_t>(), ds->hist, &ds->err, &ds->amax));
   h->launches += A->nrows > 0;
   return SPG_OK;
 }
@@ -393,6 +391,10 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(cudaMemsetAsync(PL, 0, sizeof(long long), h->stream));
     CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm,
                        h->cls.as<uint8_t>(), h->fl.as<int>(), h->Ro.as<long long>(), L3, ds, crow));
+    if (Mloc > 0) {
+      CK(launch_sort_lists(h->stream, L3, h->f.as<int>(), h->rb, ds));
+      h->launches++;
+    }
     CK(launch_incl_scan<int>(h->stream, h->fl.as<int>(), PL + 1, Mloc, h->scan_tmp.as<long long>()));
     long long r_cap = h->EQ.p && h->fl8.p ? (long long)(h->EQ.cap / sizeof(int2)) : 0;
     if (r_cap > (long long)h->fl8.cap) r_cap = (long long)h->fl8.cap;
@@ -600,7 +602,7 @@ spg_status spg_spgemm_free(spg_handle h) {
   {
     DeviceGuard g(h->device);
     cudaStreamSynchronize(h->stream);
-    DevBuf* bufs[] = {&h->f,     &h->nz,    &h->rowA,   &h->Pe,    &h->cls,    &h->fl,  &h->Ro,
+    DevBuf* bufs[] = {&h->f,     &h->nz,    &h->cls,    &h->fl,  &h->Ro,
                       &h->PL,    &h->tflag, &h->tiles,  &h->lists, &h->fblist, &h->small, &h->scan_tmp,
                       &h->EQ,    &h->fl8,   &h->dup,    &h->nd,     &h->ne,   &h->chunk_row, &h->packB, &h->Pf,     &h->splits, &h->iota,  &h->ones, &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();

@@ -1,11 +1,10 @@
 // kernels.cuh — declarations shared by the kernel translation units and the C-ABI layer.
 //
 // Pipeline:
-//   analysis   k_row_flops: f_i, run flags, log2 histogram, per-A-entry row and in-row product
-//              offset (rowA, Pe)
+//   analysis   k_row_flops: f_i, run flags, log2 histogram
 //   classify   k_classify: row path (light tile kernel / heavy bitmap kernel / identity copy),
-//              heavy row lists and their R offsets; scan of light flops -> PL; k_tiles: tile
-//              cut points in light-product space, R offsets of light rows
+//              heavy row lists and their plan (EQ) offsets; scan of light flops -> PL; k_tiles:
+//              tile cut points in light-product space, plan offsets of light rows
 //   symbolic   k_light_rank (tiles of light rows) and k_bitmap_rank (heavy rows) sort every row's
 //              products by column and emit the gather plan: for the first product of each
 //              distinct column of row i, EQ[Ro_i + rank] = {A entry, B entry}; every other
@@ -118,13 +117,14 @@ struct NumProb {
 
 // analysis.cu
 cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB, int* f,
-                             uint8_t* nz, int* rowA, int* Pe, unsigned long long* hist, int* err, int* amax);
+                             uint8_t* nz, unsigned long long* hist, int* err, int* amax);
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
                             const ClassParams& prm, uint8_t* cls, int* fl, long long* Ro, const HeavyLists& lists,
                             Small* small, long long* crow);
 cudaError_t launch_tiles(cudaStream_t st, int sms, const int* f, int rb, int re, int tile_cap, const uint8_t* cls,
                          const long long* PL, long long* Ro, uint8_t* tflag, int* tiles, Small* small,
                          long long r_cap);
+cudaError_t launch_sort_lists(cudaStream_t st, const HeavyLists& lists, const int* f, int rb, const Small* small);
 size_t scan_tmp_elems(long long n);
 int scan_launches(long long n);
 template <typename Tin>

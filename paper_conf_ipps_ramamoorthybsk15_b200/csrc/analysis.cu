@@ -373,16 +373,16 @@ cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_
   return cudaGetLastError();
 }
 
-// Largest rows first: each bitmap bin's row list is sorted by descending f_i (one block per bin,
-// bitonic sort of up to LPT_MAX (f, row) pairs in shared memory; longer lists keep their order).
+// Largest rows first: a bitmap bin's row list is sorted by descending f_i (one block, bitonic sort
+// of up to LPT_MAX (f, row) pairs in shared memory; longer lists keep their order).  Launched on
+// the bin's own stream, just before its kernel.
 // The bins' blocks take rows from a dynamic queue, so this is longest-processing-time-first
 // scheduling: the biggest HUGE rows (up to ~9x the bin average on webbase1m) start first instead
 // of forming the kernel's tail.
-constexpr int LPT_MAX = 8192;
-__global__ void __launch_bounds__(1024) k_sort_lists(HeavyLists lists, const int* __restrict__ f, int rb,
+constexpr int LPT_MAX = 2048;
+__global__ void __launch_bounds__(1024) k_sort_lists(HeavyLists lists, int b, const int* __restrict__ f, int rb,
                                                      const Small* __restrict__ sm) {
-  extern __shared__ unsigned long long key[];  // LPT_MAX entries
-  const int b = blockIdx.x;
+  __shared__ unsigned long long key[LPT_MAX];
   const int n = sm->counts[b];
   if (n <= 1 || n > LPT_MAX) return;
   int* list = lists.rows[b];
@@ -412,12 +412,9 @@ __global__ void __launch_bounds__(1024) k_sort_lists(HeavyLists lists, const int
   for (int x = threadIdx.x; x < n; x += blockDim.x) list[x] = (int)(unsigned)(key[x] & 0xffffffffu);
 }
 
-cudaError_t launch_sort_lists(cudaStream_t st, const HeavyLists& lists, const int* f, int rb, const Small* small) {
-  // (per call: the attribute is per device, and a process may drive several)
-  cudaError_t e = cudaFuncSetAttribute(k_sort_lists, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                       LPT_MAX * (int)sizeof(unsigned long long));
-  if (e != cudaSuccess) return e;
-  k_sort_lists<<<NUM_BINS, 1024, LPT_MAX * sizeof(unsigned long long), st>>>(lists, f, rb, small);
+cudaError_t launch_sort_list(cudaStream_t st, const HeavyLists& lists, int bin, const int* f, int rb,
+                             const Small* small) {
+  k_sort_lists<<<1, 1024, 0, st>>>(lists, bin, f, rb, small);
   return cudaGetLastError();
 }
 

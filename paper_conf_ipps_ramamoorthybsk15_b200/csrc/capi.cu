@@ -79,7 +79,9 @@ struct spg_ctx {
   // options
   int light_max = LIGHT_MAX_DEFAULT, tile_cap = TILE_CAP_DEFAULT, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
-  int pack_b = 0;  // numeric: gather B through a packed {column, value} copy (SPG_PACK_B=1)
+  // numeric: gather B through a packed {column, value} copy — one sector per gather instead of
+  // two when B does not stay in L2 (auto: B's columns + values > 64 MB; SPG_PACK_B=0/1 forces)
+  int pack_b = -1;
   // workspace: analysis (all rows / all A entries), classification (this rank's rows), R, windows
   DevBuf f, nz, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, EQ, fl8, dup, nd, ne, chunk_row, packB, Pf,
       splits, canonB[4], iota, ones, crow_tmp;
@@ -222,6 +224,12 @@ spg_status run_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* 
       long long grid = (long long)h->occ_heavy[b] * h->sms;
       if (h->huge_slots_opt > 0 && h->huge_slots_opt < grid) grid = h->huge_slots_opt;
       const int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
+      if (b != BIN_HEAVY && Mloc > 0) {  // largest rows first (the HEAVY bin's list is too long to pay)
+        HeavyLists L3;
+        for (int c = 0; c < NUM_BINS; ++c) L3.rows[c] = h->lists.as<int>() + (size_t)c * (size_t)Mloc;
+        CK(launch_sort_list(st, L3, b, h->f.as<int>(), h->rb, ds));
+        h->launches++;
+      }
       CK(launch_heavy_rank(b, st, (int)grid, P, list, ds->counts + b, B->ncols));
       h->launches++;
       if (conc) {
@@ -391,10 +399,6 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(cudaMemsetAsync(PL, 0, sizeof(long long), h->stream));
     CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm,
                        h->cls.as<uint8_t>(), h->fl.as<int>(), h->Ro.as<long long>(), L3, ds, crow));
-    if (Mloc > 0) {
-      CK(launch_sort_lists(h->stream, L3, h->f.as<int>(), h->rb, ds));
-      h->launches++;
-    }
     CK(launch_incl_scan<int>(h->stream, h->fl.as<int>(), PL + 1, Mloc, h->scan_tmp.as<long long>()));
     long long r_cap = h->EQ.p && h->fl8.p ? (long long)(h->EQ.cap / sizeof(int2)) : 0;
     if (r_cap > (long long)h->fl8.cap) r_cap = (long long)h->fl8.cap;
@@ -511,7 +515,8 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
     P.mloc = h->re - h->rb;
     P.nB = B->nnz;
     P.packB = nullptr;
-    if (h->pack_b && B->nnz > 0) {
+    const bool pack = h->pack_b > 0 || (h->pack_b < 0 && (long long)B->nnz * (4 + (long long)sizeof(V)) > (64LL << 20));
+    if (pack && B->nnz > 0) {
       CK(h->packB.ensure((size_t)B->nnz * (sizeof(V) == 8 ? 16 : 8)));
       P.packB = h->packB.p;
     }

@@ -115,6 +115,15 @@ __global__ void __launch_bounds__(NUM_NT, 5) k_numeric(NumProb<V> P) {
     const int n = (int)min((long long)NUM_CH, P.nnz - base);
     const int r0 = P.chunk_row[ch];
     const int r1 = ch + 1 < P.nch ? P.chunk_row[ch + 1] : P.mloc - 1;
+    // a chunk inside one row (half of webbase1m's chunks: heavy rows) needs no row heads, no
+    // shared memory and no barrier
+    const bool one = r0 == r1;
+    long long nd1 = 0;
+    int ne1 = 0;
+    if (one) {
+      nd1 = P.nd[r0];
+      ne1 = P.ne[r0];
+    } else {
     {
       int4* h4 = reinterpret_cast<int4*>(s_head);
       h4[2 * tid] = make_int4(0, 0, 0, 0);
@@ -160,15 +169,21 @@ __global__ void __launch_bounds__(NUM_NT, 5) k_numeric(NumProb<V> P) {
       h4[2 * tid + 1] = y;
     }
     __syncthreads();
+    }
     // outputs o = base + k·NUM_NT + tid: plan loads, then gathers, then stores (all batched)
     int e[NUM_PT], q[NUM_PT];
 #pragma unroll
     for (int k = 0; k < NUM_PT; ++k) {
       const int s = k * NUM_NT + tid;
       const bool ok = s < n;
-      const int h = ok ? s_head[s] - 1 : 0;
-      const long long src = base + s + s_nd[h];
-      const int es = s_ne[h];
+      long long d = nd1;
+      int es = ne1;
+      if (!one) {
+        const int h = ok ? s_head[s] - 1 : 0;
+        d = s_nd[h];
+        es = s_ne[h];
+      }
+      const long long src = base + s + d;
       const bool plan = ok && es < 0;
       const int2 eq = plan ? __ldcs(P.EQ + src) : make_int2(es, (int)src);
       e[k] = ok ? eq.x : -1;
@@ -198,7 +213,7 @@ __global__ void __launch_bounds__(NUM_NT, 5) k_numeric(NumProb<V> P) {
         __stcs(P.cval + base + s, va[k] * vb[k]);
       }
     }
-    __syncthreads();
+    if (!one) __syncthreads();
   }
 }
 

@@ -124,7 +124,8 @@ cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_
 cudaError_t launch_tiles(cudaStream_t st, int sms, const int* f, int rb, int re, int tile_cap, const uint8_t* cls,
                          const long long* PL, long long* Ro, uint8_t* tflag, int* tiles, Small* small,
                          long long r_cap);
-cudaError_t launch_sort_lists(cudaStream_t st, const HeavyLists& lists, const int* f, int rb, const Small* small);
+cudaError_t launch_sort_list(cudaStream_t st, const HeavyLists& lists, int bin, const int* f, int rb,
+                             const Small* small);
 size_t scan_tmp_elems(long long n);
 int scan_launches(long long n);
 template <typename Tin>

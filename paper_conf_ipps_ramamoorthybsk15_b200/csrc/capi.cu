@@ -82,6 +82,7 @@ struct spg_ctx {
   // numeric: gather B through a packed {column, value} copy — one sector per gather instead of
   // two when B does not stay in L2 (auto: B's columns + values > 64 MB; SPG_PACK_B=0/1 forces)
   int pack_b = -1;
+  int thresholds_set = 0;  // light_max / tile_cap set by the caller (else N-dependent defaults)
   // workspace: analysis (all rows / all A entries), classification (this rank's rows), R, windows
   DevBuf f, nz, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, EQ, fl8, dup, nd, ne, chunk_row, packB, Pf,
       splits, canonB[4], iota, ones, crow_tmp;
@@ -390,7 +391,15 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
       h->hr->splits[1] = M;
     }
     Mloc = h->re - h->rb;
-    ClassParams prm{h->light_max, h->heavy_max, h->tile_cap, h->force, h->canonical ? 1 : 0};
+    // Default thresholds depend on the column count: with N > 2^20 a bitmap row spans several
+    // column tiles (its per-row cost multiplies), so more rows go to the light tiles (measured on
+    // rmat23: symbolic 329 -> 275 ms).  Explicitly set options are kept as given.
+    int light_max = h->light_max, tile_cap = h->tile_cap;
+    if (!h->thresholds_set && B->ncols > (1 << 20)) {
+      light_max = TILE_PMAX - 1024;
+      tile_cap = 1024;
+    }
+    ClassParams prm{light_max, h->heavy_max, tile_cap, h->force, h->canonical ? 1 : 0};
     int* lists = h->lists.as<int>();
     HeavyLists L3;
     for (int b = 0; b < NUM_BINS; ++b) L3.rows[b] = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
@@ -402,7 +411,7 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(launch_incl_scan<int>(h->stream, h->fl.as<int>(), PL + 1, Mloc, h->scan_tmp.as<long long>()));
     long long r_cap = h->EQ.p && h->fl8.p ? (long long)(h->EQ.cap / sizeof(int2)) : 0;
     if (r_cap > (long long)h->fl8.cap) r_cap = (long long)h->fl8.cap;
-    CK(launch_tiles(h->stream, h->sms, h->f.as<int>(), h->rb, h->re, h->tile_cap, h->cls.as<uint8_t>(), PL,
+    CK(launch_tiles(h->stream, h->sms, h->f.as<int>(), h->rb, h->re, tile_cap, h->cls.as<uint8_t>(), PL,
                     h->Ro.as<long long>(), h->tflag.as<uint8_t>(), h->tiles.as<int>(), ds, r_cap));
     h->launches += (Mloc > 0) + scan_launches(Mloc) + 1;
     if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));
@@ -639,11 +648,13 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
       if (v < 0 || v + h->tile_cap > TILE_PMAX)
         return setf(h, SPG_ERR_INVALID_ARGUMENT, "LIGHT_MAX_FLOPS must be in [0, %d - TILE_FLOPS]", TILE_PMAX);
       h->light_max = (int)v;
+      h->thresholds_set = 1;
       break;
     case SPG_OPT_TILE_FLOPS:
       if (v < 1 || v + h->light_max > TILE_PMAX)
         return setf(h, SPG_ERR_INVALID_ARGUMENT, "TILE_FLOPS must be in [1, %d - LIGHT_MAX_FLOPS]", TILE_PMAX);
       h->tile_cap = (int)v;
+      h->thresholds_set = 1;
       break;
     case SPG_OPT_HEAVY_MAX_FLOPS:
       if (v < 0 || v > HEAVY_CAP) return setf(h, SPG_ERR_INVALID_ARGUMENT, "HEAVY_MAX_FLOPS must be in [0, %d]", HEAVY_CAP);

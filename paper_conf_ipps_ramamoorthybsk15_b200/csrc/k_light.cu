@@ -75,7 +75,8 @@ __device__ __forceinline__ int2 block_scan2(int a, int b, int2& tot, int2* scrat
 
 // Shared-memory layout of one tile block (bytes).
 struct LightSmem {
-  static constexpr int keys = 0;                                   // int[PMAX]    slot -> column (sign: not head)
+  static constexpr int keys = 0;                                   // int[PMAX]    idx -> column (expand), then
+                                                                   //              slot -> column (sign: not head)
   static constexpr int sq = keys + TILE_PMAX * 4;                  // int[PMAX]    idx -> B entry
   static constexpr int se = sq + TILE_PMAX * 4;                    // u16[PMAX]    idx -> batch A entry
   static constexpr int sidx = se + TILE_PMAX * 2;                  // u16[PMAX]    slot -> product index
@@ -257,6 +258,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
               const int b0 = s_bb[jr], nb = s_bb[jr + 1] - b0;
               const int b = b0 + (int)(((unsigned long long)(unsigned)col[x] * (unsigned)nb) >> lgN);
               const int idx = pc + jw0 + x * 32 + lane;
+              keys[idx] = col[x];
               se[idx] = (unsigned short)sae[rr[x]];
               sq[idx] = q[x];
               exb[idx] = (unsigned short)b;
@@ -303,25 +305,25 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       __syncthreads();
 
       // ---- pass 2: scatter into buckets; afterwards cnt[b] = end of bucket b -----------------
-      //      (columns re-gathered from B through L1/L2 rather than kept per product in shared
-      //      memory: that keeps two 512-thread blocks per SM at 4096 products per tile)
-      for (int i0 = tid; i0 < Pb; i0 += 4 * NT) {
-        int bk[4], cl[4];
+      //      (the expand pass parked every product's column in keys[idx]; all of them are read
+      //      into registers before the first slot is overwritten)
+      constexpr int IPT = TILE_PMAX / TILE_NT;
+      int bk[IPT], cl[IPT];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const int idx = i0 + u * NT;
-          bk[u] = idx < Pb ? (int)exb[idx] : -1;
-          cl[u] = idx < Pb ? __ldg(P.colB + sq[idx]) : 0;
-        }
+      for (int u = 0; u < IPT; ++u) {
+        const int idx = tid + u * NT;
+        bk[u] = idx < Pb ? (int)exb[idx] : -1;
+        cl[u] = idx < Pb ? keys[idx] : 0;
+      }
+      __syncthreads();
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const int b = bk[u];
-          if (b < 0 || s_bad[brow[b]]) continue;
-          const int slot = atomicAdd(&cnt[b], 1);
-          keys[slot] = cl[u];
-          sidx[slot] = (unsigned short)(i0 + u * NT);
-          sbk[slot] = (unsigned short)b;
-        }
+      for (int u = 0; u < IPT; ++u) {
+        const int b = bk[u];
+        if (b < 0 || s_bad[brow[b]]) continue;
+        const int slot = atomicAdd(&cnt[b], 1);
+        keys[slot] = cl[u];
+        sidx[slot] = (unsigned short)(tid + u * NT);
+        sbk[slot] = (unsigned short)b;
       }
       __syncthreads();
       const int Pg = NBt > 0 ? cnt[NBt - 1] : 0;

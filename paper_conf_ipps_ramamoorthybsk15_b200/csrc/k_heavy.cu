@@ -249,8 +249,21 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
         const unsigned x = u < nl1 ? l1[u] : 0u;
         int pc = 0;
         unsigned short q4[4] = {0, 0, 0, 0};
-        if (x) {
-          // all 32 words of the superblock; the 16-byte reads are rotated by lane so a warp's
+        if (x && __popc(x) <= 8) {
+          // sparse superblock (the common case: a heavy row touches ~3 of its 32 words): count
+          // the touched words only; per 256-column block a 16-bit field of one 64-bit sum
+          unsigned long long acc = 0;
+          for (unsigned y = x; y; y &= y - 1) {
+            const int b = __ffs(y) - 1;
+            acc += (unsigned long long)__popc(bm[(u << 5) + b]) << (16 * (b >> 3));
+          }
+          const int s0 = (int)(acc & 0xffff), s1 = (int)((acc >> 16) & 0xffff), s2 = (int)((acc >> 32) & 0xffff);
+          q4[1] = (unsigned short)s0;
+          q4[2] = (unsigned short)(s0 + s1);
+          q4[3] = (unsigned short)(s0 + s1 + s2);
+          pc = s0 + s1 + s2 + (int)(acc >> 48);
+        } else if (x) {
+          // dense superblock: all 32 words; the 16-byte reads are rotated by lane so a warp's
           // loads spread over all banks (a straight walk would be a 32-way conflict)
           int sub[4] = {0, 0, 0, 0};
 #pragma unroll

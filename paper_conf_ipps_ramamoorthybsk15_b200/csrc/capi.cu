@@ -204,7 +204,7 @@ spg_status run_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* 
     cudaStream_t st = conc ? h->aux[0] : h->stream;
     if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
     if (tm) CK(cudaEventRecord(h->ev_p[0], st));
-    CK(launch_light_rank(st, h->occ_light * h->sms, P, h->tiles.as<int>(), &ds->ntiles, h->tflag.as<uint8_t>(),
+    CK(launch_light_rank(st, h->occ_light * h->sms, P, h->tiles.as<int>(), &ds->ntiles, &ds->tqhead, h->tflag.as<uint8_t>(),
                          h->PL.as<long long>(), h->fblist.as<int>(), ds->fb));
     h->launches++;
     if (tm) CK(cudaEventRecord(h->ev_p[1], st));

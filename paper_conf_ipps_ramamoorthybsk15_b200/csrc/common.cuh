@@ -28,11 +28,17 @@ constexpr int TILE_CAP_DEFAULT = 2048;
 constexpr int LIGHT_MAX_DEFAULT = 2048;
 constexpr int TILE_NT = 512;          // threads per tile block
 constexpr int TILE_RM = 512;          // light rows per batch
-constexpr int TILE_BK = 4;            // expected products per bucket
+#ifndef SPG_TILE_BK
+#define SPG_TILE_BK 2
+#endif
+constexpr int TILE_BK = SPG_TILE_BK;   // expected products per bucket
 constexpr int TILE_NBMAX = TILE_PMAX / TILE_BK + TILE_RM;  // buckets per batch (ceil per row)
 // Heavy (bitmap) kernel geometry.
 constexpr int HEAVY_CAP = 8192;       // largest f of the register-cached bitmap mode (1024 threads)
-constexpr int HEAVY1_CAP = 4096;      // ... 512-thread blocks, two per SM
+#ifndef SPG_HEAVY1_CAP
+#define SPG_HEAVY1_CAP 4096
+#endif
+constexpr int HEAVY1_CAP = SPG_HEAVY1_CAP;  // ... 512-thread blocks, two per SM
 constexpr int BMP_NT = 1024;
 constexpr int BMP_NT_S = 512;
 

@@ -27,6 +27,23 @@
 
 namespace spg {
 
+// Phase timing (experiments only: nvcc -DSPG_PHASE_PROF): clock64 deltas per phase, thread 0 of
+// every block, summed into spg_phase_clk.
+#ifdef SPG_PHASE_PROF
+__device__ unsigned long long spg_phase_clk[16];
+#define SPG_PH(i)                                                               \
+  do {                                                                          \
+    if (threadIdx.x == 0) {                                                     \
+      const long long now_ = clock64();                                         \
+      if (ph_last_ >= 0) atomicAdd(&spg_phase_clk[ph_id_], (unsigned long long)(now_ - ph_last_)); \
+      ph_last_ = now_;                                                          \
+      ph_id_ = (i);                                                             \
+    }                                                                           \
+  } while (0)
+#else
+#define SPG_PH(i) do { } while (0)
+#endif
+
 constexpr int TILE_MAXB = 48;
 constexpr int TILE_EU = 4;  // 32-product windows per warp per step (loads in flight)
 
@@ -99,7 +116,7 @@ struct LightSmem {
 };
 
 __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __restrict__ tiles,
-                                                        const int* __restrict__ ntiles,
+                                                        const int* __restrict__ ntiles, int* __restrict__ tqhead,
                                                         const uint8_t* __restrict__ tflag,
                                                         const long long* __restrict__ PL, int* __restrict__ fb_list,
                                                         int* __restrict__ fb_count) {
@@ -136,11 +153,24 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
   if (!*P.r_ok) return;
   const int nt = *ntiles;
 
-  for (int t = blockIdx.x; t < nt; t += gridDim.x) {
+#ifdef SPG_PHASE_PROF
+  long long ph_last_ = -1;
+  int ph_id_ = 0;
+#endif
+  // tiles from a dynamic queue (their cost varies with their rows' shapes; static striding left
+  // a tail)
+  __shared__ int s_tile;
+  for (;;) {
+    if (tid == 0) s_tile = atomicAdd(tqhead, 1);
+    __syncthreads();
+    const int t = s_tile;
+    __syncthreads();
+    if (t >= nt) break;
     const int s = tiles[t];
     int cur = s;
     bool done = false;
     while (!done) {
+      SPG_PH(0);
       // ---- collect a batch: light rows from `cur` up to the next tile start, <= TILE_RM rows ----
       int nr = 0;
       for (;;) {
@@ -169,6 +199,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       __syncthreads();
       if (nr == 0) break;
 
+      SPG_PH(1);
       // ---- rows: A range, bucket count; prefixes over the batch ----------------------------
       int a0 = 0, a1 = 0, n0 = 0, n1 = 0;  // two rows per thread (TILE_RM = 2 * NT)
       {
@@ -209,6 +240,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       }
       __syncthreads();
 
+      SPG_PH(2);
       // ---- pass 1: expand columns, bucket of every product, bucket sizes ---------------------
       int pc = 0;  // products before this chunk
       for (int u0 = 0; u0 < AE; u0 += NT) {
@@ -270,6 +302,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       }
       const int Pb = pc;
 
+      SPG_PH(3);
       // ---- clustered columns: hand the row to the bitmap kernel -----------------------------
       int badb = 0;
       for (int b = tid; b < NBt; b += NT)
@@ -283,6 +316,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
         __syncthreads();
       }
 
+      SPG_PH(4);
       // ---- bucket starts (exclusive scan, contiguous ownership) ------------------------------
       constexpr int BPT = (TILE_NBMAX + NT - 1) / NT;
       {
@@ -304,6 +338,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       }
       __syncthreads();
 
+      SPG_PH(5);
       // ---- pass 2: scatter into buckets; afterwards cnt[b] = end of bucket b -----------------
       //      (the expand pass parked every product's column in keys[idx]; all of them are read
       //      into registers before the first slot is overwritten)
@@ -328,6 +363,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       __syncthreads();
       const int Pg = NBt > 0 ? cnt[NBt - 1] : 0;
 
+      SPG_PH(6);
       // ---- heads: first slot of its column within the bucket -------------------------------
       for (int x = tid; x < Pg; x += NT) {
         const int b = sbk[x];
@@ -366,6 +402,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       }
       __syncthreads();
 
+      SPG_PH(7);
       // ---- ranks: heads of the row's earlier buckets + distinct smaller columns in the bucket;
       //      heads -> gather plan (slots are in (row, bucket) order: nearly coalesced), others
       //      -> dup list --------------------------------------------------------------------
@@ -396,6 +433,7 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
       for (int j = tid; j < nr; j += NT)
         if (!s_bad[j]) P.crow[s_row[j] + 1] = hc[s_bb[j + 1]] - hc[s_bb[j]];
       __syncthreads();
+      SPG_PH(8);
     }
   }
 }
@@ -410,10 +448,21 @@ int light_occupancy() {
   return nb < 1 ? 1 : nb;
 }
 
-cudaError_t launch_light_rank(cudaStream_t st, int grid, const SymProb& P, const int* tiles, const int* ntiles,
+cudaError_t launch_light_rank(cudaStream_t st, int grid, const SymProb& P, const int* tiles, const int* ntiles, int* tqhead,
                               const uint8_t* tflag, const long long* PL, int* fb_list, int* fb_count) {
-  k_light_rank<<<grid, TILE_NT, LightSmem::bytes, st>>>(P, tiles, ntiles, tflag, PL, fb_list, fb_count);
+  k_light_rank<<<grid, TILE_NT, LightSmem::bytes, st>>>(P, tiles, ntiles, tqhead, tflag, PL, fb_list, fb_count);
   return cudaGetLastError();
 }
 
 }  // namespace spg
+
+#ifdef SPG_PHASE_PROF
+extern "C" int spg_debug_phase_clk(unsigned long long* out, int reset) {
+  cudaMemcpyFromSymbol(out, spg::spg_phase_clk, 16 * sizeof(unsigned long long));
+  if (reset) {
+    unsigned long long z[16] = {};
+    cudaMemcpyToSymbol(spg::spg_phase_clk, z, sizeof z);
+  }
+  return 0;
+}
+#endif

@@ -40,7 +40,7 @@ struct Small {
   int r_ok;                 // EQ capacity sufficient (written by k_tiles)
   int amax;                 // longest row of A
   int nch_need;             // numeric chunks (+1) the plan needed
-  int pad0;
+  int tqhead;               // light tiles: dynamic queue head
   unsigned long long dupn;  // non-first products (dup list entries)
   long long heavy_total;    // products of heavy rows (EQ offsets of heavy rows, relative)
   long long fr;             // products of rows with a gather plan (light + heavy)
@@ -142,7 +142,7 @@ cudaError_t launch_narrow(cudaStream_t st, const long long* in, int* out, long l
 // k_light.cu — symbolic ranks of the light rows, one tile per block iteration.
 cudaError_t light_configure();
 int light_occupancy();
-cudaError_t launch_light_rank(cudaStream_t st, int grid, const SymProb& P, const int* tiles, const int* ntiles,
+cudaError_t launch_light_rank(cudaStream_t st, int grid, const SymProb& P, const int* tiles, const int* ntiles, int* tqhead,
                               const uint8_t* tflag, const long long* PL, int* fb_list, int* fb_count);
 
 // k_heavy.cu — symbolic ranks of heavy rows (column bitmap), per bin or over an explicit list.

@@ -179,7 +179,8 @@ __global__ void __launch_bounds__(CL_NT) k_classify(const int* __restrict__ f, c
 
 // Tiles of light rows.  PL = exclusive prefix of fl (light products, row order).  A light row
 // starts a tile when its product range [PL_i, PL_i + f_i) contains a multiple of `cap` (so a
-// tile holds < cap + light_max products).  Light rows get Ro = PL_i, heavy rows Ro += F_L.
+// tile holds < cap + light_max products).  Light rows get Ro = F_H + PL_i: the plan holds the heavy
+// rows first (their offsets come from k_classify alone, so the heavy kernels start before this).
 // r_ok = (F_L + F_H <= capacity of R): the symbolic kernels do nothing when R is too small and
 // the host re-runs them after growing R.
 __global__ void __launch_bounds__(256) k_tiles(const int* __restrict__ f, int rb, int re, int cap,
@@ -187,7 +188,7 @@ __global__ void __launch_bounds__(256) k_tiles(const int* __restrict__ f, int rb
                                                long long* __restrict__ Ro, uint8_t* __restrict__ tflag,
                                                int* __restrict__ tiles, Small* __restrict__ sm, long long r_cap) {
   const long long n = (long long)re - rb;
-  const long long FL = PL[n];
+  const long long FL = PL[n], HT = sm->heavy_total;
   const int lane = threadIdx.x & 31;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     const long long fr = FL + sm->heavy_total;
@@ -203,10 +204,8 @@ __global__ void __launch_bounds__(256) k_tiles(const int* __restrict__ f, int rb
       if (c & CLS_LIGHT_PATH) {
         const long long pl = PL[li];
         const long long fi = f[rb + li];
-        Ro[li] = pl;
+        Ro[li] = HT + pl;
         start = (pl % cap == 0) || (pl / cap != (pl + fi - 1) / cap);
-      } else if ((c & 7) == CLS_HEAVY || (c & 7) == CLS_HUGE) {
-        Ro[li] += FL;
       }
       tflag[li] = start ? 1 : 0;
     }

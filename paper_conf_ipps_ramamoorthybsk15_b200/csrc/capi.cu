@@ -91,7 +91,7 @@ struct spg_ctx {
   long long iota_n = -1, ones_n = -1;
   HostRead* hr = nullptr;
   cudaStream_t aux[6] = {};
-  cudaEvent_t ev_fork = nullptr, ev_join[6] = {};
+  cudaEvent_t ev_fork = nullptr, ev_fork2 = nullptr, ev_join[6] = {};
   cudaEvent_t ev_t[8] = {};
   cudaEvent_t ev_p[4] = {};  // light path start/end, heavy path start/end
   int occ_light = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1;
@@ -182,30 +182,65 @@ SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* cr
   P.fl8 = h->fl8.as<uint8_t>();
   P.crow = crow;
   P.r_ok = &h->small.as<Small>()->r_ok;
+  P.heavy_total = &h->small.as<Small>()->heavy_total;
+  {
+    long long r_cap = h->EQ.p && h->fl8.p ? (long long)(h->EQ.cap / sizeof(int2)) : 0;
+    if (r_cap > (long long)h->fl8.cap) r_cap = (long long)h->fl8.cap;
+    P.r_cap = r_cap;
+  }
   P.row_begin = h->rb;
   P.row_end = h->re;
   P.lgN = ceil_log2(B->ncols);
   return P;
 }
 
-// Symbolic class kernels: light tiles and the heavy bitmap bins on concurrent streams (the
+// Symbolic class kernels: the heavy bitmap bins and the light tiles on concurrent streams (the
 // paper's concurrent CPU and GPU legs of Phases II/III, recast as
 // concurrent kernels on one GPU), then the rows the light kernel handed over.  Bin sizes are
 // device-side: every kernel is a persistent grid that exits at once when its list is empty.
-spg_status run_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
+// The heavy bins fork right after k_classify (their plan offsets are final there), so they
+// overlap the light-product scan and the tile cut; the light tiles fork after k_tiles.
+spg_status run_heavy(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
   const SymProb P = make_sym(h, A, B, crow);
   Small* ds = h->small.as<Small>();
   const bool conc = h->concurrent != 0;
-  CK(cudaMemsetAsync(ds->qhead, 0, sizeof(ds->qhead) + sizeof(ds->fb), h->stream));
-  if (conc) CK(cudaEventRecord(h->ev_fork, h->stream));
   const bool tm = h->timing != 0;
-  // light tiles
+  if (conc) CK(cudaEventRecord(h->ev_fork, h->stream));
+  const long long Mloc = h->re - h->rb;
+  const int order[NUM_BINS] = {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY};
+  for (int x = 0; x < NUM_BINS; ++x) {
+    const int b = order[x];
+    cudaStream_t st = conc ? h->aux[1 + x] : h->stream;
+    if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
+    if (tm && x == 0) CK(cudaEventRecord(h->ev_p[2], st));
+    long long grid = (long long)h->occ_heavy[b] * h->sms;
+    if (h->huge_slots_opt > 0 && h->huge_slots_opt < grid) grid = h->huge_slots_opt;
+    const int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
+    if (b != BIN_HEAVY && Mloc > 0) {  // largest rows first (the HEAVY bin's list is too long to pay)
+      HeavyLists L3;
+      for (int c = 0; c < NUM_BINS; ++c) L3.rows[c] = h->lists.as<int>() + (size_t)c * (size_t)Mloc;
+      CK(launch_sort_list(st, L3, b, h->f.as<int>(), h->rb, ds));
+      h->launches++;
+    }
+    CK(launch_heavy_rank(b, st, (int)grid, P, list, ds->counts + b, B->ncols, 0));
+    h->launches++;
+    if (conc) CK(cudaEventRecord(h->ev_join[1 + x], st));
+  }
+  return SPG_OK;
+}
+
+spg_status run_light(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
+  const SymProb P = make_sym(h, A, B, crow);
+  Small* ds = h->small.as<Small>();
+  const bool conc = h->concurrent != 0;
+  const bool tm = h->timing != 0;
+  if (conc) CK(cudaEventRecord(h->ev_fork2, h->stream));
   {
     cudaStream_t st = conc ? h->aux[0] : h->stream;
-    if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
+    if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork2, 0));
     if (tm) CK(cudaEventRecord(h->ev_p[0], st));
-    CK(launch_light_rank(st, h->occ_light * h->sms, P, h->tiles.as<int>(), &ds->ntiles, &ds->tqhead, h->tflag.as<uint8_t>(),
-                         h->PL.as<long long>(), h->fblist.as<int>(), ds->fb));
+    CK(launch_light_rank(st, h->occ_light * h->sms, P, h->tiles.as<int>(), &ds->ntiles, &ds->tqhead,
+                         h->tflag.as<uint8_t>(), h->PL.as<long long>(), h->fblist.as<int>(), ds->fb));
     h->launches++;
     if (tm) CK(cudaEventRecord(h->ev_p[1], st));
     if (conc) {
@@ -213,37 +248,13 @@ spg_status run_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* 
       CK(cudaStreamWaitEvent(h->stream, h->ev_join[0], 0));
     }
   }
-  // heavy bins, each on its own stream (the HUGE bin's long rows overlap the others' work)
-  {
-    const long long Mloc = h->re - h->rb;
-    const int order[NUM_BINS] = {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY};
-    for (int x = 0; x < NUM_BINS; ++x) {
-      const int b = order[x];
-      cudaStream_t st = conc ? h->aux[1 + x] : h->stream;
-      if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
-      if (tm && x == 0) CK(cudaEventRecord(h->ev_p[2], st));
-      long long grid = (long long)h->occ_heavy[b] * h->sms;
-      if (h->huge_slots_opt > 0 && h->huge_slots_opt < grid) grid = h->huge_slots_opt;
-      const int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
-      if (b != BIN_HEAVY && Mloc > 0) {  // largest rows first (the HEAVY bin's list is too long to pay)
-        HeavyLists L3;
-        for (int c = 0; c < NUM_BINS; ++c) L3.rows[c] = h->lists.as<int>() + (size_t)c * (size_t)Mloc;
-        CK(launch_sort_list(st, L3, b, h->f.as<int>(), h->rb, ds));
-        h->launches++;
-      }
-      CK(launch_heavy_rank(b, st, (int)grid, P, list, ds->counts + b, B->ncols));
-      h->launches++;
-      if (conc) {
-        CK(cudaEventRecord(h->ev_join[1 + x], st));
-        CK(cudaStreamWaitEvent(h->stream, h->ev_join[1 + x], 0));
-      }
-    }
-    if (tm) CK(cudaEventRecord(h->ev_p[3], h->stream));
-  }
+  if (conc)
+    for (int x = 0; x < NUM_BINS; ++x) CK(cudaStreamWaitEvent(h->stream, h->ev_join[1 + x], 0));
+  if (tm) CK(cudaEventRecord(h->ev_p[3], h->stream));
   h->paths_timed = tm;
   // rows with clustered columns, handed over by the light kernel
   long long grid = (long long)h->occ_heavy[BIN_HUGE] * h->sms;
-  CK(launch_heavy_rank(BIN_HUGE, h->stream, (int)grid, P, h->fblist.as<int>(), ds->fb, B->ncols));
+  CK(launch_heavy_rank(BIN_HUGE, h->stream, (int)grid, P, h->fblist.as<int>(), ds->fb, B->ncols, 1));
   h->launches++;
   return SPG_OK;
 }
@@ -408,6 +419,8 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(cudaMemsetAsync(PL, 0, sizeof(long long), h->stream));
     CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm,
                        h->cls.as<uint8_t>(), h->fl.as<int>(), h->Ro.as<long long>(), L3, ds, crow));
+    CK(cudaMemsetAsync(ds->qhead, 0, sizeof(ds->qhead) + sizeof(ds->fb), h->stream));
+    if ((s = run_heavy(h, A, B, crow)) != SPG_OK) return s;
     CK(launch_incl_scan<int>(h->stream, h->fl.as<int>(), PL + 1, Mloc, h->scan_tmp.as<long long>()));
     long long r_cap = h->EQ.p && h->fl8.p ? (long long)(h->EQ.cap / sizeof(int2)) : 0;
     if (r_cap > (long long)h->fl8.cap) r_cap = (long long)h->fl8.cap;
@@ -415,7 +428,7 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
                     h->Ro.as<long long>(), h->tflag.as<uint8_t>(), h->tiles.as<int>(), ds, r_cap));
     h->launches += (Mloc > 0) + scan_launches(Mloc) + 1;
     if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));
-    if ((s = run_sym(h, A, B, crow)) != SPG_OK) return s;
+    if ((s = run_light(h, A, B, crow)) != SPG_OK) return s;
     CK(launch_incl_scan<long long>(h->stream, crow + 1, crow + 1, Mloc, h->scan_tmp.as<long long>()));
     // numeric plan: per-row EQ-to-C offsets and chunk -> row (capacity from the last call; a
     // larger need reruns the plan below)
@@ -579,6 +592,7 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     if (e == cudaSuccess && c < 4) e = cudaEventCreate(&h->ev_p[c]);
   }
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_fork2, cudaEventDisableTiming);
   for (int k = 0; k < 8 && e == cudaSuccess; ++k) e = cudaEventCreate(&h->ev_t[k]);
   if (e != cudaSuccess) {
     h->err = cudaGetErrorString(e);
@@ -629,6 +643,7 @@ spg_status spg_spgemm_free(spg_handle h) {
       if (c < 4 && h->ev_p[c]) cudaEventDestroy(h->ev_p[c]);
     }
     if (h->ev_fork) cudaEventDestroy(h->ev_fork);
+    if (h->ev_fork2) cudaEventDestroy(h->ev_fork2);
     for (auto& e : h->ev_t)
       if (e) cudaEventDestroy(e);
     if (h->hr) cudaFreeHost(h->hr);

@@ -48,7 +48,7 @@ __device__ __forceinline__ int bmp_need(int lw, int f) {
 template <int MODE, int NT, int SMEM>
 __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(SymProb P, const int* __restrict__ list,
                                                                               const int* __restrict__ count, int lwmax,
-                                                                              int N) {
+                                                                              int N, int fallback) {
   constexpr int RCAP = NT;
   constexpr bool CACHED = MODE == MODE_CACHED;
   extern __shared__ __align__(16) unsigned char sm[];
@@ -62,7 +62,9 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
   const Group<NT> g{(int)threadIdx.x, scratch};
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const unsigned upto = (2u << lane) - 1u;  // lanes <= me
-  if (!*P.r_ok) return;
+  // bin lists start right after k_classify and need only the heavy part of the plan to fit;
+  // the fallback list (light rows) runs after k_tiles set r_ok
+  if (fallback ? !*P.r_ok : *P.heavy_total > P.r_cap) return;
 
   // invariant between rows: the whole region is zero
   for (int x = tid; x < REGION / 4; x += NT) reinterpret_cast<unsigned*>(region)[x] = 0;
@@ -412,11 +414,11 @@ int heavy_occupancy(int bin) {
 }
 
 cudaError_t launch_heavy_rank(int bin, cudaStream_t st, int grid, const SymProb& P, const int* list,
-                              const int* count, long long N) {
+                              const int* count, long long N, int fallback) {
   int lwmax = 10;
   while (lwmax < 20 && ((long long)1 << lwmax) < N) ++lwmax;
   int n32 = (int)N;
-  void* args[] = {(void*)&P, (void*)&list, (void*)&count, (void*)&lwmax, (void*)&n32};
+  void* args[] = {(void*)&P, (void*)&list, (void*)&count, (void*)&lwmax, (void*)&n32, (void*)&fallback};
   return cudaLaunchKernel(bitmap_kernel(bin), dim3(grid), dim3(bitmap_threads(bin)), args, bitmap_smem(bin), st);
 }
 

@@ -72,6 +72,8 @@ struct SymProb {
   uint8_t* fl8;             // uncached bitmap rows: first-claim flag per product (Ro_i + offset)
   long long* crow;          // C row offsets (local); symbolic writes counts at [li + 1]
   const int* r_ok;
+  const long long* heavy_total;  // heavy rows' plan size (final after k_classify)
+  long long r_cap;               // plan capacity (entries)
   int row_begin, row_end;
   int lgN;                  // ceil(log2 N), N = columns of B
 };
@@ -149,7 +151,7 @@ cudaError_t launch_light_rank(cudaStream_t st, int grid, const SymProb& P, const
 cudaError_t heavy_configure();
 int heavy_occupancy(int bin);
 cudaError_t launch_heavy_rank(int bin, cudaStream_t st, int grid, const SymProb& P, const int* list,
-                              const int* count, long long N);
+                              const int* count, long long N, int fallback);
 
 // k_numeric.cu — numeric plan (end of symbolic) and numeric phase.
 cudaError_t launch_plan(cudaStream_t st, int sms, const long long* crow, int mloc, const int* rpA, const int* colA,

@@ -20,6 +20,10 @@
 // HBM traffic per output: 8 B of EQ read + 12 B (fp64) of C written; A and B mostly from L2.
 #include "kernels.cuh"
 
+#ifndef SPG_EQ_LOAD
+#define SPG_EQ_LOAD 0  // plan loads: 0 streaming (ld.global.cs), 1 read-only path, 2 plain
+#endif
+
 namespace spg {
 
 // ---- plan (end of symbolic) ---------------------------------------------------------------------
@@ -185,7 +189,13 @@ __global__ void __launch_bounds__(NUM_NT, 5) k_numeric(NumProb<V> P) {
       }
       const long long src = base + s + d;
       const bool plan = ok && es < 0;
+#if SPG_EQ_LOAD == 1
+      const int2 eq = plan ? __ldg(P.EQ + src) : make_int2(es, (int)src);
+#elif SPG_EQ_LOAD == 2
+      const int2 eq = plan ? P.EQ[src] : make_int2(es, (int)src);
+#else
       const int2 eq = plan ? __ldcs(P.EQ + src) : make_int2(es, (int)src);
+#endif
       e[k] = ok ? eq.x : -1;
       q[k] = eq.y;
     }

@@ -9,5 +9,8 @@ python tools/ncu_sum.py gpurun_out/launches.csv > gpurun_out/launches_summary.tx
 python tools/traffic.py gpurun_out/launches.csv webbase1m
 timeout 900 python bench.py --out gpurun_out/bench_webbase1m.jsonl > gpurun_out/bench.log 2>&1; tail -1 gpurun_out/bench.log | cut -c1-600
 timeout 600 python bench.py --impl reference --steps 3 --warmup 3 --out gpurun_out/bench_reference.jsonl > gpurun_out/bench_ref.log 2>&1; tail -1 gpurun_out/bench_ref.log | cut -c1-300
+for c in webgoogle citpatents ab2m cl10k; do
+  timeout 600 python bench.py --config $c --steps 20 --warmup 3 --no-cpu-baseline --no-e2e --out gpurun_out/bench_configs.jsonl > gpurun_out/bench_$c.log 2>&1; tail -1 gpurun_out/bench_$c.log | cut -c1-200
+done
 timeout 1200 python bench.py --config rmat23 --steps 5 --warmup 3 --no-cpu-baseline --no-e2e --out gpurun_out/bench_rmat23.jsonl > gpurun_out/bench_rmat.log 2>&1; tail -1 gpurun_out/bench_rmat.log | cut -c1-600
 timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k regex:"k_numeric<" -s 3 -c 1 -o gpurun_out/prof_numeric -f python bench.py --profile > gpurun_out/ncu_full.log 2>&1; echo "ncu full rc=$?"

@@ -109,7 +109,10 @@ typedef enum {
                                    0: the library canonicalises a copy of B                   */
   SPG_OPT_TIMING = 6,           /* 1: record per-phase CUDA-event times into the stats        */
   SPG_OPT_HUGE_SLOTS = 7,       /* max concurrent heavy-row blocks per bin (0 = full occupancy) */
-  SPG_OPT_CONCURRENT = 8        /* 1 (default): light and heavy kernels on concurrent streams  */
+  SPG_OPT_CONCURRENT = 8,       /* 1 (default): light and heavy kernels on concurrent streams  */
+  SPG_OPT_WARP_MAX_FLOPS = 9    /* 0..256, default 0 (off): light rows with f <= this are sorted
+                                   one warp per row in registers (bitonic network) instead of
+                                   in tiles.  Ignored while FORCE_CLASS is set                */
 } spg_option;
 
 typedef struct {

@@ -94,8 +94,10 @@ __device__ __forceinline__ int classify_row(int f, int nz, const ClassParams& p,
   nz &= 0x3f;
   if (p.force < 0 && nz == 1 && p.single_ok) return CLS_SINGLE;
   if (f <= p.light_max && p.force < CLS_HEAVY) {
-    light = true;
-    return f <= TINY_MAX ? CLS_TINY : (f <= LIGHTC_MAX ? CLS_LIGHT : CLS_MEDIUM);
+    const int c = f <= TINY_MAX ? CLS_TINY : (f <= LIGHTC_MAX ? CLS_LIGHT : CLS_MEDIUM);
+    if (f <= p.warp_max && p.force < 0) bin = BIN_WARP;  // one warp per row (k_warp.cu)
+    else light = true;                                   // light tiles (k_light.cu)
+    return c;
   }
   const int hm = min(p.heavy_max, HEAVY_CAP);
   if (p.force == CLS_HUGE || f > hm) bin = BIN_HUGE;

@@ -82,7 +82,9 @@ struct spg_ctx {
   // numeric: gather B through a packed {column, value} copy — one sector per gather instead of
   // two when B does not stay in L2 (auto: B's columns + values > 64 MB; SPG_PACK_B=0/1 forces)
   int pack_b = -1;
-  int thresholds_set = 0;  // light_max / tile_cap set by the caller (else N-dependent defaults)
+  int thresholds_set = 0;
+  int warp_max = WARP_MAX_DEFAULT;  // light rows with f <= warp_max: one warp per row (k_warp.cu)
+  int occ_warp = 1;  // light_max / tile_cap set by the caller (else N-dependent defaults)
   // workspace: analysis (all rows / all A entries), classification (this rank's rows), R, windows
   DevBuf f, nz, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, EQ, fl8, dup, nd, ne, chunk_row, packB, Pf,
       splits, canonB[4], iota, ones, crow_tmp;
@@ -218,13 +220,21 @@ spg_status run_heavy(spg_handle h, const spg_csr* A, const spg_csr* B, long long
     const int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
     if (b != BIN_HEAVY && Mloc > 0) {  // largest rows first (the HEAVY bin's list is too long to pay)
       HeavyLists L3;
-      for (int c = 0; c < NUM_BINS; ++c) L3.rows[c] = h->lists.as<int>() + (size_t)c * (size_t)Mloc;
+      for (int c = 0; c < NUM_LISTS; ++c) L3.rows[c] = h->lists.as<int>() + (size_t)c * (size_t)Mloc;
       CK(launch_sort_list(st, L3, b, h->f.as<int>(), h->rb, ds));
       h->launches++;
     }
     CK(launch_heavy_rank(b, st, (int)grid, P, list, ds->counts + b, B->ncols, 0));
     h->launches++;
     if (conc) CK(cudaEventRecord(h->ev_join[1 + x], st));
+  }
+  {  // the smallest light rows, one warp per row, on their own stream
+    cudaStream_t st = conc ? h->aux[4] : h->stream;
+    if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
+    const int* list = h->lists.as<int>() + (size_t)BIN_WARP * (size_t)(Mloc > 0 ? Mloc : 1);
+    CK(launch_warp_rank(st, h->occ_warp * h->sms, P, list, ds->counts + BIN_WARP));
+    h->launches++;
+    if (conc) CK(cudaEventRecord(h->ev_join[4], st));
   }
   return SPG_OK;
 }
@@ -249,7 +259,7 @@ spg_status run_light(spg_handle h, const spg_csr* A, const spg_csr* B, long long
     }
   }
   if (conc)
-    for (int x = 0; x < NUM_BINS; ++x) CK(cudaStreamWaitEvent(h->stream, h->ev_join[1 + x], 0));
+    for (int x = 0; x < NUM_BINS + 1; ++x) CK(cudaStreamWaitEvent(h->stream, h->ev_join[1 + x], 0));
   if (tm) CK(cudaEventRecord(h->ev_p[3], h->stream));
   h->paths_timed = tm;
   // rows with clustered columns, handed over by the light kernel
@@ -270,7 +280,7 @@ spg_status ensure_ws(spg_handle h, int M, long long nnzA) {
   CK(h->PL.ensure((m + 1) * sizeof(long long)));
   CK(h->tflag.ensure(m));
   CK(h->tiles.ensure(m * sizeof(int)));
-  CK(h->lists.ensure(m * NUM_BINS * sizeof(int)));
+  CK(h->lists.ensure(m * NUM_LISTS * sizeof(int)));
   CK(h->fblist.ensure(m * sizeof(int)));
   CK(h->nd.ensure(m * sizeof(long long)));
   CK(h->ne.ensure(m * sizeof(int)));
@@ -410,10 +420,11 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
       light_max = TILE_PMAX - 1024;
       tile_cap = 1024;
     }
-    ClassParams prm{light_max, h->heavy_max, tile_cap, h->force, h->canonical ? 1 : 0};
+    ClassParams prm{light_max, h->heavy_max, tile_cap, h->force, h->canonical ? 1 : 0,
+                    h->warp_max < light_max ? h->warp_max : light_max};
     int* lists = h->lists.as<int>();
     HeavyLists L3;
-    for (int b = 0; b < NUM_BINS; ++b) L3.rows[b] = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
+    for (int b = 0; b < NUM_LISTS; ++b) L3.rows[b] = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
     long long* PL = h->PL.as<long long>();
     CK(cudaMemsetAsync(crow, 0, sizeof(long long), h->stream));
     CK(cudaMemsetAsync(PL, 0, sizeof(long long), h->stream));
@@ -603,6 +614,7 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
   h->occ_num = dtype == SPG_FP64 ? numeric_occupancy<double>() : numeric_occupancy<float>();
   if (const char* pb = getenv("SPG_PACK_B")) h->pack_b = atoi(pb);
   for (int b = 0; b < NUM_BINS; ++b) h->occ_heavy[b] = heavy_occupancy(b);
+  h->occ_warp = warp_occupancy();
   cudaGetLastError();
   *out = h;
   return SPG_OK;
@@ -688,6 +700,11 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
       h->huge_slots_opt = (int)v;
       break;
     case SPG_OPT_CONCURRENT: h->concurrent = v != 0; break;
+    case SPG_OPT_WARP_MAX_FLOPS:
+      if (v < 0 || v > WARP_MAX_CAP)
+        return setf(h, SPG_ERR_INVALID_ARGUMENT, "WARP_MAX_FLOPS must be in [0, %d]", WARP_MAX_CAP);
+      h->warp_max = (int)v;
+      break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   h->sym_ok = false;
@@ -706,6 +723,7 @@ spg_status spg_get_option(spg_handle h, spg_option opt, int64_t* v) {
     case SPG_OPT_TIMING: *v = h->timing; break;
     case SPG_OPT_HUGE_SLOTS: *v = h->huge_slots_opt; break;
     case SPG_OPT_CONCURRENT: *v = h->concurrent; break;
+    case SPG_OPT_WARP_MAX_FLOPS: *v = h->warp_max; break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   return SPG_OK;

@@ -16,6 +16,11 @@ enum : int { CLS_EMPTY = 0, CLS_SINGLE, CLS_TINY, CLS_LIGHT, CLS_MEDIUM, CLS_HEA
 // the register-cached bitmap kernel (512 threads when f <= HEAVY1_CAP, else 1024); HUGE rows
 // (and rows the light kernel hands over) the uncached bitmap kernel.
 enum : int { BIN_HEAVY = 0, BIN_HEAVY2, BIN_HUGE, NUM_BINS };
+// Row lists: the bitmap bins, then the warp-per-row rows (f <= warp_max, k_warp.cu).
+constexpr int BIN_WARP = NUM_BINS;
+constexpr int NUM_LISTS = NUM_BINS + 1;
+constexpr int WARP_MAX_CAP = 256;      // largest f of the warp-per-row symbolic kernel
+constexpr int WARP_MAX_DEFAULT = 0;  // off: measured slower than the tiles (k_warp.cu header)
 
 // Per-row path code stored in the cls[] array (low 3 bits = class, bit 3 = light path).
 constexpr uint8_t CLS_LIGHT_PATH = 8;

@@ -24,10 +24,11 @@ struct ClassParams {
   int tile_cap;    // nominal products per tile (light_max + tile_cap <= TILE_PMAX)
   int force;       // -1 or a class id >= CLS_TINY
   int single_ok;   // B rows canonical -> SINGLE (identity) shortcut allowed
+  int warp_max;    // light rows with f <= warp_max -> warp-per-row kernel (0: none)
 };
 
 struct HeavyLists {
-  int* rows[NUM_BINS];
+  int* rows[NUM_LISTS];
 };
 
 // Small per-call device scratch (zeroed at the start of every symbolic call).
@@ -146,6 +147,10 @@ cudaError_t light_configure();
 int light_occupancy();
 cudaError_t launch_light_rank(cudaStream_t st, int grid, const SymProb& P, const int* tiles, const int* ntiles, int* tqhead,
                               const uint8_t* tflag, const long long* PL, int* fb_list, int* fb_count);
+
+// k_warp.cu — symbolic plan of the smallest light rows, one warp per row.
+int warp_occupancy();
+cudaError_t launch_warp_rank(cudaStream_t st, int grid, const SymProb& P, const int* list, const int* count);
 
 // k_heavy.cu — symbolic ranks of heavy rows (column bitmap), per bin or over an explicit list.
 cudaError_t heavy_configure();

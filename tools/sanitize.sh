@@ -1,0 +1,22 @@
+# compute-sanitizer passes on small inputs (memcheck: out-of-bounds / misaligned; racecheck and
+# synccheck: shared-memory hazards and barrier misuse in the block-cooperative kernels)
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+cat > /tmp/san_case.py <<'PY'
+import sys, torch, numpy as np
+sys.path.insert(0, ".")
+import paper_conf_ipps_ramamoorthybsk15_b200 as spg, workloads as W
+A, _ = W.make("cl10k")
+dA = spg.DeviceCSR.from_host(A, "cuda:0")
+for opts in ({}, {"warp_max_flops": 256}, {"force_class": 6}, {"light_max_flops": 0}):
+    plan = spg.SpGEMM(0, torch.float64)
+    for k, v in opts.items():
+        plan.set_option(k, v)
+    C = plan(dA, dA)
+    torch.cuda.synchronize()
+    plan.close()
+print("case ok", int(C.row_ptr[-1]))
+PY
+for tool in memcheck racecheck synccheck; do
+  timeout 1500 compute-sanitizer --tool $tool --error-exitcode 9 python /tmp/san_case.py > gpurun_out/san_$tool.log 2>&1
+  echo "$tool rc=$?"; grep -E "ERROR SUMMARY|RACECHECK SUMMARY|case ok" gpurun_out/san_$tool.log | tail -3
+done

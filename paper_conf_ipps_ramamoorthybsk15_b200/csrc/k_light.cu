@@ -45,6 +45,7 @@ __device__ unsigned long long spg_phase_clk[16];
 #endif
 
 constexpr int TILE_MAXB = 48;
+static_assert(TILE_PMAX / TILE_NT <= 32, "head marks of a thread fit one 32-bit mask");
 constexpr int TILE_EU = 4;  // 32-product windows per warp per step (loads in flight)
 
 // Run of product jw + lane for a window starting inside run rb (warp-uniform); advances rb to
@@ -365,16 +366,22 @@ __global__ void __launch_bounds__(TILE_NT) k_light_rank(SymProb P, const int* __
 
       SPG_PH(6);
       // ---- heads: first slot of its column within the bucket -------------------------------
-      for (int x = tid; x < Pg; x += NT) {
+      //      (non-head marks are applied after a barrier, so no thread reads a key while
+      //      another marks it)
+      unsigned nonhead = 0;  // bit u: slot tid + u·NT is not a head (<= TILE_PMAX / NT slots)
+      for (int x = tid, u = 0; x < Pg; x += NT, ++u) {
         const int b = sbk[x];
         const int s0 = b ? cnt[b - 1] : 0;
         const int kx = keys[x];
         bool head = true;
         for (int y = s0; y < x; ++y)
-          if ((keys[y] & 0x7fffffff) == kx) { head = false; break; }
+          if (keys[y] == kx) { head = false; break; }
         if (head) atomicAdd(&hc[b], 1);
-        else keys[x] = kx | int(0x80000000);
+        else nonhead |= 1u << u;
       }
+      __syncthreads();
+      for (int x = tid, u = 0; x < Pg; x += NT, ++u)
+        if (nonhead >> u & 1u) keys[x] |= int(0x80000000);
       __syncthreads();
       {  // head prefix per bucket; hc[NBt] = total
         int c8[BPT], mine = 0;

@@ -412,11 +412,13 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
       h->hr->splits[1] = M;
     }
     Mloc = h->re - h->rb;
-    // Default thresholds depend on the column count: with N > 2^20 a bitmap row spans several
-    // column tiles (its per-row cost multiplies), so more rows go to the light tiles (measured on
-    // rmat23: symbolic 329 -> 275 ms).  Explicitly set options are kept as given.
+    // Default thresholds depend on the column count: a bitmap row spans ceil(N / 2^20) column
+    // tiles and its per-row cost multiplies with them.  With more than 4 tiles more rows go to the
+    // light tiles (tools/sweep.py, profiles/r01_threshold_sweep_configs.jsonl: rmat23, 8 tiles,
+    // 28.3 -> 31.5 GFLOP/s; at 2-4 tiles (ab2m, citpatents) 2048/2048 stays best).  Explicitly
+    // set options are kept as given.
     int light_max = h->light_max, tile_cap = h->tile_cap;
-    if (!h->thresholds_set && B->ncols > (1 << 20)) {
+    if (!h->thresholds_set && B->ncols > (1 << 22)) {
       light_max = TILE_PMAX - 1024;
       tile_cap = 1024;
     }

@@ -29,8 +29,8 @@ constexpr uint8_t CLS_LIGHT_PATH = 8;
 constexpr int TINY_MAX = 32;          // class boundaries for statistics only (same kernel)
 constexpr int LIGHTC_MAX = 256;
 constexpr int TILE_PMAX = 4096;       // products per tile: tile capacity + light threshold <= this
-constexpr int TILE_CAP_DEFAULT = 2048;
-constexpr int LIGHT_MAX_DEFAULT = 2048;
+constexpr int TILE_CAP_DEFAULT = 3072;
+constexpr int LIGHT_MAX_DEFAULT = 1024;
 constexpr int TILE_NT = 512;          // threads per tile block
 constexpr int TILE_RM = 512;          // light rows per batch
 #ifndef SPG_TILE_BK

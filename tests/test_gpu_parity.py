@@ -200,7 +200,7 @@ def test_error_paths():
     with pytest.raises(spg.SpgError, match="INVALID_ARGUMENT"):
         plan.set_option("force_class", 1)
     with pytest.raises(spg.SpgError, match="INVALID_ARGUMENT"):
-        plan.set_option("light_max_flops", 3000)  # + tile_flops 2048 > 4096
+        plan.set_option("light_max_flops", 3000)  # + tile_flops 3072 > 4096
     # validation: unsorted B rows and out-of-range columns are reported, not executed
     plan.set_option("validate", 1)
     Bu = W.random_csr(8, 8, 0.5, 3)

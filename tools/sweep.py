@@ -22,6 +22,8 @@ import workloads as W  # noqa: E402
 
 def time_plan(dA, dB, steps, **opts):
     h = spg.spg_create(0, None, dA.vals.dtype)
+    if "tile_flops" in opts and "light_max_flops" in opts:
+        spg.spg_set_option(h, "light_max_flops", 0)  # light + tile <= TILE_PMAX after every call
     for k, v in opts.items():
         spg.spg_set_option(h, k, v)
     rp = torch.empty(dA.nrows + 1, dtype=torch.int64, device="cuda")

@@ -95,7 +95,8 @@ typedef enum {
 } spg_row_class;
 
 typedef enum {
-  SPG_OPT_LIGHT_MAX_FLOPS = 0,  /* heavy/light threshold t: 0..4096-TILE_FLOPS,
+  SPG_OPT_LIGHT_MAX_FLOPS = 0,  /* heavy/light threshold t: 0..4096; light rows
+                                   above 4096 - TILE_FLOPS are tiles of their own;
                                    default 1024 with tile 3072 (tools/sweep.py, profiles/); when
                                    B has > 2^22 columns and neither option was set: 3072 with
                                    tile 1024.  0 sends every non-SINGLE row to the heavy path  */

@@ -180,8 +180,11 @@ __global__ void __launch_bounds__(CL_NT) k_classify(const int* __restrict__ f, c
 }
 
 // Tiles of light rows.  PL = exclusive prefix of fl (light products, row order).  A light row
-// starts a tile when its product range [PL_i, PL_i + f_i) contains a multiple of `cap` (so a
-// tile holds < cap + light_max products).  Light rows get Ro = F_H + PL_i: the plan holds the heavy
+// starts a tile when its product range [PL_i, PL_i + f_i) contains a multiple of `cap`, so a tile
+// of rows with f <= TILE_PMAX - cap holds < TILE_PMAX products; a row with more (up to light_max
+// <= TILE_PMAX) is a solo tile: it starts a tile, and so does the next light row (found by a
+// short look-back; if none within 64 rows the row starts a tile anyway — an extra tile start is
+// always safe).  Light rows get Ro = F_H + PL_i: the plan holds the heavy
 // rows first (their offsets come from k_classify alone, so the heavy kernels start before this).
 // r_ok = (F_L + F_H <= capacity of R): the symbolic kernels do nothing when R is too small and
 // the host re-runs them after growing R.
@@ -207,7 +210,15 @@ __global__ void __launch_bounds__(256) k_tiles(const int* __restrict__ f, int rb
         const long long pl = PL[li];
         const long long fi = f[rb + li];
         Ro[li] = HT + pl;
-        start = (pl % cap == 0) || (pl / cap != (pl + fi - 1) / cap);
+        start = (pl % cap == 0) || (pl / cap != (pl + fi - 1) / cap) || fi > TILE_PMAX - cap;
+        if (!start) {  // the row after a solo row starts a tile (no light row within 64: start anyway)
+          start = true;
+          for (long long j = li - 1; j >= 0 && j >= li - 64; --j)
+            if (cls[j] & CLS_LIGHT_PATH) {
+              start = f[rb + j] > TILE_PMAX - cap;
+              break;
+            }
+        }
       }
       tflag[li] = start ? 1 : 0;
     }

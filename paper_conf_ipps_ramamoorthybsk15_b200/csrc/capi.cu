@@ -674,14 +674,14 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
   if (!h) return SPG_ERR_INVALID_ARGUMENT;
   switch (opt) {
     case SPG_OPT_LIGHT_MAX_FLOPS:
-      if (v < 0 || v + h->tile_cap > TILE_PMAX)
-        return setf(h, SPG_ERR_INVALID_ARGUMENT, "LIGHT_MAX_FLOPS must be in [0, %d - TILE_FLOPS]", TILE_PMAX);
+      if (v < 0 || v > TILE_PMAX)
+        return setf(h, SPG_ERR_INVALID_ARGUMENT, "LIGHT_MAX_FLOPS must be in [0, %d]", TILE_PMAX);
       h->light_max = (int)v;
       h->thresholds_set = 1;
       break;
     case SPG_OPT_TILE_FLOPS:
-      if (v < 1 || v + h->light_max > TILE_PMAX)
-        return setf(h, SPG_ERR_INVALID_ARGUMENT, "TILE_FLOPS must be in [1, %d - LIGHT_MAX_FLOPS]", TILE_PMAX);
+      if (v < 1 || v > TILE_PMAX)
+        return setf(h, SPG_ERR_INVALID_ARGUMENT, "TILE_FLOPS must be in [1, %d]", TILE_PMAX);
       h->tile_cap = (int)v;
       h->thresholds_set = 1;
       break;

@@ -21,7 +21,7 @@ namespace spg {
 struct ClassParams {
   int light_max;   // f <= light_max -> light (tile) kernel
   int heavy_max;   // f <= heavy_max -> register-cached bitmap kernel, else HUGE (uncached)
-  int tile_cap;    // nominal products per tile (light_max + tile_cap <= TILE_PMAX)
+  int tile_cap;    // nominal products per tile; rows above TILE_PMAX - tile_cap are solo tiles
   int force;       // -1 or a class id >= CLS_TINY
   int single_ok;   // B rows canonical -> SINGLE (identity) shortcut allowed
   int warp_max;    // light rows with f <= warp_max -> warp-per-row kernel (0: none)

@@ -69,13 +69,14 @@ def test_power_law_rows_span_all_classes(force):
 
 @pytest.mark.parametrize("heavy_max,tile,light_max", [(64, 64, 40), (256, 128, 64), (8192, 2048, 1024),
                                                       (8192, 2048, 2048), (0, 1, 0), (4096, 16, 4000),
-                                                      (33, 4000, 32)])
+                                                      (33, 4000, 32), (8192, 3072, 4096), (8192, 1024, 4096),
+                                                      (8192, 4096, 4096)])
 def test_thresholds_do_not_change_result(heavy_max, tile, light_max):
     """the threshold moves work between kernels, never changes C (tile 1: a tile
     per light row; light_max 0: every row on the heavy path; heavy_max 0: every heavy row HUGE)."""
     A, B = W.make("cl10k")
     ref = oracle.spgemm(A, B, nthreads=8)
-    # ordered: light_max + tile_flops <= 4096 (TILE_PMAX) must hold after every call
+    # light rows above 4096 - tile are solo tiles; light_max <= 4096 (TILE_PMAX)
     got = run_gpu(A, B, light_max_flops=0, tile_flops=tile, heavy_max_flops=heavy_max, _then={"light_max_flops": light_max})
     compare(A, B, got, ref=ref)
 
@@ -200,7 +201,7 @@ def test_error_paths():
     with pytest.raises(spg.SpgError, match="INVALID_ARGUMENT"):
         plan.set_option("force_class", 1)
     with pytest.raises(spg.SpgError, match="INVALID_ARGUMENT"):
-        plan.set_option("light_max_flops", 3000)  # + tile_flops 3072 > 4096
+        plan.set_option("light_max_flops", 5000)  # > TILE_PMAX (4096)
     # validation: unsorted B rows and out-of-range columns are reported, not executed
     plan.set_option("validate", 1)
     Bu = W.random_csr(8, 8, 0.5, 3)

@@ -433,6 +433,7 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm,
                        h->cls.as<uint8_t>(), h->fl.as<int>(), h->Ro.as<long long>(), L3, ds, crow));
     CK(cudaMemsetAsync(ds->qhead, 0, sizeof(ds->qhead) + sizeof(ds->fb), h->stream));
+    if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));  // analysis = row flops + classify
     if ((s = run_heavy(h, A, B, crow)) != SPG_OK) return s;
     CK(launch_incl_scan<int>(h->stream, h->fl.as<int>(), PL + 1, Mloc, h->scan_tmp.as<long long>()));
     long long r_cap = h->EQ.p && h->fl8.p ? (long long)(h->EQ.cap / sizeof(int2)) : 0;
@@ -440,7 +441,6 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(launch_tiles(h->stream, h->sms, h->f.as<int>(), h->rb, h->re, tile_cap, h->cls.as<uint8_t>(), PL,
                     h->Ro.as<long long>(), h->tflag.as<uint8_t>(), h->tiles.as<int>(), ds, r_cap));
     h->launches += (Mloc > 0) + scan_launches(Mloc) + 1;
-    if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));
     if ((s = run_light(h, A, B, crow)) != SPG_OK) return s;
     CK(launch_incl_scan<long long>(h->stream, crow + 1, crow + 1, Mloc, h->scan_tmp.as<long long>()));
     // numeric plan: per-row EQ-to-C offsets and chunk -> row (capacity from the last call; a

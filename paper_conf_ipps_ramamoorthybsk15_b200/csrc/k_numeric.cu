@@ -20,6 +20,9 @@
 // HBM traffic per output: 8 B of EQ read + 12 B (fp64) of C written; A and B mostly from L2.
 #include "kernels.cuh"
 
+#ifndef SPG_NUM_MINB
+#define SPG_NUM_MINB 5  // k_numeric blocks per SM the register budget is cut for
+#endif
 #ifndef SPG_EQ_LOAD
 #define SPG_EQ_LOAD 0  // plan loads: 0 streaming (ld.global.cs), 1 read-only path, 2 plain
 #endif
@@ -108,7 +111,7 @@ __global__ void __launch_bounds__(256) k_pack_b(const int* __restrict__ colB, co
 }
 
 template <typename V, bool PACK>
-__global__ void __launch_bounds__(NUM_NT, 5) k_numeric(NumProb<V> P) {
+__global__ void __launch_bounds__(NUM_NT, SPG_NUM_MINB) k_numeric(NumProb<V> P) {
   __shared__ __align__(16) int s_head[NUM_CH];   // slot -> 1 + slot of its row's first output in the chunk
   __shared__ long long s_nd[NUM_CH];             // head slot -> nd of its row
   __shared__ int s_ne[NUM_CH];                   // head slot -> ne of its row

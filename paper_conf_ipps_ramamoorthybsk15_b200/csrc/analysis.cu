@@ -119,11 +119,15 @@ __global__ void __launch_bounds__(CL_NT) k_classify(const int* __restrict__ f, c
                                                     int re, ClassParams prm, uint8_t* __restrict__ cls,
                                                     int* __restrict__ fl, long long* __restrict__ Ro,
                                                     HeavyLists lists, Small* __restrict__ sm,
-                                                    long long* __restrict__ crow) {
+                                                    long long* __restrict__ crow, long long* __restrict__ PL) {
   __shared__ unsigned s_rows[NUM_CLS], s_flo[NUM_CLS], s_fhi[NUM_CLS], s_fmax;
   const int tid = threadIdx.x, lane = tid & 31;
   if (tid < NUM_CLS) { s_rows[tid] = 0; s_flo[tid] = 0; s_fhi[tid] = 0; }
   if (tid == 0) s_fmax = 0;
+  if (blockIdx.x == 0 && tid == 0) {
+    crow[0] = 0;
+    PL[0] = 0;
+  }
   __syncthreads();
   const long long n = (long long)re - rb;
   const long long nup = (n + 31) & ~31LL;  // warp-uniform trip count
@@ -376,12 +380,16 @@ cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* 
 
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
                             const ClassParams& prm, uint8_t* cls, int* fl, long long* Ro, const HeavyLists& lists,
-                            Small* small, long long* crow) {
+                            Small* small, long long* crow, long long* PL) {
   const long long n = (long long)re - rb;
-  if (n <= 0) return cudaSuccess;
+  if (n <= 0) {
+    cudaError_t e = cudaMemsetAsync(crow, 0, sizeof(long long), st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(PL, 0, sizeof(long long), st);
+    return e;
+  }
   long long blocks = (n + CL_NT - 1) / CL_NT;
   if (blocks > (long long)sms * 8) blocks = (long long)sms * 8;
-  k_classify<<<(int)blocks, CL_NT, 0, st>>>(f, nz, rb, re, prm, cls, fl, Ro, lists, small, crow);
+  k_classify<<<(int)blocks, CL_NT, 0, st>>>(f, nz, rb, re, prm, cls, fl, Ro, lists, small, crow, PL);
   return cudaGetLastError();
 }
 

@@ -428,11 +428,9 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     HeavyLists L3;
     for (int b = 0; b < NUM_LISTS; ++b) L3.rows[b] = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
     long long* PL = h->PL.as<long long>();
-    CK(cudaMemsetAsync(crow, 0, sizeof(long long), h->stream));
-    CK(cudaMemsetAsync(PL, 0, sizeof(long long), h->stream));
+    // (also zeroes crow[0] and PL[0]; the queue heads were zeroed with Small in analysis())
     CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm,
-                       h->cls.as<uint8_t>(), h->fl.as<int>(), h->Ro.as<long long>(), L3, ds, crow));
-    CK(cudaMemsetAsync(ds->qhead, 0, sizeof(ds->qhead) + sizeof(ds->fb), h->stream));
+                       h->cls.as<uint8_t>(), h->fl.as<int>(), h->Ro.as<long long>(), L3, ds, crow, PL));
     if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));  // analysis = row flops + classify
     if ((s = run_heavy(h, A, B, crow)) != SPG_OK) return s;
     CK(launch_incl_scan<int>(h->stream, h->fl.as<int>(), PL + 1, Mloc, h->scan_tmp.as<long long>()));

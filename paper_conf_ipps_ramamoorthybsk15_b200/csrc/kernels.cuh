@@ -123,7 +123,7 @@ cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* 
                              uint8_t* nz, unsigned long long* hist, int* err, int* amax);
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
                             const ClassParams& prm, uint8_t* cls, int* fl, long long* Ro, const HeavyLists& lists,
-                            Small* small, long long* crow);
+                            Small* small, long long* crow, long long* PL);
 cudaError_t launch_tiles(cudaStream_t st, int sms, const int* f, int rb, int re, int tile_cap, const uint8_t* cls,
                          const long long* PL, long long* Ro, uint8_t* tflag, int* tiles, Small* small,
                          long long r_cap);

@@ -25,6 +25,9 @@ namespace spg {
 constexpr int BMP_CTCAP = 2048;      // 32-product windows per chunk with a precomputed run index
 constexpr int BMP_SLOTS = 8;         // products per lane cached in registers
 constexpr int MODE_CACHED = 0, MODE_PLAIN = 1;
+#ifndef SPG_BMP_SPAN
+#define SPG_BMP_SPAN 0  // 1: cached rows tile their own column span (measured: no gain, r01)
+#endif
 
 __host__ __device__ constexpr int al16(int x) { return (x + 15) & ~15; }
 
@@ -100,8 +103,9 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
     unsigned short* sbq = reinterpret_cast<unsigned short*>(sbp + nl1);   // .. / 256 columns (4 per 1024)
     unsigned* flags = reinterpret_cast<unsigned*>(sbq + 4 * nl1);
     const int nfw = CACHED ? (f + 31) >> 5 : 0;
-    const int ntiles = (int)(((long long)N + Wt - 1) >> lw);
+    int ntiles = (int)(((long long)N + Wt - 1) >> lw);
     const int nchunks = (pa1 - pa0 + RCAP - 1) / RCAP;
+    int lo0 = 0;  // first column of tile 0
     int out = 0;
     int nz = 0, Lt = 0;  // current chunk: runs, products
     int cc[BMP_SLOTS];   // cached mode: this lane's product columns
@@ -200,13 +204,35 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
       return r;
     };
 
+#if SPG_BMP_SPAN
+    // Cached rows (one chunk): the tiles cover the row's column span [cmin, cmax] instead of
+    // [0, N) — the columns of a web-graph row are local, so one tile pass usually suffices.
+    const bool pre = CACHED && nchunks == 1;
+    if (pre) {
+      gather(0);
+      fill_cache();
+      int cmin = INT_MAX, cmax = -1;
+#pragma unroll
+      for (int s = 0; s < BMP_SLOTS; ++s)
+        if (cc[s] >= 0) {
+          cmin = min(cmin, cc[s]);
+          cmax = max(cmax, cc[s]);
+        }
+      cmin = -g.max(-cmin);
+      cmax = g.max(cmax);
+      lo0 = cmin & ~31;
+      ntiles = ((cmax - lo0) >> lw) + 1;
+    }
+#else
+    constexpr bool pre = false;
+#endif
     for (int tile = 0; tile < ntiles; ++tile) {
-      const int lo = tile << lw;
+      const int lo = lo0 + (tile << lw);
       // ---- pass 1: claim bits; first claimers flagged -----------------------------------------
       int cbase = 0;
       int npin = 0;  // this thread's products inside the tile
       for (int c = 0; c < nchunks; ++c) {
-        if (nchunks > 1 || tile == 0) {
+        if (nchunks > 1 || (tile == 0 && !pre)) {
           gather(c);
           if constexpr (CACHED) fill_cache();
         }

@@ -110,124 +110,189 @@ __global__ void __launch_bounds__(256) k_pack_b(const int* __restrict__ colB, co
     out[x] = pack_b<V>(colB[x], valB[x]);
 }
 
+#ifndef SPG_NUM_PIPE
+#define SPG_NUM_PIPE 0  // 1: software-pipelined chunks (next chunk's row heads + plan loads overlap the gathers)
+#endif
+
+// Row heads of chunk ch in shared memory: s_head[slot] = 1 + slot of its row's first output.
+// Returns false for a chunk inside one row (nd1/ne1 set; no shared memory, no barrier).
+__device__ __forceinline__ bool num_setup(const long long* __restrict__ crow, const long long* __restrict__ ndv,
+                                          const int* __restrict__ nev, const int* __restrict__ chunk_row, int nch,
+                                          int mloc, int ch, long long base, int* s_head, long long* s_nd, int* s_ne,
+                                          int* s_wmax, long long& nd1, int& ne1) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int r0 = chunk_row[ch];
+  const int r1 = ch + 1 < nch ? chunk_row[ch + 1] : mloc - 1;
+  if (r0 == r1) {
+    nd1 = ndv[r0];
+    ne1 = nev[r0];
+    return false;
+  }
+  {
+    int4* h4 = reinterpret_cast<int4*>(s_head);
+    h4[2 * tid] = make_int4(0, 0, 0, 0);
+    h4[2 * tid + 1] = make_int4(0, 0, 0, 0);
+  }
+  __syncthreads();
+  if (tid == 0) {
+    s_head[0] = 1;
+    s_nd[0] = ndv[r0];
+    s_ne[0] = nev[r0];
+  }
+  // rows starting inside the chunk (every row is visited by exactly one chunk: O(M) in total)
+  for (int r = r0 + 1 + tid; r <= r1; r += NUM_NT) {
+    const long long a = crow[r], b = crow[r + 1];
+    const long long s = a - base;
+    if (b > a && s < NUM_CH) {
+      s_head[s] = (int)s + 1;
+      s_nd[s] = ndv[r];
+      s_ne[s] = nev[r];
+    }
+  }
+  __syncthreads();
+  // fill forward: slot -> its row's head slot (max scan over 8 slots per thread, then warps)
+  int4* h4 = reinterpret_cast<int4*>(s_head);
+  int4 x = h4[2 * tid], y = h4[2 * tid + 1];
+  x.y = max(x.y, x.x); x.z = max(x.z, x.y); x.w = max(x.w, x.z);
+  y.x = max(y.x, x.w); y.y = max(y.y, y.x); y.z = max(y.z, y.y); y.w = max(y.w, y.z);
+  int m = y.w;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const int o = __shfl_up_sync(FULL, m, d);
+    if (lane >= d) m = max(m, o);
+  }
+  if (lane == 31) s_wmax[warp] = m;
+  int carry = __shfl_up_sync(FULL, m, 1);
+  if (lane == 0) carry = 0;
+  __syncthreads();
+  for (int w = 0; w < warp; ++w) carry = max(carry, s_wmax[w]);
+  x.x = max(x.x, carry); x.y = max(x.y, carry); x.z = max(x.z, carry); x.w = max(x.w, carry);
+  y.x = max(y.x, carry); y.y = max(y.y, carry); y.z = max(y.z, carry); y.w = max(y.w, carry);
+  h4[2 * tid] = x;
+  h4[2 * tid + 1] = y;
+  __syncthreads();
+  return true;
+}
+
+// Plan loads of the chunk: output slot s = k·NUM_NT + tid gets {A entry e, B entry q}; e = -1 past
+// the chunk's end.
+__device__ __forceinline__ void num_plan_loads(const int2* __restrict__ EQ, long long base, int n, bool one,
+                                               long long nd1, int ne1, const int* s_head, const long long* s_nd,
+                                               const int* s_ne, int* e, int* q) {
+  const int tid = threadIdx.x;
+#pragma unroll
+  for (int k = 0; k < NUM_PT; ++k) {
+    const int s = k * NUM_NT + tid;
+    const bool ok = s < n;
+    long long d = nd1;
+    int es = ne1;
+    if (!one) {
+      const int h = ok ? s_head[s] - 1 : 0;
+      d = s_nd[h];
+      es = s_ne[h];
+    }
+    const long long src = base + s + d;
+    const bool plan = ok && es < 0;
+#if SPG_EQ_LOAD == 1
+    const int2 eq = plan ? __ldg(EQ + src) : make_int2(es, (int)src);
+#elif SPG_EQ_LOAD == 2
+    const int2 eq = plan ? EQ[src] : make_int2(es, (int)src);
+#else
+    const int2 eq = plan ? __ldcs(EQ + src) : make_int2(es, (int)src);
+#endif
+    e[k] = ok ? eq.x : -1;
+    q[k] = eq.y;
+  }
+}
+
+template <typename V, bool PACK>
+__device__ __forceinline__ void num_gathers(const NumProb<V>& P, const int* e, const int* q, int* col, V* va, V* vb) {
+#pragma unroll
+  for (int k = 0; k < NUM_PT; ++k) {
+    const bool ok = e[k] >= 0;
+    if constexpr (PACK) {
+      using T = typename PackB<V>::T;
+      const T t = ok ? __ldg(reinterpret_cast<const T*>(P.packB) + q[k]) : T{};
+      col[k] = t.x;
+      vb[k] = unpack_v(t, V(0));
+    } else {
+      col[k] = ok ? __ldg(P.colB + q[k]) : 0;
+      vb[k] = ok ? __ldg(P.valB + q[k]) : V(0);
+    }
+    va[k] = ok ? __ldg(P.valA + e[k]) : V(0);
+  }
+}
+
+template <typename V>
+__device__ __forceinline__ void num_stores(const NumProb<V>& P, long long base, int n, const int* col, const V* va,
+                                           const V* vb) {
+  const int tid = threadIdx.x;
+#pragma unroll
+  for (int k = 0; k < NUM_PT; ++k) {
+    const int s = k * NUM_NT + tid;
+    if (s < n) {
+      __stcs(P.ccol + base + s, col[k]);
+      __stcs(P.cval + base + s, va[k] * vb[k]);
+    }
+  }
+}
+
 template <typename V, bool PACK>
 __global__ void __launch_bounds__(NUM_NT, SPG_NUM_MINB) k_numeric(NumProb<V> P) {
   __shared__ __align__(16) int s_head[NUM_CH];   // slot -> 1 + slot of its row's first output in the chunk
   __shared__ long long s_nd[NUM_CH];             // head slot -> nd of its row
   __shared__ int s_ne[NUM_CH];                   // head slot -> ne of its row
   __shared__ int s_wmax[NUM_NT / 32];
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  for (int ch = blockIdx.x; ch < P.nch; ch += gridDim.x) {
-    const long long base = (long long)ch * NUM_CH;
-    const int n = (int)min((long long)NUM_CH, P.nnz - base);
-    const int r0 = P.chunk_row[ch];
-    const int r1 = ch + 1 < P.nch ? P.chunk_row[ch + 1] : P.mloc - 1;
-    // a chunk inside one row (half of webbase1m's chunks: heavy rows) needs no row heads, no
-    // shared memory and no barrier
-    const bool one = r0 == r1;
+  auto chunk_n = [&](int ch) { return (int)min((long long)NUM_CH, P.nnz - (long long)ch * NUM_CH); };
+#if SPG_NUM_PIPE
+  // Software pipeline over this block's chunks: the gathers of chunk ch are in flight while the
+  // row heads and plan loads of the next chunk are computed; the stores of ch come last.
+  int ch = blockIdx.x;
+  if (ch >= P.nch) return;
+  int e[NUM_PT], q[NUM_PT];
+  {
     long long nd1 = 0;
     int ne1 = 0;
-    if (one) {
-      nd1 = P.nd[r0];
-      ne1 = P.ne[r0];
-    } else {
-    {
-      int4* h4 = reinterpret_cast<int4*>(s_head);
-      h4[2 * tid] = make_int4(0, 0, 0, 0);
-      h4[2 * tid + 1] = make_int4(0, 0, 0, 0);
-    }
-    __syncthreads();
-    if (tid == 0) {
-      s_head[0] = 1;
-      s_nd[0] = P.nd[r0];
-      s_ne[0] = P.ne[r0];
-    }
-    // rows starting inside the chunk (every row is visited by exactly one chunk: O(M) in total)
-    for (int r = r0 + 1 + tid; r <= r1; r += NUM_NT) {
-      const long long a = P.crow[r], b = P.crow[r + 1];
-      const long long s = a - base;
-      if (b > a && s < NUM_CH) {
-        s_head[s] = (int)s + 1;
-        s_nd[s] = P.nd[r];
-        s_ne[s] = P.ne[r];
-      }
-    }
-    __syncthreads();
-    // fill forward: slot -> its row's head slot (max scan over 8 slots per thread, then warps)
-    {
-      int4* h4 = reinterpret_cast<int4*>(s_head);
-      int4 x = h4[2 * tid], y = h4[2 * tid + 1];
-      x.y = max(x.y, x.x); x.z = max(x.z, x.y); x.w = max(x.w, x.z);
-      y.x = max(y.x, x.w); y.y = max(y.y, y.x); y.z = max(y.z, y.y); y.w = max(y.w, y.z);
-      int m = y.w;
-#pragma unroll
-      for (int d = 1; d < 32; d <<= 1) {
-        const int o = __shfl_up_sync(FULL, m, d);
-        if (lane >= d) m = max(m, o);
-      }
-      if (lane == 31) s_wmax[warp] = m;
-      int carry = __shfl_up_sync(FULL, m, 1);
-      if (lane == 0) carry = 0;
-      __syncthreads();
-      for (int w = 0; w < warp; ++w) carry = max(carry, s_wmax[w]);
-      x.x = max(x.x, carry); x.y = max(x.y, carry); x.z = max(x.z, carry); x.w = max(x.w, carry);
-      y.x = max(y.x, carry); y.y = max(y.y, carry); y.z = max(y.z, carry); y.w = max(y.w, carry);
-      h4[2 * tid] = x;
-      h4[2 * tid + 1] = y;
-    }
-    __syncthreads();
-    }
-    // outputs o = base + k·NUM_NT + tid: plan loads, then gathers, then stores (all batched)
-    int e[NUM_PT], q[NUM_PT];
-#pragma unroll
-    for (int k = 0; k < NUM_PT; ++k) {
-      const int s = k * NUM_NT + tid;
-      const bool ok = s < n;
-      long long d = nd1;
-      int es = ne1;
-      if (!one) {
-        const int h = ok ? s_head[s] - 1 : 0;
-        d = s_nd[h];
-        es = s_ne[h];
-      }
-      const long long src = base + s + d;
-      const bool plan = ok && es < 0;
-#if SPG_EQ_LOAD == 1
-      const int2 eq = plan ? __ldg(P.EQ + src) : make_int2(es, (int)src);
-#elif SPG_EQ_LOAD == 2
-      const int2 eq = plan ? P.EQ[src] : make_int2(es, (int)src);
-#else
-      const int2 eq = plan ? __ldcs(P.EQ + src) : make_int2(es, (int)src);
-#endif
-      e[k] = ok ? eq.x : -1;
-      q[k] = eq.y;
-    }
+    const long long base = (long long)ch * NUM_CH;
+    const bool multi = num_setup(P.crow, P.nd, P.ne, P.chunk_row, P.nch, P.mloc, ch, base, s_head, s_nd, s_ne,
+                                 s_wmax, nd1, ne1);
+    num_plan_loads(P.EQ, base, chunk_n(ch), !multi, nd1, ne1, s_head, s_nd, s_ne, e, q);
+  }
+  for (; ch < P.nch; ch += gridDim.x) {
     int col[NUM_PT];
     V va[NUM_PT], vb[NUM_PT];
-#pragma unroll
-    for (int k = 0; k < NUM_PT; ++k) {
-      const bool ok = e[k] >= 0;
-      if constexpr (PACK) {
-        using T = typename PackB<V>::T;
-        const T t = ok ? __ldg(reinterpret_cast<const T*>(P.packB) + q[k]) : T{};
-        col[k] = t.x;
-        vb[k] = unpack_v(t, V(0));
-      } else {
-        col[k] = ok ? __ldg(P.colB + q[k]) : 0;
-        vb[k] = ok ? __ldg(P.valB + q[k]) : V(0);
-      }
-      va[k] = ok ? __ldg(P.valA + e[k]) : V(0);
+    num_gathers<V, PACK>(P, e, q, col, va, vb);
+    const int nx = ch + gridDim.x;
+    if (nx < P.nch) {
+      __syncthreads();  // every thread's plan loads of ch read s_head before it is rebuilt
+      long long nd1 = 0;
+      int ne1 = 0;
+      const long long base = (long long)nx * NUM_CH;
+      const bool multi = num_setup(P.crow, P.nd, P.ne, P.chunk_row, P.nch, P.mloc, nx, base, s_head, s_nd, s_ne,
+                                   s_wmax, nd1, ne1);
+      num_plan_loads(P.EQ, base, chunk_n(nx), !multi, nd1, ne1, s_head, s_nd, s_ne, e, q);
     }
-#pragma unroll
-    for (int k = 0; k < NUM_PT; ++k) {
-      const int s = k * NUM_NT + tid;
-      if (s < n) {
-        __stcs(P.ccol + base + s, col[k]);
-        __stcs(P.cval + base + s, va[k] * vb[k]);
-      }
-    }
-    if (!one) __syncthreads();
+    num_stores<V>(P, (long long)ch * NUM_CH, chunk_n(ch), col, va, vb);
   }
+#else
+  for (int ch = blockIdx.x; ch < P.nch; ch += gridDim.x) {
+    const long long base = (long long)ch * NUM_CH;
+    long long nd1 = 0;
+    int ne1 = 0;
+    // a chunk inside one row (half of webbase1m's chunks: heavy rows) needs no row heads, no
+    // shared memory and no barrier
+    const bool multi = num_setup(P.crow, P.nd, P.ne, P.chunk_row, P.nch, P.mloc, ch, base, s_head, s_nd, s_ne,
+                                 s_wmax, nd1, ne1);
+    // outputs o = base + k·NUM_NT + tid: plan loads, then gathers, then stores (all batched)
+    int e[NUM_PT], q[NUM_PT];
+    num_plan_loads(P.EQ, base, chunk_n(ch), !multi, nd1, ne1, s_head, s_nd, s_ne, e, q);
+    int col[NUM_PT];
+    V va[NUM_PT], vb[NUM_PT];
+    num_gathers<V, PACK>(P, e, q, col, va, vb);
+    num_stores<V>(P, base, chunk_n(ch), col, va, vb);
+    if (multi) __syncthreads();
+  }
+#endif
 }
 
 template <typename V>

@@ -80,8 +80,10 @@ struct spg_ctx {
   int light_max = LIGHT_MAX_DEFAULT, tile_cap = TILE_CAP_DEFAULT, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
   // numeric: gather B through a packed {column, value} copy — one sector per gather instead of
-  // two when B does not stay in L2 (auto: B's columns + values > 64 MB; SPG_PACK_B=0/1 forces)
+  // two when B does not stay in L2 (auto: B's columns + values > 64 MB; SPG_PACK_B=0/1 forces;
+  // always-on measured neutral on the L2-resident configs)
   int pack_b = -1;
+  int l2_persist = 0;  // experimental: 1 persisting-L2 window over B during numeric (reset after), 2 without the reset
   int thresholds_set = 0;
   int warp_max = WARP_MAX_DEFAULT;  // light rows with f <= warp_max: one warp per row (k_warp.cu)
   int occ_warp = 1;  // light_max / tile_cap set by the caller (else N-dependent defaults)
@@ -557,8 +559,33 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
     P.cval = (V*)C_val;
     int grid = h->occ_num * h->sms;
     if (h->nch < grid) grid = h->nch;
+    // Experimental (SPG_L2_PERSIST=1): keep the gathered B (packed copy, else B's values) in
+    // the persisting part of L2 while the streaming plan reads and C stores pass through.
+    const void* win = P.packB ? (const void*)P.packB : (const void*)P.valB;
+    const size_t win_bytes = P.packB ? (size_t)B->nnz * (sizeof(V) == 8 ? 16 : 8) : (size_t)B->nnz * sizeof(V);
+    const bool persist = h->l2_persist > 0 && win_bytes > 0;
+    if (persist) {
+      int dev = 0, maxp = 0, maxw = 0;
+      CK(cudaGetDevice(&dev));
+      CK(cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev));
+      CK(cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev));
+      CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp));
+      cudaStreamAttrValue a = {};
+      a.accessPolicyWindow.base_ptr = const_cast<void*>(win);
+      a.accessPolicyWindow.num_bytes = win_bytes < (size_t)maxw ? win_bytes : (size_t)maxw;
+      a.accessPolicyWindow.hitRatio = win_bytes <= (size_t)maxp ? 1.0f : (float)maxp / (float)win_bytes;
+      a.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+      a.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+      CK(cudaStreamSetAttribute(h->stream, cudaStreamAttributeAccessPolicyWindow, &a));
+    }
     CK(launch_numeric<V>(h->stream, grid, P));
     h->launches += (h->nch > 0) + (h->ndup > 0) + (P.packB != nullptr);
+    if (persist) {
+      cudaStreamAttrValue a = {};
+      a.accessPolicyWindow.num_bytes = 0;
+      CK(cudaStreamSetAttribute(h->stream, cudaStreamAttributeAccessPolicyWindow, &a));
+      if (h->l2_persist == 1) CK(cudaCtxResetPersistingL2Cache());
+    }
   }
   h->stats.launches_numeric = h->launches;
   if (h->timing) {
@@ -613,6 +640,7 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
   h->occ_light = light_occupancy();
   h->occ_num = dtype == SPG_FP64 ? numeric_occupancy<double>() : numeric_occupancy<float>();
   if (const char* pb = getenv("SPG_PACK_B")) h->pack_b = atoi(pb);
+  if (const char* lp = getenv("SPG_L2_PERSIST")) h->l2_persist = atoi(lp);
   for (int b = 0; b < NUM_BINS; ++b) h->occ_heavy[b] = heavy_occupancy(b);
   h->occ_warp = warp_occupancy();
   cudaGetLastError();

@@ -110,6 +110,9 @@ __global__ void __launch_bounds__(256) k_pack_b(const int* __restrict__ colB, co
     out[x] = pack_b<V>(colB[x], valB[x]);
 }
 
+#ifndef SPG_C_STORE
+#define SPG_C_STORE 0  // C stores: 0 streaming (st.global.cs), 1 plain
+#endif
 #ifndef SPG_NUM_PIPE
 #define SPG_NUM_PIPE 0  // 1: software-pipelined chunks (next chunk's row heads + plan loads overlap the gathers)
 #endif
@@ -231,8 +234,13 @@ __device__ __forceinline__ void num_stores(const NumProb<V>& P, long long base, 
   for (int k = 0; k < NUM_PT; ++k) {
     const int s = k * NUM_NT + tid;
     if (s < n) {
+#if SPG_C_STORE == 1
+      P.ccol[base + s] = col[k];
+      P.cval[base + s] = va[k] * vb[k];
+#else
       __stcs(P.ccol + base + s, col[k]);
       __stcs(P.cval + base + s, va[k] * vb[k]);
+#endif
     }
   }
 }

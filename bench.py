@@ -298,7 +298,7 @@ def run_ours(args):
     # phase's output (the gather plan: EQ entries of non-SINGLE outputs + the dup list)
     abc_bytes = (csr_bytes(re - rb, nnzA_loc, vb) + csr_bytes(B.nrows, B.nnz, vb)
                  + csr_bytes(re - rb, nnz, vb, rp_bytes=8))
-    plan_bytes = int(st["rank_bytes"])
+    plan_bytes = int(st["plan_bytes"])
     alg_bytes = abc_bytes + plan_bytes
     num_ms = float(np.mean(num))
     peak, peak_src = load_peaks()
@@ -372,8 +372,8 @@ def run_ours(args):
             "phases": {"symbolic_ms": float(np.mean(sym)), "numeric_ms": num_ms,
                        "numeric_gflops": 2.0 * int(st["flops"]) / (num_ms * 1e-3) / 1e9,
                        "symbolic_path_ms": dict(zip(["analysis", "light", "heavy"], (path_ms / K).round(4).tolist())),
-                       "tiles": int(st["tiles"]), "fallback_rows": int(st["fallback_rows"]),
-                       "plan_bytes": int(st["rank_bytes"]),
+                       "tiles": int(st["tiles"]), "heavy_rows": int(st["heavy_rows"]), "dup_products": int(st["dup_products"]),
+                       "plan_bytes": int(st["plan_bytes"]),
                        "class_rows": dict(zip(spg.CLASS_NAMES, stl["class_rows"])),
                        "class_flops": dict(zip(spg.CLASS_NAMES, stl["class_flops"]))},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

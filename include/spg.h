@@ -24,9 +24,10 @@
  *     in which case the library sorts and de-duplicates a copy of B first.
  *
  * Ownership and threading
- *   - The caller owns A, B and C.  The handle owns all workspace (row flops, class lists,
- *     the gather plan — 8 bytes per intermediate product of the non-SINGLE rows plus a
- *     16-byte dup entry per repeated column — and the NCCL communicator) and caches the symbolic analysis that spg_spgemm_numeric consumes.
+ *   - The caller owns A, B and C.  The handle owns all workspace (row flops, classes, the item
+ *     list, the plan — 4 bytes per intermediate product (8 for rows with an A row or a referenced
+ *     B row longer than 65535 entries) plus 1 byte per product of the largest rows — and the NCCL
+ *     communicator) and caches the symbolic analysis that spg_spgemm_numeric consumes.
  *     spg_spgemm_free releases everything.
  *   - A handle is bound to one device and one CUDA stream and is not thread-safe;
  *     several handles may coexist.
@@ -41,6 +42,9 @@
  *     (host-side when the value is known), dtype, call order (SPG_ERR_BAD_STATE), and
  *     per-row flop counts < 2^31 (SPG_ERR_INDEX_OVERFLOW, reported by symbolic).
  *   - Index ranges and ordering of device inputs are checked only under SPG_OPT_VALIDATE.
+ *   - Values are not bitwise reproducible run to run when a row has repeated columns: the
+ *     repeated products are added with atomics in a nondeterministic order (R6).
+ *     Structure (C_row_ptr, C_col_idx) is deterministic.
  */
 #ifndef SPG_H
 #define SPG_H
@@ -81,8 +85,9 @@ typedef struct {
 /* Row classes (PAPER.md L104 logical reordering A = [A_H; A_L]).
  * f_i = number of intermediate products of row i.  The heavy/light threshold t of the paper
  * (Phase I) is SPG_OPT_LIGHT_MAX_FLOPS: rows with f_i <= t are "light"
- * (TINY / LIGHT / MEDIUM, one shared kernel that sorts whole tiles of rows per thread block),
- * the rest "heavy" (one thread block and a shared-memory column bitmap per row). */
+ * (TINY / LIGHT / MEDIUM: tiles of consecutive rows, sorted by one thread block each), the rest
+ * "heavy" (one thread block and a shared-memory column bitmap per row).  SINGLE rows (one
+ * non-empty B row) are copied; they ride in tiles when f_i <= t. */
 typedef enum {
   SPG_CLASS_EMPTY = 0,  /* f_i = 0: no work, c_i = 0                                         */
   SPG_CLASS_SINGLE = 1, /* exactly one non-empty B row referenced: scaled copy, c_i = f_i    */
@@ -110,10 +115,7 @@ typedef enum {
                                    0: the library canonicalises a copy of B                   */
   SPG_OPT_TIMING = 6,           /* 1: record per-phase CUDA-event times into the stats        */
   SPG_OPT_HUGE_SLOTS = 7,       /* max concurrent heavy-row blocks per bin (0 = full occupancy) */
-  SPG_OPT_CONCURRENT = 8,       /* 1 (default): light and heavy kernels on concurrent streams  */
-  SPG_OPT_WARP_MAX_FLOPS = 9    /* 0..256, default 0 (off): light rows with f <= this are sorted
-                                   one warp per row in registers (bitonic network) instead of
-                                   in tiles.  Ignored while FORCE_CLASS is set                */
+  SPG_OPT_CONCURRENT = 8        /* 1 (default): light and heavy kernels on concurrent streams  */
 } spg_option;
 
 typedef struct {
@@ -126,10 +128,11 @@ typedef struct {
   int64_t class_flops[SPG_NUM_CLASSES];   /* products per class (this rank)              */
   int64_t bin_hist[65];                   /* rows with f = 0 (index 0) and with
                                              ceil(log2 f) = b (index b + 1), all rows    */
-  int64_t tiles;                          /* light tiles of the last symbolic call       */
-  int64_t fallback_rows;                  /* light rows moved to the heavy path (clustered
-                                             columns)                                    */
-  int64_t rank_bytes;                     /* bytes of the gather plan (EQ + dup list)    */
+  int64_t tiles;                          /* tiles of the last symbolic call              */
+  int64_t heavy_rows;                     /* rows on the heavy (bitmap) path             */
+  int64_t dup_products;                   /* products adding to an output another product
+                                             created (f - c summed over rows)            */
+  int64_t plan_bytes;                     /* bytes of the plan numeric reads             */
   float ms_analysis;                      /* SPG_OPT_TIMING: row analysis + classify     */
   float ms_symbolic;                      /*   symbolic kernels + row_ptr scan            */
   float ms_numeric;                       /*   numeric (last numeric call)                */
@@ -160,10 +163,12 @@ spg_status spg_spgemm_symbolic(spg_handle h, const spg_csr* A, const spg_csr* B,
                                int64_t* nnzC, int32_t* row_begin, int32_t* row_end);
 
 /* Numeric phase (Phase IV "add like-tuples, compact"): symbolic sorted every
- * row's products and left, for each output of C, the A and B entry of its first product (plus a
- * list of the repeated ones); numeric streams C in output order, C(i,r) = a·b, then adds the
- * repeats — C comes out sorted and compacted.  Requires a preceding symbolic call on this handle
- * with the same A/B structure pointers and the same C_row_ptr contents.  C_col_idx: device int32[nnzC];
+ * row's products and left a plan — for each output of C, in C order, the A entry and B entry of
+ * one of its products, then the repeated products; numeric streams C in output order,
+ * C(i,r) = a·b, then adds the repeats — C comes out sorted and compacted.  Requires a preceding
+ * symbolic call on this handle with the same A/B structure (checked by pointers, shapes and nnz
+ * only: a different structure at recycled addresses is not detected — the caller's contract) and
+ * the same C_row_ptr contents.  C_col_idx: device int32[nnzC];
  * C_vals: device fp32/fp64[nnzC].  Values of A and B may differ from the symbolic call
  * (re-run numeric on new values with the same structure).  Asynchronous. */
 spg_status spg_spgemm_numeric(spg_handle h, const spg_csr* A, const spg_csr* B, const int64_t* C_row_ptr,

@@ -26,7 +26,7 @@ CLASS_NAMES = ["empty", "single", "tiny", "light", "medium", "heavy", "huge"]
 NUM_CLASSES = 7
 # options
 OPTIONS = {"light_max_flops": 0, "tile_flops": 1, "heavy_max_flops": 2, "force_class": 3, "validate": 4,
-           "input_canonical": 5, "timing": 6, "huge_slots": 7, "concurrent": 8, "warp_max_flops": 9}
+           "input_canonical": 5, "timing": 6, "huge_slots": 7, "concurrent": 8}
 
 EXPORTED = ["spg_create", "spg_set_option", "spg_get_option", "spg_spgemm_free", "spg_last_error", "spg_get_stats",
             "spg_version", "spg_spgemm_symbolic", "spg_spgemm_numeric", "spg_spgemm_host_symbolic",
@@ -43,8 +43,8 @@ class spg_stats(ctypes.Structure):
     _fields_ = [("flops", c_int64), ("flops_total", c_int64), ("f_max", c_int64), ("nnz_c", c_int64),
                 ("row_begin", c_int32), ("row_end", c_int32),
                 ("class_rows", c_int64 * NUM_CLASSES), ("class_flops", c_int64 * NUM_CLASSES),
-                ("bin_hist", c_int64 * 65), ("tiles", c_int64), ("fallback_rows", c_int64),
-                ("rank_bytes", c_int64), ("ms_analysis", c_float), ("ms_symbolic", c_float),
+                ("bin_hist", c_int64 * 65), ("tiles", c_int64), ("heavy_rows", c_int64),
+                ("dup_products", c_int64), ("plan_bytes", c_int64), ("ms_analysis", c_float), ("ms_symbolic", c_float),
                 ("ms_numeric", c_float), ("ms_light", c_float), ("ms_heavy", c_float),
                 ("launches_symbolic", c_int32), ("launches_numeric", c_int32)]
 

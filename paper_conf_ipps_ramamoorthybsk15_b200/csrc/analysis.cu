@@ -11,19 +11,21 @@
 
 namespace spg {
 
-// f_i = sum over stored A(i,k) of len_B(k); nz_i = #entries with len_B(k) > 0 (capped at 2, plus
-// bits 6/7 for A rows longer than one 512- / 1024-thread bitmap chunk).  One block owns ROWS
+// f_i = sum over stored A(i,k) of len_B(k); nz_i = #entries with len_B(k) > 0 (capped at 2), plus
+// the NZ_* size flags (A row longer than 512 / 1024 / 65535 entries, a B row longer than 65535).  One block owns ROWS
 // consecutive rows; its threads stride over the rows' A entries (coalesced), find the owning row
 // by binary search in the cached row_ptr tile, pre-reduce per warp and row, and add into shared
 // 32-bit accumulators.
 template <int ROWS>
 __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict__ rpA, const int* __restrict__ colA,
                                                     int K, const int* __restrict__ rpB, int* __restrict__ f_out,
-                                                    uint8_t* __restrict__ nz_out, unsigned long long* __restrict__ hist,
+                                                    uint8_t* __restrict__ nz_out, int* __restrict__ Tb,
+                                                    int* __restrict__ Tl, unsigned long long* __restrict__ hist,
                                                     int* __restrict__ err, int* __restrict__ amax) {
   __shared__ int s_rp[ROWS + 1];
   __shared__ unsigned s_f[ROWS];
   __shared__ int s_nz[ROWS];
+  __shared__ int s_lb[ROWS];
   __shared__ unsigned s_hist[65];
   __shared__ int s_amax;
   const int t = threadIdx.x, lane = t & 31;
@@ -33,6 +35,7 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
   if (t == 0 && nr == ROWS) s_rp[ROWS] = rpA[r0 + ROWS];
   s_f[t] = 0;
   s_nz[t] = 0;
+  s_lb[t] = 0;
   if (t < 65) s_hist[t] = 0;
   if (t == 0) s_amax = 0;
   __syncthreads();
@@ -45,8 +48,12 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
     if (act) {
       const int k = colA[e];
       r = upper_idx(s_rp, nr, e);
+      int bs = 0;
       if ((unsigned)k >= (unsigned)K) bad |= 1;
-      else L = rpB[k + 1] - rpB[k];
+      else { bs = rpB[k]; L = rpB[k + 1] - bs; }
+      Tb[e] = bs;
+      Tl[e] = L;
+      if (L > 65535) atomicOr(&s_lb[r], 1);
     }
     act = r >= 0;
     const unsigned nzb = __ballot_sync(FULL, act && L > 0);
@@ -71,10 +78,12 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
     unsigned f = s_f[t];
     if (f > (unsigned)INT_MAX) f = INT_MAX;
     f_out[r0 + t] = (int)f;
-    // bits 6/7: the A row has more entries than a 512- / 1024-thread bitmap block gathers in one
-    // chunk (register-cached HEAVY kernels need single-chunk rows; longer rows move up)
+    // size flags: the A row has more entries than a 512- / 1024-thread bitmap block gathers in one
+    // chunk (register-cached HEAVY kernels need single-chunk rows; TILE_EC = 1024 bounds tiles),
+    // or than a 16-bit plan field holds; a referenced B row longer than 65535 (16-bit offset)
     const int alen = s_rp[t + 1] - s_rp[t];
-    nz_out[r0 + t] = (uint8_t)(min(s_nz[t], 2) | (alen > BMP_NT_S ? 0x40 : 0) | (alen > BMP_NT ? 0x80 : 0));
+    nz_out[r0 + t] = (uint8_t)(min(s_nz[t], 2) | (alen > BMP_NT_S ? NZ_ALEN512 : 0) | (alen > BMP_NT ? NZ_ALEN1K : 0) |
+                               (alen > 65535 ? NZ_ALEN64K : 0) | (s_lb[t] ? NZ_LONGB : 0));
     const int b = f == 0 ? 0 : 1 + (f == 1 ? 0 : 32 - __clz((int)f - 1));
     atomicAdd(&s_hist[b], 1u);
     atomicMax(&s_amax, alen);
@@ -85,64 +94,63 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
   if (t == 0) atomicMax(amax, s_amax);
 }
 
-// Row path.  Returns the class (CLS_*) and, through `bin`, the bitmap bin (-1: none).
-__device__ __forceinline__ int classify_row(int f, int nz, const ClassParams& p, int& bin, bool& light) {
+// Row path.  Returns the class (CLS_*); heavy: the row is an item of its own on the bitmap path
+// (bin = its bitmap bin), else it belongs to a tile.
+static_assert(TILE_EC == BMP_NT, "NZ_ALEN1K marks rows too long for a tile");
+__device__ __forceinline__ int classify_row(int f, int nz, const ClassParams& p, int& bin, bool& heavy) {
   bin = -1;
-  light = false;
+  heavy = false;
   if (f == 0) return CLS_EMPTY;
-  const bool long1 = nz & 0x40, long2 = nz & 0x80;
-  nz &= 0x3f;
-  if (p.force < 0 && nz == 1 && p.single_ok) return CLS_SINGLE;
-  if (f <= p.light_max && p.force < CLS_HEAVY) {
-    const int c = f <= TINY_MAX ? CLS_TINY : (f <= LIGHTC_MAX ? CLS_LIGHT : CLS_MEDIUM);
-    if (f <= p.warp_max && p.force < 0) bin = BIN_WARP;  // one warp per row (k_warp.cu)
-    else light = true;                                   // light tiles (k_light.cu)
-    return c;
+  const bool long1 = nz & NZ_ALEN512, long2 = nz & NZ_ALEN1K;
+  const int runs = nz & 3;
+  int c;
+  if (p.force < 0 && runs == 1 && p.single_ok) {
+    c = CLS_SINGLE;  // one non-empty B row: c_i = f_i, no sort
+    if (f <= p.light_max && !long2) return c;
+  } else {
+    if (f <= p.light_max && p.force < CLS_HEAVY && !long2)
+      return f <= TINY_MAX ? CLS_TINY : (f <= LIGHTC_MAX ? CLS_LIGHT : CLS_MEDIUM);
+    c = -1;
   }
+  heavy = true;
   const int hm = min(p.heavy_max, HEAVY_CAP);
-  if (p.force == CLS_HUGE || f > hm) bin = BIN_HUGE;
+  if (c == CLS_SINGLE || p.force == CLS_HUGE || f > hm) bin = BIN_HUGE;
   else if (f <= HEAVY1_CAP && !long1) bin = BIN_HEAVY;
   else if (!long2) bin = BIN_HEAVY2;
   else bin = BIN_HUGE;
-  return bin == BIN_HUGE ? CLS_HUGE : CLS_HEAVY;
+  return c >= 0 ? c : (bin == BIN_HUGE ? CLS_HUGE : CLS_HEAVY);
 }
 
-// Classify this rank's rows [rb, re) (local index li = i - rb): cls[li] = class | light-path bit;
-// fl[li] = f_i for light rows (scanned into the light-product prefix PL); heavy rows are
-// appended to their bitmap bin's list and get R offsets (relative to the end of the light
-// region) from one 64-bit atomic per warp; c_i is written for rows needing no symbolic work
-// (EMPTY: 0; SINGLE: f_i — B canonical, one run).  Per-class statistics are pre-reduced per
-// warp (MATCH.ANY + REDUX, 16-bit halves) and flushed once per block.
+// Classify this rank's rows [rb, re) (local index li = i - rb): cls[li] = class | path flags;
+// pw[li] = plan words of the row (f_i, 2 f_i for wide heavy rows; scanned into Ro).  Heavy rows
+// are appended to their bitmap bin's list.  Per-class statistics are pre-reduced per warp
+// (MATCH.ANY + REDUX, 16-bit halves) and flushed once per block.
 constexpr int CL_NT = 256;
 
 __global__ void __launch_bounds__(CL_NT) k_classify(const int* __restrict__ f, const uint8_t* __restrict__ nz, int rb,
                                                     int re, ClassParams prm, uint8_t* __restrict__ cls,
-                                                    int* __restrict__ fl, long long* __restrict__ Ro,
-                                                    HeavyLists lists, Small* __restrict__ sm,
-                                                    long long* __restrict__ crow, long long* __restrict__ PL) {
+                                                    int* __restrict__ pw, HeavyLists lists, Small* __restrict__ sm) {
   __shared__ unsigned s_rows[NUM_CLS], s_flo[NUM_CLS], s_fhi[NUM_CLS], s_fmax;
   const int tid = threadIdx.x, lane = tid & 31;
   if (tid < NUM_CLS) { s_rows[tid] = 0; s_flo[tid] = 0; s_fhi[tid] = 0; }
   if (tid == 0) s_fmax = 0;
-  if (blockIdx.x == 0 && tid == 0) {
-    crow[0] = 0;
-    PL[0] = 0;
-  }
   __syncthreads();
   const long long n = (long long)re - rb;
   const long long nup = (n + 31) & ~31LL;  // warp-uniform trip count
+  int bad = 0;
   for (long long li = (long long)blockIdx.x * CL_NT + tid; li < nup; li += (long long)gridDim.x * CL_NT) {
     const bool act = li < n;
     int fi = 0, bin = -1, c = -1;
-    bool light = false;
+    bool heavy = false;
     if (act) {
       fi = f[rb + li];
-      c = classify_row(fi, nz[rb + li], prm, bin, light);
-      cls[li] = (uint8_t)(c | (light ? CLS_LIGHT_PATH : 0));
-      fl[li] = light ? fi : 0;
-      if (c == CLS_EMPTY) crow[li + 1] = 0;
-      else if (c == CLS_SINGLE) crow[li + 1] = fi;
-      if (bin < 0) Ro[li] = -1;
+      const int z = nz[rb + li];
+      c = classify_row(fi, z, prm, bin, heavy);
+      const bool wide = heavy && (z & (NZ_LONGB | NZ_ALEN64K));
+      const bool solo = !heavy && (fi > TILE_PMAX - prm.tile_cap || (z & NZ_ALEN1K));
+      cls[li] = (uint8_t)(c | (heavy ? CLS_HEAVY_PATH : 0) | (wide ? CLS_WIDE : 0) | (solo ? CLS_SOLO : 0));
+      if (wide && fi >= (1 << 30)) bad = 2;
+      pw[li] = wide ? 2 * fi : fi;
     }
     const unsigned gc = __match_any_sync(FULL, c);
     if (act) {
@@ -156,16 +164,10 @@ __global__ void __launch_bounds__(CL_NT) k_classify(const int* __restrict__ f, c
     }
     const unsigned fm = __reduce_max_sync(FULL, (unsigned)fi);
     if (lane == 0 && fm) atomicMax(&s_fmax, fm);
-    // heavy rows: list append + R offset (rare: one warp-level scan and atomic when present)
+    // heavy rows: list append (rare: one warp-level atomic per bin when present)
     if (__ballot_sync(FULL, bin >= 0)) {
-      const long long hv = bin >= 0 ? fi : 0;
-      const long long incl = warp_incl_scan(hv);
-      unsigned long long hb = 0;
-      if (lane == 31) hb = atomicAdd(reinterpret_cast<unsigned long long*>(&sm->heavy_total), (unsigned long long)incl);
-      hb = __shfl_sync(FULL, hb, 31);
       const unsigned gb = __match_any_sync(FULL, bin);
       if (bin >= 0) {
-        Ro[li] = (long long)hb + incl - hv;
         const int leader = __ffs(gb) - 1;
         int pos = 0;
         if (lane == leader) pos = atomicAdd(&sm->counts[bin], __popc(gb));
@@ -174,6 +176,7 @@ __global__ void __launch_bounds__(CL_NT) k_classify(const int* __restrict__ f, c
       }
     }
   }
+  if (bad) atomicOr(&sm->err, bad);
   __syncthreads();
   if (tid < NUM_CLS) {
     const unsigned long long fl2 = ((unsigned long long)s_fhi[tid] << 16) + s_flo[tid];
@@ -183,57 +186,68 @@ __global__ void __launch_bounds__(CL_NT) k_classify(const int* __restrict__ f, c
   if (tid == 0 && s_fmax) atomicMax(&sm->cstats[2 * NUM_CLS], (unsigned long long)s_fmax);
 }
 
-// Tiles of light rows.  PL = exclusive prefix of fl (light products, row order).  A light row
-// starts a tile when its product range [PL_i, PL_i + f_i) contains a multiple of `cap`, so a tile
-// of rows with f <= TILE_PMAX - cap holds < TILE_PMAX products; a row with more (up to light_max
-// <= TILE_PMAX) is a solo tile: it starts a tile, and so does the next light row (found by a
-// short look-back; if none within 64 rows the row starts a tile anyway — an extra tile start is
-// always safe).  Light rows get Ro = F_H + PL_i: the plan holds the heavy
-// rows first (their offsets come from k_classify alone, so the heavy kernels start before this).
-// r_ok = (F_L + F_H <= capacity of R): the symbolic kernels do nothing when R is too small and
-// the host re-runs them after growing R.
-__global__ void __launch_bounds__(256) k_tiles(const int* __restrict__ f, int rb, int re, int cap,
-                                               const uint8_t* __restrict__ cls, const long long* __restrict__ PL,
-                                               long long* __restrict__ Ro, uint8_t* __restrict__ tflag,
-                                               int* __restrict__ tiles, Small* __restrict__ sm, long long r_cap) {
+// Item starts.  A heavy row is an item; a non-heavy row starts a tile when the row before it is
+// heavy or solo, when it is solo itself, when its index is a multiple of TILE_RM, or when its plan
+// range [Ro_i, Ro_i + f_i) contains a multiple of `cap` or its A entry range a multiple of TILE_EC.
+// So a tile holds <= TILE_RM rows, < cap + f_first <= TILE_PMAX products and < 2 TILE_EC A
+// entries (rows longer than TILE_EC are heavy, or solo when f = 0).
+__global__ void __launch_bounds__(256) k_tile_flags(const int* __restrict__ f, const int* __restrict__ rpA, int rb,
+                                                    int re, int cap, const uint8_t* __restrict__ cls,
+                                                    const long long* __restrict__ Ro, int* __restrict__ tflag) {
   const long long n = (long long)re - rb;
-  const long long FL = PL[n], HT = sm->heavy_total;
-  const int lane = threadIdx.x & 31;
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    const long long fr = FL + sm->heavy_total;
-    sm->fr = fr;
-    sm->r_ok = fr <= r_cap ? 1 : 0;
-  }
-  const long long nup = (n + 31) & ~31LL;
-  for (long long li = (long long)blockIdx.x * blockDim.x + threadIdx.x; li < nup;
-       li += (long long)gridDim.x * blockDim.x) {
-    bool start = false;
-    if (li < n) {
-      const int c = cls[li];
-      if (c & CLS_LIGHT_PATH) {
-        const long long pl = PL[li];
-        const long long fi = f[rb + li];
-        Ro[li] = HT + pl;
-        start = (pl % cap == 0) || (pl / cap != (pl + fi - 1) / cap) || fi > TILE_PMAX - cap;
-        if (!start) {  // the row after a solo row starts a tile (no light row within 64: start anyway)
-          start = true;
-          for (long long j = li - 1; j >= 0 && j >= li - 64; --j)
-            if (cls[j] & CLS_LIGHT_PATH) {
-              start = f[rb + j] > TILE_PMAX - cap;
-              break;
-            }
-        }
+  for (long long li = (long long)blockIdx.x * blockDim.x + threadIdx.x; li < n; li += (long long)gridDim.x * blockDim.x) {
+    const int c = cls[li];
+    bool start = (c & CLS_HEAVY_PATH) || (c & CLS_SOLO) || li == 0 || (li % TILE_RM) == 0;
+    if (!start) {
+      const int cp = cls[li - 1];
+      start = (cp & CLS_HEAVY_PATH) || (cp & CLS_SOLO);
+    }
+    if (!start) {
+      const long long fi = f[rb + li];
+      if (fi > 0) {
+        const long long pl = Ro[li];
+        start = (pl % cap == 0) || (pl / cap != (pl + fi - 1) / cap);
       }
-      tflag[li] = start ? 1 : 0;
+      const long long ea = rpA[rb + li], al = rpA[rb + li + 1] - ea;
+      if (al > 0) start = start || (ea % TILE_EC == 0) || (ea / TILE_EC != (ea + al - 1) / TILE_EC);
     }
-    const unsigned m = __ballot_sync(FULL, start);
-    if (m) {
-      int base = 0;
-      if (lane == 0) base = atomicAdd(&sm->ntiles, __popc(m));
-      base = __shfl_sync(FULL, base, 0);
-      if (start) tiles[base + __popc(m & lanemask_lt())] = (int)li;
-    }
+    tflag[li] = start ? 1 : 0;
   }
+}
+
+// items[k] = the k-th item start (tscan = inclusive scan of the start flags); items[n] = Mloc.
+__global__ void __launch_bounds__(256) k_items(const int* __restrict__ tflag, const long long* __restrict__ tscan,
+                                               int mloc, int* __restrict__ items, Small* __restrict__ sm) {
+  for (long long li = (long long)blockIdx.x * blockDim.x + threadIdx.x; li < mloc; li += (long long)gridDim.x * blockDim.x)
+    if (tflag[li]) items[tscan[li] - 1] = (int)li;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    const int n = mloc > 0 ? (int)tscan[mloc - 1] : 0;
+    items[n] = mloc;
+    sm->nitems = n;
+  }
+}
+
+// Numeric work units per item t (unit counts ucnt[t]; hd[t] = 0: no output unit done yet).
+__global__ void __launch_bounds__(256) k_unit_count(const int* __restrict__ items, const long long* __restrict__ crow,
+                                                    const long long* __restrict__ Ro, const uint8_t* __restrict__ cls,
+                                                    int n, int* __restrict__ ucnt, int* __restrict__ hd) {
+  for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < n; t += (long long)gridDim.x * blockDim.x) {
+    const int r = items[t], r2 = items[t + 1];
+    const long long c = crow[r2] - crow[r];
+    ucnt[t] = (int)((c + NUM_SH - 1) / NUM_SH);
+    hd[t] = 0;
+  }
+}
+
+__global__ void __launch_bounds__(256) k_unit_fill(const int* __restrict__ ucnt, const long long* __restrict__ uscan,
+                                                   int n, int2* __restrict__ units, Small* __restrict__ sm,
+                                                   const int* __restrict__ items, const long long* __restrict__ crow) {
+  for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < n; t += (long long)gridDim.x * blockDim.x) {
+    const int u = ucnt[t];
+    const long long b = uscan[t] - u;
+    for (int k = 0; k < u; ++k) units[b + k] = make_int2((int)t, k);
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) sm->nunits = n > 0 ? uscan[n - 1] : 0;
 }
 
 // ---- inclusive scan to int64 (three passes: tile scan, tile-sum scan, add) -------------------
@@ -371,25 +385,53 @@ __global__ void k_narrow(const long long* __restrict__ in, int* __restrict__ out
 
 // ---- host launchers ------------------------------------------------------------------------
 cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB,
-                             int* f, uint8_t* nz, unsigned long long* hist, int* err, int* amax) {
+                             int* f, uint8_t* nz, int* Tb, int* Tl, unsigned long long* hist, int* err, int* amax) {
   if (M <= 0) return cudaSuccess;
   constexpr int ROWS = 256;
-  k_row_flops<ROWS><<<(M + ROWS - 1) / ROWS, ROWS, 0, st>>>(M, rpA, colA, K, rpB, f, nz, hist, err, amax);
+  k_row_flops<ROWS><<<(M + ROWS - 1) / ROWS, ROWS, 0, st>>>(M, rpA, colA, K, rpB, f, nz, Tb, Tl, hist, err, amax);
   return cudaGetLastError();
 }
 
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
-                            const ClassParams& prm, uint8_t* cls, int* fl, long long* Ro, const HeavyLists& lists,
-                            Small* small, long long* crow, long long* PL) {
+                            const ClassParams& prm, uint8_t* cls, int* pw, const HeavyLists& lists, Small* small) {
   const long long n = (long long)re - rb;
-  if (n <= 0) {
-    cudaError_t e = cudaMemsetAsync(crow, 0, sizeof(long long), st);
-    if (e == cudaSuccess) e = cudaMemsetAsync(PL, 0, sizeof(long long), st);
-    return e;
-  }
+  if (n <= 0) return cudaSuccess;
   long long blocks = (n + CL_NT - 1) / CL_NT;
   if (blocks > (long long)sms * 8) blocks = (long long)sms * 8;
-  k_classify<<<(int)blocks, CL_NT, 0, st>>>(f, nz, rb, re, prm, cls, fl, Ro, lists, small, crow, PL);
+  k_classify<<<(int)blocks, CL_NT, 0, st>>>(f, nz, rb, re, prm, cls, pw, lists, small);
+  return cudaGetLastError();
+}
+
+static int grid_for_rows(long long n, int sms) {
+  long long g = (n + 255) / 256;
+  if (g > (long long)sms * 8) g = (long long)sms * 8;
+  return (int)(g < 1 ? 1 : g);
+}
+
+cudaError_t launch_tile_flags(cudaStream_t st, int sms, const int* f, const int* rpA, int rb, int re, int tile_cap,
+                              const uint8_t* cls, const long long* Ro, int* tflag) {
+  const long long n = (long long)re - rb;
+  if (n <= 0) return cudaSuccess;
+  k_tile_flags<<<grid_for_rows(n, sms), 256, 0, st>>>(f, rpA, rb, re, tile_cap, cls, Ro, tflag);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_unit_count(cudaStream_t st, int sms, const int* items, const long long* crow, const long long* Ro,
+                              const uint8_t* cls, int n, int* ucnt, int* hd) {
+  if (n <= 0) return cudaSuccess;
+  k_unit_count<<<grid_for_rows(n, sms), 256, 0, st>>>(items, crow, Ro, cls, n, ucnt, hd);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_unit_fill(cudaStream_t st, int sms, const int* ucnt, const long long* uscan, int n, int2* units,
+                             Small* small, const int* items, const long long* crow) {
+  k_unit_fill<<<grid_for_rows(n, sms), 256, 0, st>>>(ucnt, uscan, n, units, small, items, crow);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_items(cudaStream_t st, int sms, const int* tflag, const long long* tscan, int mloc, int* items,
+                         Small* small) {
+  k_items<<<grid_for_rows(mloc, sms), 256, 0, st>>>(tflag, tscan, mloc, items, small);
   return cudaGetLastError();
 }
 
@@ -435,17 +477,6 @@ __global__ void __launch_bounds__(1024) k_sort_lists(HeavyLists lists, int b, co
 cudaError_t launch_sort_list(cudaStream_t st, const HeavyLists& lists, int bin, const int* f, int rb,
                              const Small* small) {
   k_sort_lists<<<1, 1024, 0, st>>>(lists, bin, f, rb, small);
-  return cudaGetLastError();
-}
-
-cudaError_t launch_tiles(cudaStream_t st, int sms, const int* f, int rb, int re, int tile_cap, const uint8_t* cls,
-                         const long long* PL, long long* Ro, uint8_t* tflag, int* tiles, Small* small,
-                         long long r_cap) {
-  const long long n = (long long)re - rb;
-  long long blocks = (n + 255) / 256;
-  if (blocks > (long long)sms * 8) blocks = (long long)sms * 8;
-  if (blocks < 1) blocks = 1;
-  k_tiles<<<(int)blocks, 256, 0, st>>>(f, rb, re, tile_cap, cls, PL, Ro, tflag, tiles, small, r_cap);
   return cudaGetLastError();
 }
 

@@ -79,17 +79,10 @@ struct spg_ctx {
   // options
   int light_max = LIGHT_MAX_DEFAULT, tile_cap = TILE_CAP_DEFAULT, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
-  // numeric: gather B through a packed {column, value} copy — one sector per gather instead of
-  // two when B does not stay in L2 (auto: B's columns + values > 64 MB; SPG_PACK_B=0/1 forces;
-  // always-on measured neutral on the L2-resident configs)
-  int pack_b = -1;
-  int l2_persist = 0;  // experimental: 1 persisting-L2 window over B during numeric (reset after), 2 without the reset
-  int thresholds_set = 0;
-  int warp_max = WARP_MAX_DEFAULT;  // light rows with f <= warp_max: one warp per row (k_warp.cu)
-  int occ_warp = 1;  // light_max / tile_cap set by the caller (else N-dependent defaults)
-  // workspace: analysis (all rows / all A entries), classification (this rank's rows), R, windows
-  DevBuf f, nz, cls, fl, Ro, PL, tflag, tiles, lists, fblist, small, scan_tmp, EQ, fl8, dup, nd, ne, chunk_row, packB, Pf,
-      splits, canonB[4], iota, ones, crow_tmp;
+  int thresholds_set = 0;  // light_max / tile_cap set by the caller (else N-dependent defaults)
+  // workspace: analysis (all rows), classification and items (this rank's rows), the plan
+  DevBuf f, nz, Tb, Tl, cls, pw, Ro, tflag, tscan, items, lists, small, scan_tmp, plan, fl8, D, ucnt, uscan,
+      units, hd, ticket, Pf, splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
   long long iota_n = -1, ones_n = -1;
@@ -97,15 +90,16 @@ struct spg_ctx {
   cudaStream_t aux[6] = {};
   cudaEvent_t ev_fork = nullptr, ev_fork2 = nullptr, ev_join[6] = {};
   cudaEvent_t ev_t[8] = {};
-  cudaEvent_t ev_p[4] = {};  // light path start/end, heavy path start/end
-  int occ_light = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1;
+  cudaEvent_t ev_p[4] = {};  // tile path start/end, heavy path start/end
+  int occ_tile = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1;
+  int epoch = 0;  // numeric calls since the last symbolic
   // cached symbolic state
   bool sym_ok = false;
   SymKey key{};
   int32_t rb = 0, re = 0;
   int64_t nnzC = 0;
-  long long ndup = 0, dupcap = 0;
-  int nch = 0, chcap = 0;
+  long long plan_words = 0;
+  int nitems = 0;
   int counts[NUM_BINS] = {};
   spg_stats stats{};
   bool num_timed = false, paths_timed = false;
@@ -115,6 +109,14 @@ struct spg_ctx {
   spg_csr hA{}, hB{};
   bool host_sym_ok = false;
   std::string err;
+  // plan words every plan-indexed buffer can hold (plan, D: a word each; fl8: a byte)
+  long long plan_cap() const {
+    if (!plan.p || !D.p || !fl8.p) return 0;
+    long long c = (long long)(plan.cap / sizeof(unsigned));
+    if ((long long)(D.cap / sizeof(unsigned)) < c) c = (long long)(D.cap / sizeof(unsigned));
+    if ((long long)fl8.cap < c) c = (long long)fl8.cap;
+    return c;
+  }
 };
 
 namespace {
@@ -176,35 +178,29 @@ int ceil_log2(long long n) {
 SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
   SymProb P;
   P.rpA = A->row_ptr; P.colA = A->col_idx; P.rpB = B->row_ptr; P.colB = B->col_idx;
+  P.Tb = h->Tb.as<int>();
+  P.Tl = h->Tl.as<int>();
   P.frow = h->f.as<int>();
   P.cls = h->cls.as<uint8_t>();
   P.Ro = h->Ro.as<long long>();
-  P.EQ = h->EQ.as<int2>();
-  P.dup = h->dup.as<int4>();
-  P.dupn = &h->small.as<Small>()->dupn;
-  P.dupcap = h->dupcap;
+  P.plan = h->plan.as<unsigned>();
   P.fl8 = h->fl8.as<uint8_t>();
   P.crow = crow;
-  P.r_ok = &h->small.as<Small>()->r_ok;
-  P.heavy_total = &h->small.as<Small>()->heavy_total;
-  {
-    long long r_cap = h->EQ.p && h->fl8.p ? (long long)(h->EQ.cap / sizeof(int2)) : 0;
-    if (r_cap > (long long)h->fl8.cap) r_cap = (long long)h->fl8.cap;
-    P.r_cap = r_cap;
-  }
+  P.D = h->D.as<unsigned>();
+  P.dups = &h->small.as<Small>()->dups;
+  long long r_cap = h->plan_cap();
+  P.r_cap = r_cap;
   P.row_begin = h->rb;
   P.row_end = h->re;
-  P.lgN = ceil_log2(B->ncols);
   return P;
 }
 
-// Symbolic class kernels: the heavy bitmap bins and the light tiles on concurrent streams (the
+// Symbolic class kernels: the heavy bitmap bins and the tiles on concurrent streams (the
 // paper's concurrent CPU and GPU legs of Phases II/III, recast as
-// concurrent kernels on one GPU), then the rows the light kernel handed over.  Bin sizes are
-// device-side: every kernel is a persistent grid that exits at once when its list is empty.
-// The heavy bins fork right after k_classify (their plan offsets are final there), so they
-// overlap the light-product scan and the tile cut; the light tiles fork after k_tiles.
-spg_status run_heavy(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
+// concurrent kernels on one GPU).  Bin sizes are device-side: every kernel is a persistent grid
+// that exits at once when its list is empty.  The heavy bins fork as soon as the plan offsets Ro
+// exist, so they overlap the tile cut.
+spg_status fork_heavy(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
   const SymProb P = make_sym(h, A, B, crow);
   Small* ds = h->small.as<Small>();
   const bool conc = h->concurrent != 0;
@@ -219,84 +215,65 @@ spg_status run_heavy(spg_handle h, const spg_csr* A, const spg_csr* B, long long
     if (tm && x == 0) CK(cudaEventRecord(h->ev_p[2], st));
     long long grid = (long long)h->occ_heavy[b] * h->sms;
     if (h->huge_slots_opt > 0 && h->huge_slots_opt < grid) grid = h->huge_slots_opt;
-    const int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
+    int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
     if (b != BIN_HEAVY && Mloc > 0) {  // largest rows first (the HEAVY bin's list is too long to pay)
       HeavyLists L3;
-      for (int c = 0; c < NUM_LISTS; ++c) L3.rows[c] = h->lists.as<int>() + (size_t)c * (size_t)Mloc;
+      for (int c = 0; c < NUM_BINS; ++c) L3.rows[c] = h->lists.as<int>() + (size_t)c * (size_t)Mloc;
       CK(launch_sort_list(st, L3, b, h->f.as<int>(), h->rb, ds));
       h->launches++;
     }
-    CK(launch_heavy_rank(b, st, (int)grid, P, list, ds->counts + b, B->ncols, 0));
+    CK(launch_heavy_rank(b, st, (int)grid, P, list, ds->counts + b, B->ncols));
     h->launches++;
     if (conc) CK(cudaEventRecord(h->ev_join[1 + x], st));
-  }
-  {  // the smallest light rows, one warp per row, on their own stream
-    cudaStream_t st = conc ? h->aux[4] : h->stream;
-    if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
-    const int* list = h->lists.as<int>() + (size_t)BIN_WARP * (size_t)(Mloc > 0 ? Mloc : 1);
-    CK(launch_warp_rank(st, h->occ_warp * h->sms, P, list, ds->counts + BIN_WARP));
-    h->launches++;
-    if (conc) CK(cudaEventRecord(h->ev_join[4], st));
   }
   return SPG_OK;
 }
 
-spg_status run_light(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
+spg_status run_tiles(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
   const SymProb P = make_sym(h, A, B, crow);
   Small* ds = h->small.as<Small>();
   const bool conc = h->concurrent != 0;
   const bool tm = h->timing != 0;
-  if (conc) CK(cudaEventRecord(h->ev_fork2, h->stream));
-  {
-    cudaStream_t st = conc ? h->aux[0] : h->stream;
-    if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork2, 0));
-    if (tm) CK(cudaEventRecord(h->ev_p[0], st));
-    CK(launch_light_rank(st, h->occ_light * h->sms, P, h->tiles.as<int>(), &ds->ntiles, &ds->tqhead,
-                         h->tflag.as<uint8_t>(), h->PL.as<long long>(), h->fblist.as<int>(), ds->fb));
-    h->launches++;
-    if (tm) CK(cudaEventRecord(h->ev_p[1], st));
-    if (conc) {
-      CK(cudaEventRecord(h->ev_join[0], st));
-      CK(cudaStreamWaitEvent(h->stream, h->ev_join[0], 0));
-    }
-  }
+  if (tm) CK(cudaEventRecord(h->ev_p[0], h->stream));
+  CK(launch_tile_rank(h->stream, h->occ_tile * h->sms, P, h->items.as<int>(), &ds->nitems, &ds->tqhead));
+  h->launches++;
+  if (tm) CK(cudaEventRecord(h->ev_p[1], h->stream));
   if (conc)
-    for (int x = 0; x < NUM_BINS + 1; ++x) CK(cudaStreamWaitEvent(h->stream, h->ev_join[1 + x], 0));
+    for (int x = 0; x < NUM_BINS; ++x) CK(cudaStreamWaitEvent(h->stream, h->ev_join[1 + x], 0));
   if (tm) CK(cudaEventRecord(h->ev_p[3], h->stream));
   h->paths_timed = tm;
-  // rows with clustered columns, handed over by the light kernel
-  long long grid = (long long)h->occ_heavy[BIN_HUGE] * h->sms;
-  CK(launch_heavy_rank(BIN_HUGE, h->stream, (int)grid, P, h->fblist.as<int>(), ds->fb, B->ncols, 1));
-  h->launches++;
   return SPG_OK;
 }
 
 spg_status ensure_ws(spg_handle h, int M, long long nnzA) {
   size_t m = (size_t)(M > 0 ? M : 1);
   size_t na = (size_t)(nnzA > 0 ? nnzA : 1);
+  CK(h->Tb.ensure(na * sizeof(int)));
+  CK(h->Tl.ensure(na * sizeof(int)));
+  CK(h->ucnt.ensure((m + 1) * sizeof(int)));
+  CK(h->uscan.ensure((m + 1) * sizeof(long long)));
+  CK(h->hd.ensure((m + 1) * sizeof(int)));
+  CK(h->ticket.ensure(sizeof(int)));
   CK(h->f.ensure(m * sizeof(int)));
   CK(h->nz.ensure(m));
   CK(h->cls.ensure(m));
-  CK(h->fl.ensure(m * sizeof(int)));
-  CK(h->Ro.ensure(m * sizeof(long long)));
-  CK(h->PL.ensure((m + 1) * sizeof(long long)));
-  CK(h->tflag.ensure(m));
-  CK(h->tiles.ensure(m * sizeof(int)));
-  CK(h->lists.ensure(m * NUM_LISTS * sizeof(int)));
-  CK(h->fblist.ensure(m * sizeof(int)));
-  CK(h->nd.ensure(m * sizeof(long long)));
-  CK(h->ne.ensure(m * sizeof(int)));
+  CK(h->pw.ensure(m * sizeof(int)));
+  CK(h->Ro.ensure((m + 1) * sizeof(long long)));
+  CK(h->tflag.ensure(m * sizeof(int)));
+  CK(h->tscan.ensure(m * sizeof(long long)));
+  CK(h->items.ensure((m + 1) * sizeof(int)));
+  CK(h->lists.ensure(m * NUM_BINS * sizeof(int)));
   CK(h->small.ensure(sizeof(Small)));
   CK(h->scan_tmp.ensure(scan_tmp_elems((long long)m + 1) * sizeof(long long)));
   return SPG_OK;
 }
 
-// Row analysis over all rows (f_i, run flags, log2 histogram, per-entry row and offset).
+// Row analysis over all rows (f_i, run count and size flags, log2 histogram).
 spg_status analysis(spg_handle h, const spg_csr* A, const spg_csr* B) {
   Small* ds = h->small.as<Small>();
   CK(cudaMemsetAsync(ds, 0, sizeof(Small), h->stream));
   CK(launch_row_flops(h->stream, A->nrows, A->row_ptr, A->col_idx, B->nrows, B->row_ptr, h->f.as<int>(),
-                      h->nz.as<uint8_t>(), ds->hist, &ds->err, &ds->amax));
+                      h->nz.as<uint8_t>(), h->Tb.as<int>(), h->Tl.as<int>(), ds->hist, &ds->err, &ds->amax));
   h->launches += A->nrows > 0;
   return SPG_OK;
 }
@@ -380,8 +357,11 @@ spg_status validate_device(spg_handle h, const spg_csr* A, const spg_csr* B) {
   return SPG_OK;
 }
 
-// a2 + symbolic classes: after analysis / classification (this rank's rows), the light and heavy
-// kernels compute R and c_i; scan of c_i -> C_row_ptr; one readback of nnz(C) and the stats.
+// Phase I + symbolic: analysis and classification (this rank's rows), plan offsets, the item
+// list, then the heavy and tile kernels compute c_i and the plan; scan of c_i -> C_row_ptr; one
+// readback of nnz(C) and the statistics.  The first call (or a larger plan) finds the plan too
+// small: the kernels then skip their work, the plan is grown to the exact size read back and the
+// pass reruns.
 spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64_t* C_row_ptr, int64_t* nnzC,
                          int32_t* row_begin, int32_t* row_end) {
   const int M = A->nrows;
@@ -395,9 +375,6 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   long long Mloc = 0;
   Small* ds = h->small.as<Small>();
   long long* crow = reinterpret_cast<long long*>(C_row_ptr);
-  // The first call (or a larger product count) finds the gather plan too small — the kernels then
-  // skip their work, EQ is grown to the exact size read back, and the pass reruns; likewise a dup
-  // list that overflowed.
   for (int attempt = 0;; ++attempt) {
     h->launches = 0;
     if (h->timing) CK(cudaEventRecord(h->ev_t[0], h->stream));
@@ -416,80 +393,68 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     Mloc = h->re - h->rb;
     // Default thresholds depend on the column count: a bitmap row spans ceil(N / 2^20) column
     // tiles and its per-row cost multiplies with them.  With more than 4 tiles more rows go to the
-    // light tiles (tools/sweep.py, profiles/r01_threshold_sweep_configs.jsonl: rmat23, 8 tiles,
-    // 28.3 -> 31.5 GFLOP/s; at 2-4 tiles (ab2m, citpatents) 2048/2048 stays best).  Explicitly
-    // set options are kept as given.
+    // tiles (tools/sweep.py, profiles/r01_threshold_sweep_configs.jsonl).  Explicitly set options
+    // are kept as given.
     int light_max = h->light_max, tile_cap = h->tile_cap;
     if (!h->thresholds_set && B->ncols > (1 << 22)) {
       light_max = TILE_PMAX - 1024;
       tile_cap = 1024;
     }
-    ClassParams prm{light_max, h->heavy_max, tile_cap, h->force, h->canonical ? 1 : 0,
-                    h->warp_max < light_max ? h->warp_max : light_max};
-    int* lists = h->lists.as<int>();
+    ClassParams prm{light_max, h->heavy_max, tile_cap, h->force, h->canonical ? 1 : 0};
     HeavyLists L3;
-    for (int b = 0; b < NUM_LISTS; ++b) L3.rows[b] = lists + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
-    long long* PL = h->PL.as<long long>();
-    // (also zeroes crow[0] and PL[0]; the queue heads were zeroed with Small in analysis())
+    for (int b = 0; b < NUM_BINS; ++b) L3.rows[b] = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
+    long long* Ro = h->Ro.as<long long>();
+    CK(cudaMemsetAsync(crow, 0, sizeof(long long), h->stream));
+    CK(cudaMemsetAsync(Ro, 0, sizeof(long long), h->stream));
     CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm,
-                       h->cls.as<uint8_t>(), h->fl.as<int>(), h->Ro.as<long long>(), L3, ds, crow, PL));
-    if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));  // analysis = row flops + classify
-    if ((s = run_heavy(h, A, B, crow)) != SPG_OK) return s;
-    CK(launch_incl_scan<int>(h->stream, h->fl.as<int>(), PL + 1, Mloc, h->scan_tmp.as<long long>()));
-    long long r_cap = h->EQ.p && h->fl8.p ? (long long)(h->EQ.cap / sizeof(int2)) : 0;
-    if (r_cap > (long long)h->fl8.cap) r_cap = (long long)h->fl8.cap;
-    CK(launch_tiles(h->stream, h->sms, h->f.as<int>(), h->rb, h->re, tile_cap, h->cls.as<uint8_t>(), PL,
-                    h->Ro.as<long long>(), h->tflag.as<uint8_t>(), h->tiles.as<int>(), ds, r_cap));
-    h->launches += (Mloc > 0) + scan_launches(Mloc) + 1;
-    if ((s = run_light(h, A, B, crow)) != SPG_OK) return s;
+                       h->cls.as<uint8_t>(), h->pw.as<int>(), L3, ds));
+    CK(launch_incl_scan<int>(h->stream, h->pw.as<int>(), Ro + 1, Mloc, h->scan_tmp.as<long long>()));
+    CK(launch_tile_flags(h->stream, h->sms, h->f.as<int>(), A->row_ptr, h->rb, h->re, tile_cap, h->cls.as<uint8_t>(),
+                         Ro, h->tflag.as<int>()));
+    CK(launch_incl_scan<int>(h->stream, h->tflag.as<int>(), h->tscan.as<long long>(), Mloc,
+                             h->scan_tmp.as<long long>()));
+    h->launches += 2 * (Mloc > 0) + 2 * scan_launches(Mloc);
+    if (h->timing) CK(cudaEventRecord(h->ev_t[1], h->stream));  // analysis = row flops, classify, Ro, items
+    if ((s = fork_heavy(h, A, B, crow)) != SPG_OK) return s;
+    CK(launch_items(h->stream, h->sms, h->tflag.as<int>(), h->tscan.as<long long>(), (int)Mloc, h->items.as<int>(), ds));
+    h->launches += 1;
+    if ((s = run_tiles(h, A, B, crow)) != SPG_OK) return s;
     CK(launch_incl_scan<long long>(h->stream, crow + 1, crow + 1, Mloc, h->scan_tmp.as<long long>()));
-    // numeric plan: per-row EQ-to-C offsets and chunk -> row (capacity from the last call; a
-    // larger need reruns the plan below)
-    if (h->chcap < 2) h->chcap = 2;
-    CK(h->chunk_row.ensure((size_t)h->chcap * sizeof(int)));
-    CK(launch_plan(h->stream, h->sms, crow, (int)Mloc, A->row_ptr, A->col_idx, B->row_ptr, h->cls.as<uint8_t>(),
-                   h->Ro.as<long long>(), h->rb, h->nd.as<long long>(), h->ne.as<int>(), h->chunk_row.as<int>(),
-                   h->chcap, ds));
-    h->launches += scan_launches(Mloc) + (Mloc > 0);
+    h->launches += scan_launches(Mloc);
     if (h->timing) CK(cudaEventRecord(h->ev_t[2], h->stream));
     CK(cudaMemcpyAsync(&h->hr->small, ds, sizeof(Small), cudaMemcpyDeviceToHost, h->stream));
     CK(cudaMemcpyAsync(&h->hr->nnz, crow + Mloc, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
+    CK(cudaMemcpyAsync(&h->hr->ncut, Ro + Mloc, sizeof(long long), cudaMemcpyDeviceToHost, h->stream));
     CK(cudaStreamSynchronize(h->stream));
     const Small& hs = h->hr->small;
     if (hs.err & 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "A has a column index outside [0, B.nrows)");
-    if (hs.err & 2) return setf(h, SPG_ERR_INDEX_OVERFLOW, "a row of A has >= 2^31 intermediate products");
-    const bool dup_ok = (long long)hs.dupn <= h->dupcap;
-    if (hs.r_ok && dup_ok && hs.nch_need > h->chcap) {  // more chunks than room: grow, rerun the plan
-      h->chcap = hs.nch_need + 64;
-      CK(h->chunk_row.ensure((size_t)h->chcap * sizeof(int)));
-      CK(launch_plan(h->stream, h->sms, crow, (int)Mloc, A->row_ptr, A->col_idx, B->row_ptr, h->cls.as<uint8_t>(),
-                     h->Ro.as<long long>(), h->rb, h->nd.as<long long>(), h->ne.as<int>(), h->chunk_row.as<int>(),
-                     h->chcap, ds));
-      h->launches += (Mloc > 0);
-      CK(cudaStreamSynchronize(h->stream));
+    if (hs.err & 2) return setf(h, SPG_ERR_INDEX_OVERFLOW, "a row of A has too many intermediate products (>= 2^31, or >= 2^30 with 64-bit plan entries)");
+    const long long words = h->hr->ncut;
+    if (words <= h->plan_cap()) {
+      h->plan_words = words;
+      break;
     }
-    if (hs.r_ok && !dup_ok && attempt < 3) {  // dup list too small: grow to the exact need, rerun
-      h->dupcap = (long long)hs.dupn + 1024;
-      CK(h->dup.ensure((size_t)h->dupcap * sizeof(int4)));
-      continue;
-    }
-    if (!dup_ok && hs.r_ok) return setf(h, SPG_ERR_OUT_OF_MEMORY, "dup list could not be sized");
-    if (hs.r_ok || attempt > 0) break;
-    {  // gather plan, first-claim flags and a first dup list sized from the product count
-      const size_t fr = (size_t)(hs.fr > 0 ? hs.fr : 1);
-      CK(h->EQ.ensure(fr * sizeof(int2)));
-      CK(h->fl8.ensure(fr));
-      if (h->dupcap < (long long)(fr / 8 + 1024)) {
-        h->dupcap = (long long)(fr / 8 + 1024);
-        CK(h->dup.ensure((size_t)h->dupcap * sizeof(int4)));
-      }
-    }
+    if (attempt > 0) return setf(h, SPG_ERR_OUT_OF_MEMORY, "plan could not be sized");
+    // too small: nothing ran; grow to the exact size and rerun
+    CK(h->plan.ensure((size_t)words * sizeof(unsigned)));
+    CK(h->D.ensure((size_t)words * sizeof(unsigned)));
+    CK(h->fl8.ensure((size_t)words));
   }
   const Small& hs = h->hr->small;
-  if (!hs.r_ok && hs.fr > 0) return setf(h, SPG_ERR_OUT_OF_MEMORY, "gather plan could not be sized");
   h->nnzC = h->hr->nnz;
-  h->ndup = (long long)hs.dupn;
-  h->nch = (int)((h->nnzC + NUM_CH - 1) / NUM_CH);
+  h->nitems = hs.nitems;
+  {  // numeric work units (structure only: built once, reused by every numeric call)
+    const long long ucap = (long long)hs.nitems + h->nnzC / NUM_SH + 2;
+    CK(h->units.ensure((size_t)ucap * sizeof(int2)));
+    const int n = hs.nitems;
+    CK(launch_unit_count(h->stream, h->sms, h->items.as<int>(), crow, h->Ro.as<long long>(), h->cls.as<uint8_t>(), n,
+                         h->ucnt.as<int>(), h->hd.as<int>()));
+    CK(launch_incl_scan<int>(h->stream, h->ucnt.as<int>(), h->uscan.as<long long>(), n, h->scan_tmp.as<long long>()));
+    CK(launch_unit_fill(h->stream, h->sms, h->ucnt.as<int>(), h->uscan.as<long long>(), n, h->units.as<int2>(), ds,
+                        h->items.as<int>(), crow));
+    h->launches += 2 + scan_launches(n);
+    h->epoch = 0;
+  }
   for (int b = 0; b < NUM_BINS; ++b) h->counts[b] = hs.counts[b];
   spg_stats& st = h->stats;
   std::memset(&st, 0, sizeof st);
@@ -505,11 +470,12 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     st.class_flops[c] = (int64_t)hs.cstats[NUM_CLS + c];
   }
   for (int b = 0; b < 65; ++b) st.bin_hist[b] = (int64_t)hs.hist[b];
-  st.tiles = hs.ntiles;
-  st.fallback_rows = hs.fb[0];
-  // gather-plan bytes numeric reads: an EQ entry per output of a non-SINGLE row (a SINGLE row's
-  // c_i = f_i outputs need none) and the dup list
-  st.rank_bytes = (h->nnzC - st.class_flops[CLS_SINGLE]) * (int64_t)sizeof(int2) + h->ndup * (int64_t)sizeof(int4);
+  int nheavy = 0;
+  for (int b = 0; b < NUM_BINS; ++b) nheavy += hs.counts[b];
+  st.heavy_rows = nheavy;
+  st.tiles = hs.nitems - nheavy;
+  st.dup_products = hs.dups;
+  st.plan_bytes = h->plan_words * (int64_t)sizeof(unsigned);
   st.launches_symbolic = h->launches;
   if (h->timing) {
     cudaEventElapsedTime(&st.ms_analysis, h->ev_t[0], h->ev_t[1]);
@@ -535,64 +501,28 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
   h->launches = 0;
   if (h->nnzC > 0) {
     NumProb<V> P;
+    P.rpA = A->row_ptr;
     P.valA = (const V*)A->vals;
+    P.Tb = h->Tb.as<int>();
     P.colB = B->col_idx;
     P.valB = (const V*)B->vals;
-    P.EQ = h->EQ.as<int2>();
-    P.dup = h->dup.as<int4>();
+    P.plan = h->plan.as<unsigned>();
+    P.Ro = h->Ro.as<long long>();
     P.crow = reinterpret_cast<const long long*>(C_row_ptr);
-    P.nd = h->nd.as<long long>();
-    P.ne = h->ne.as<int>();
-    P.chunk_row = h->chunk_row.as<int>();
-    P.nnz = h->nnzC;
-    P.ndup = h->ndup;
-    P.nch = h->nch;
-    P.mloc = h->re - h->rb;
-    P.nB = B->nnz;
-    P.packB = nullptr;
-    const bool pack = h->pack_b > 0 || (h->pack_b < 0 && (long long)B->nnz * (4 + (long long)sizeof(V)) > (64LL << 20));
-    if (pack && B->nnz > 0) {
-      CK(h->packB.ensure((size_t)B->nnz * (sizeof(V) == 8 ? 16 : 8)));
-      P.packB = h->packB.p;
-    }
+    P.cls = h->cls.as<uint8_t>();
+    P.items = h->items.as<int>();
+    P.units = h->units.as<int2>();
+    P.nunits = &h->small.as<Small>()->nunits;
+    P.D = h->D.as<unsigned>();
+    P.hd = h->hd.as<int>();
+    P.ticket = h->ticket.as<int>();
+    P.epoch = ++h->epoch;
+    P.row_begin = h->rb;
     P.ccol = C_col;
     P.cval = (V*)C_val;
-    // One block per chunk: finished blocks are replaced by the hardware block scheduler, so the
-    // chunks' dependent load chains overlap better than in a resident grid-stride loop
-    // (tools/grid_ab.sh: webbase1m numeric 0.677 -> 0.639 ms, webgoogle 0.47 -> 0.454, citpatents
-    // 1.28 -> 1.27). -DSPG_NUM_RESIDENT_GRID restores occupancy x SMs blocks.
-    int grid = (int)(h->nch < INT_MAX ? h->nch : INT_MAX);
-#ifdef SPG_NUM_RESIDENT_GRID
-    grid = h->occ_num * h->sms;
-    if (h->nch < grid) grid = h->nch;
-#endif
-    // Experimental (SPG_L2_PERSIST=1): keep the gathered B (packed copy, else B's values) in
-    // the persisting part of L2 while the streaming plan reads and C stores pass through.
-    const void* win = P.packB ? (const void*)P.packB : (const void*)P.valB;
-    const size_t win_bytes = P.packB ? (size_t)B->nnz * (sizeof(V) == 8 ? 16 : 8) : (size_t)B->nnz * sizeof(V);
-    const bool persist = h->l2_persist > 0 && win_bytes > 0;
-    if (persist) {
-      int dev = 0, maxp = 0, maxw = 0;
-      CK(cudaGetDevice(&dev));
-      CK(cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev));
-      CK(cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev));
-      CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp));
-      cudaStreamAttrValue a = {};
-      a.accessPolicyWindow.base_ptr = const_cast<void*>(win);
-      a.accessPolicyWindow.num_bytes = win_bytes < (size_t)maxw ? win_bytes : (size_t)maxw;
-      a.accessPolicyWindow.hitRatio = win_bytes <= (size_t)maxp ? 1.0f : (float)maxp / (float)win_bytes;
-      a.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-      a.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-      CK(cudaStreamSetAttribute(h->stream, cudaStreamAttributeAccessPolicyWindow, &a));
-    }
-    CK(launch_numeric<V>(h->stream, grid, P));
-    h->launches += (h->nch > 0) + (h->ndup > 0) + (P.packB != nullptr);
-    if (persist) {
-      cudaStreamAttrValue a = {};
-      a.accessPolicyWindow.num_bytes = 0;
-      CK(cudaStreamSetAttribute(h->stream, cudaStreamAttributeAccessPolicyWindow, &a));
-      if (h->l2_persist == 1) CK(cudaCtxResetPersistingL2Cache());
-    }
+    CK(cudaMemsetAsync(P.ticket, 0, sizeof(int), h->stream));
+    CK(launch_numeric<V>(h->stream, h->occ_num * h->sms, P));
+    h->launches += 1;
   }
   h->stats.launches_numeric = h->launches;
   if (h->timing) {
@@ -627,9 +557,8 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     return SPG_ERR_CUDA;
   }
   cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, device);
-  e = light_configure();
+  e = tile_configure();
   if (e == cudaSuccess) e = heavy_configure();
-  if (e == cudaSuccess) e = dtype == SPG_FP64 ? numeric_configure<double>() : numeric_configure<float>();
   if (e == cudaSuccess) e = cudaHostAlloc((void**)&h->hr, sizeof(HostRead), cudaHostAllocDefault);
   for (int c = 0; c < 6 && e == cudaSuccess; ++c) {
     e = cudaStreamCreateWithFlags(&h->aux[c], cudaStreamNonBlocking);
@@ -644,12 +573,9 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     spg_spgemm_free(h);
     return SPG_ERR_CUDA;
   }
-  h->occ_light = light_occupancy();
+  h->occ_tile = tile_occupancy();
   h->occ_num = dtype == SPG_FP64 ? numeric_occupancy<double>() : numeric_occupancy<float>();
-  if (const char* pb = getenv("SPG_PACK_B")) h->pack_b = atoi(pb);
-  if (const char* lp = getenv("SPG_L2_PERSIST")) h->l2_persist = atoi(lp);
   for (int b = 0; b < NUM_BINS; ++b) h->occ_heavy[b] = heavy_occupancy(b);
-  h->occ_warp = warp_occupancy();
   cudaGetLastError();
   *out = h;
   return SPG_OK;
@@ -666,7 +592,7 @@ spg_status upload(spg_handle h, DevBuf& b, const void* src, size_t bytes) {
 // ===================================== ABI =====================================================
 extern "C" {
 
-const char* spg_version(void) { return "spg 0.2 (sm_100a, heavy/light-row Gustavson SpGEMM, gather-plan numeric)"; }
+const char* spg_version(void) { return "spg 0.3 (sm_100a, heavy/light-row Gustavson SpGEMM, C-order plan numeric)"; }
 
 spg_status spg_create(spg_handle* h, int device, void* cuda_stream, spg_dtype dtype) {
   return create_common(h, device, cuda_stream, dtype);
@@ -677,9 +603,10 @@ spg_status spg_spgemm_free(spg_handle h) {
   {
     DeviceGuard g(h->device);
     cudaStreamSynchronize(h->stream);
-    DevBuf* bufs[] = {&h->f,     &h->nz,    &h->cls,    &h->fl,  &h->Ro,
-                      &h->PL,    &h->tflag, &h->tiles,  &h->lists, &h->fblist, &h->small, &h->scan_tmp,
-                      &h->EQ,    &h->fl8,   &h->dup,    &h->nd,     &h->ne,   &h->chunk_row, &h->packB, &h->Pf,     &h->splits, &h->iota,  &h->ones, &h->crow_tmp};
+    DevBuf* bufs[] = {&h->f,     &h->nz,    &h->Tb,    &h->Tl,    &h->cls,    &h->pw,   &h->Ro,    &h->tflag,
+                      &h->tscan, &h->items, &h->lists, &h->small, &h->scan_tmp, &h->plan, &h->fl8, &h->D,
+                      &h->ucnt,  &h->uscan, &h->units, &h->hd,    &h->ticket, &h->Pf,     &h->splits,
+                      &h->iota,  &h->ones,  &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
     if (h->canon) spg_spgemm_free(h->canon);
@@ -735,11 +662,6 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
       h->huge_slots_opt = (int)v;
       break;
     case SPG_OPT_CONCURRENT: h->concurrent = v != 0; break;
-    case SPG_OPT_WARP_MAX_FLOPS:
-      if (v < 0 || v > WARP_MAX_CAP)
-        return setf(h, SPG_ERR_INVALID_ARGUMENT, "WARP_MAX_FLOPS must be in [0, %d]", WARP_MAX_CAP);
-      h->warp_max = (int)v;
-      break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   h->sym_ok = false;
@@ -758,7 +680,6 @@ spg_status spg_get_option(spg_handle h, spg_option opt, int64_t* v) {
     case SPG_OPT_TIMING: *v = h->timing; break;
     case SPG_OPT_HUGE_SLOTS: *v = h->huge_slots_opt; break;
     case SPG_OPT_CONCURRENT: *v = h->concurrent; break;
-    case SPG_OPT_WARP_MAX_FLOPS: *v = h->warp_max; break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   return SPG_OK;

@@ -12,40 +12,48 @@ constexpr int KEY_INF = INT_MAX;  // sentinel column (> any valid column: N <= I
 // Row classes — must match spg_row_class in include/spg.h.
 enum : int { CLS_EMPTY = 0, CLS_SINGLE, CLS_TINY, CLS_LIGHT, CLS_MEDIUM, CLS_HEAVY, CLS_HUGE, NUM_CLS };
 
-// Kernel paths ("bins").  TINY/LIGHT/MEDIUM rows all take the light (tile) kernel; HEAVY rows
-// the register-cached bitmap kernel (512 threads when f <= HEAVY1_CAP, else 1024); HUGE rows
-// (and rows the light kernel hands over) the uncached bitmap kernel.
+// Heavy-row kernel bins (k_heavy.cu): HEAVY rows are register-cached in 512-thread blocks,
+// HEAVY2 in 1024-thread blocks, HUGE rows are re-gathered per pass.
 enum : int { BIN_HEAVY = 0, BIN_HEAVY2, BIN_HUGE, NUM_BINS };
-// Row lists: the bitmap bins, then the warp-per-row rows (f <= warp_max, k_warp.cu).
-constexpr int BIN_WARP = NUM_BINS;
-constexpr int NUM_LISTS = NUM_BINS + 1;
-constexpr int WARP_MAX_CAP = 256;      // largest f of the warp-per-row symbolic kernel
-constexpr int WARP_MAX_DEFAULT = 0;  // off: measured slower than the tiles (k_warp.cu header)
 
-// Per-row path code stored in the cls[] array (low 3 bits = class, bit 3 = light path).
-constexpr uint8_t CLS_LIGHT_PATH = 8;
+// Per-row flags in the cls[] byte: low 3 bits = class, plus
+constexpr uint8_t CLS_HEAVY_PATH = 8;   // the row is its own item (bitmap symbolic, row item in numeric)
+constexpr uint8_t CLS_WIDE = 16;        // heavy row whose plan entries take two words (A row or a
+                                        // referenced B row longer than 65535 entries)
+constexpr uint8_t CLS_SOLO = 32;        // tile row that is a tile of its own (the next row starts one)
 
-// Light (tile) kernel geometry.
+// Flags k_row_flops stores next to the run count (bits 0-1) in nz[]
+constexpr uint8_t NZ_LONGB = 0x10;      // a referenced B row has more than 65535 entries
+constexpr uint8_t NZ_ALEN64K = 0x20;    // the A row has more than 65535 entries
+constexpr uint8_t NZ_ALEN512 = 0x40;    // ... more than 512 (one 512-thread bitmap gather chunk)
+constexpr uint8_t NZ_ALEN1K = 0x80;     // ... more than 1024
+
+// Tiles (k_light.cu, k_numeric.cu): runs of consecutive non-heavy rows.
 constexpr int TINY_MAX = 32;          // class boundaries for statistics only (same kernel)
 constexpr int LIGHTC_MAX = 256;
 constexpr int TILE_PMAX = 4096;       // products per tile: tile capacity + light threshold <= this
 constexpr int TILE_CAP_DEFAULT = 3072;
 constexpr int LIGHT_MAX_DEFAULT = 1024;
-constexpr int TILE_NT = 512;          // threads per tile block
-constexpr int TILE_RM = 512;          // light rows per batch
-#ifndef SPG_TILE_BK
-#define SPG_TILE_BK 2
-#endif
-constexpr int TILE_BK = SPG_TILE_BK;   // expected products per bucket
-constexpr int TILE_NBMAX = TILE_PMAX / TILE_BK + TILE_RM;  // buckets per batch (ceil per row)
+constexpr int TILE_EC = 1024;         // entries: a tile never crosses a multiple of TILE_EC in A's
+                                      // entry space, so with rows of <= TILE_EC entries it has
+                                      // < 2 * TILE_EC entries
+constexpr int TILE_RM = 256;          // rows per tile (tiles never cross a multiple of TILE_RM)
+constexpr int TILE_NT = 512;          // threads per symbolic tile block
+constexpr int TILE_BK = 2;            // expected products per bucket
+constexpr int TILE_NBMAX = TILE_PMAX / TILE_BK + TILE_RM;  // buckets per tile (ceil per row)
 // Heavy (bitmap) kernel geometry.
 constexpr int HEAVY_CAP = 8192;       // largest f of the register-cached bitmap mode (1024 threads)
-#ifndef SPG_HEAVY1_CAP
-#define SPG_HEAVY1_CAP 4096
-#endif
-constexpr int HEAVY1_CAP = SPG_HEAVY1_CAP;  // ... 512-thread blocks, two per SM
+constexpr int HEAVY1_CAP = 4096;      // ... 512-thread blocks, two per SM
 constexpr int BMP_NT = 1024;
 constexpr int BMP_NT_S = 512;
+
+// The plan (symbolic -> numeric contract).  For an item (a tile of rows, or one heavy row) with
+// plan region [P0, P0 + products) — a prefix over rows of their product counts — the first
+// c entries describe the item's outputs in C order (output P0 + o -> C offset crow_item + o) and
+// the remaining products - c entries are its repeated products ("dups"), in any order.  An entry
+// is {e_rel: A entry relative to the item's first A entry, qoff: offset within that entry's B
+// row}, packed e_rel | qoff << 16 in one word (two words, e_rel then qoff, for CLS_WIDE rows).
+__host__ __device__ __forceinline__ unsigned plan_pack(unsigned e_rel, unsigned qoff) { return e_rel | (qoff << 16); }
 
 __device__ __forceinline__ unsigned lanemask_lt() {
   unsigned m;

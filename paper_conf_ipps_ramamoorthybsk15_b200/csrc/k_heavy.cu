@@ -6,18 +6,19 @@
 // becomes a bitmap over a column tile of width Wt (TR_b of L88):
 //   pass 1  every product claims its column's bit with ATOMS.OR (on sm_100a as fast as a plain
 //           STS, tools/microbench_atomics.cu); the claimer that found the bit clear is the
-//           column's first occurrence.  A level-1 summary bit per bitmap word keeps every later
-//           step proportional to the touched words.
+//           column's head.  A level-1 summary bit per bitmap word keeps every later step
+//           proportional to the touched words.
 //   build   rank prefixes: an int per 1024 columns and a u16 per 256 columns.
 //   pass 2  rank(col) = prefix + popcount of the <= 8 bitmap words below it in its 256-column
-//           block; the first claimer writes {A entry, B entry} to the gather plan at
-//           EQ[Ro_i + rank], every other product goes to the dup list.
+//           block; the head writes its plan word {e_rel, qoff} at Ro_i + rank (C order), every
+//           other product at the end of the row's plan region (the row's dups, each with its
+//           output in D at the same word).
 //   c_i     = claimed bits (summed over column tiles).
 // HEAVY rows (f <= 8192, one gather chunk) keep their products (column) in registers across
-// the passes and their first-occurrence flags in a shared bit array; other rows (HUGE, and rows
-// the light kernel handed over) re-gather columns per pass and keep the flag in a global byte
-// per product (fl8) between pass 1 and pass 2.  Products are visited in 32-product warp windows (coalesced within
-// a B row); the run of each lane comes from a REDUX.OR mask of run starts.
+// the passes and their head flags in a shared bit array; HUGE rows re-gather columns per pass
+// and keep the flag in a global byte per product (fl8) between pass 1 and pass 2.  Products are
+// visited in 32-product warp windows (coalesced within a B row); the run of each lane comes from
+// a REDUX.OR mask of run starts.  SINGLE rows (one non-empty B row) only copy their run.
 #include "kernels.cuh"
 
 namespace spg {
@@ -25,9 +26,6 @@ namespace spg {
 constexpr int BMP_CTCAP = 2048;      // 32-product windows per chunk with a precomputed run index
 constexpr int BMP_SLOTS = 8;         // products per lane cached in registers
 constexpr int MODE_CACHED = 0, MODE_PLAIN = 1;
-#ifndef SPG_BMP_SPAN
-#define SPG_BMP_SPAN 0  // 1: cached rows tile their own column span (measured: no gain, r01)
-#endif
 
 __host__ __device__ constexpr int al16(int x) { return (x + 15) & ~15; }
 
@@ -51,7 +49,7 @@ __device__ __forceinline__ int bmp_need(int lw, int f) {
 template <int MODE, int NT, int SMEM>
 __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(SymProb P, const int* __restrict__ list,
                                                                               const int* __restrict__ count, int lwmax,
-                                                                              int N, int fallback) {
+                                                                              int N) {
   constexpr int RCAP = NT;
   constexpr bool CACHED = MODE == MODE_CACHED;
   extern __shared__ __align__(16) unsigned char sm[];
@@ -65,9 +63,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
   const Group<NT> g{(int)threadIdx.x, scratch};
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const unsigned upto = (2u << lane) - 1u;  // lanes <= me
-  // bin lists start right after k_classify and need only the heavy part of the plan to fit;
-  // the fallback list (light rows) runs after k_tiles set r_ok
-  if (fallback ? !*P.r_ok : *P.heavy_total > P.r_cap) return;
+  if (P.Ro[P.row_end - P.row_begin] > P.r_cap) return;  // plan too small: the host grows it and reruns
 
   // invariant between rows: the whole region is zero
   for (int x = tid; x < REGION / 4; x += NT) reinterpret_cast<unsigned*>(region)[x] = 0;
@@ -78,8 +74,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
   // queue in its intra-GPU form.  count[0] = rows, count[8] = queue head.
   const int n = count[0];
   __shared__ int s_next;
-  __shared__ unsigned long long s_dbase;
-  __shared__ int s_dcnt;
+  __shared__ int s_dcnt, s_single;
   for (;;) {
     if (tid == 0) s_next = atomicAdd(const_cast<int*>(count) + 8, 1);
     __syncthreads();
@@ -91,8 +86,36 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
     const int pa0 = P.rpA[i], pa1 = P.rpA[i + 1];
     const int f = P.frow[i];
     const long long ro = P.Ro[li];
-    int2* EQrow = P.EQ + ro;
+    const uint8_t rc = P.cls[li];
+    unsigned* prow = P.plan + ro;
     uint8_t* frow8 = P.fl8 + ro;
+    const bool wide = rc & CLS_WIDE;
+    // plan word(s) of output / dup position pos
+    auto put = [&](int pos, int e_rel, int qoff) {
+      if (wide) {
+        prow[2 * (long long)pos] = (unsigned)e_rel;
+        prow[2 * (long long)pos + 1] = (unsigned)qoff;
+      } else {
+        prow[pos] = plan_pack((unsigned)e_rel, (unsigned)qoff);
+      }
+    };
+    // a repeated product: plan entry from the end of the region, its output o in D at the same word
+    auto put_dup = [&](int o, int e_rel, int qoff) {
+      const int pos = f - 1 - atomicAdd(&s_dcnt, 1);
+      put(pos, e_rel, qoff);
+      P.D[ro + (wide ? 2 * (long long)pos : (long long)pos)] = (unsigned)o;
+    };
+    if (tid == 0) s_dcnt = 0;
+    if ((rc & 7) == CLS_SINGLE) {  // one non-empty B row (B canonical): output t = its entry t
+      for (int p = pa0 + tid; p < pa1; p += NT)
+        if (P.Tl[p] > 0) s_single = p - pa0;
+      __syncthreads();
+      const int er = s_single;
+      for (int t2 = tid; t2 < f; t2 += NT) put(t2, er, t2);
+      if (tid == 0) P.crow[li + 1] = f;
+      __syncthreads();
+      continue;
+    }
     // Column tile: the widest whose structures (and, cached, the flag bits) fit.
     int lw = lwmax;
     while (lw > 10 && bmp_need<MODE>(lw, f) > REGION) --lw;
@@ -115,9 +138,8 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
       const int pend = min(pa1, pa0 + (c + 1) * RCAP);
       int L = 0, bs = 0;
       if (p < pend) {
-        const int k = P.colA[p];
-        bs = P.rpB[k];
-        L = P.rpB[k + 1] - bs;
+        bs = P.Tb[p];
+        L = P.Tl[p];
       }
       const int rk = g.excl_scan(L > 0 ? 1 : 0, nz);
       const int off = g.excl_scan(L, Lt);  // f_i < 2^31 (checked in analysis)
@@ -204,35 +226,12 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
       return r;
     };
 
-#if SPG_BMP_SPAN
-    // Cached rows (one chunk): the tiles cover the row's column span [cmin, cmax] instead of
-    // [0, N) — the columns of a web-graph row are local, so one tile pass usually suffices.
-    const bool pre = CACHED && nchunks == 1;
-    if (pre) {
-      gather(0);
-      fill_cache();
-      int cmin = INT_MAX, cmax = -1;
-#pragma unroll
-      for (int s = 0; s < BMP_SLOTS; ++s)
-        if (cc[s] >= 0) {
-          cmin = min(cmin, cc[s]);
-          cmax = max(cmax, cc[s]);
-        }
-      cmin = -g.max(-cmin);
-      cmax = g.max(cmax);
-      lo0 = cmin & ~31;
-      ntiles = ((cmax - lo0) >> lw) + 1;
-    }
-#else
-    constexpr bool pre = false;
-#endif
     for (int tile = 0; tile < ntiles; ++tile) {
       const int lo = lo0 + (tile << lw);
       // ---- pass 1: claim bits; first claimers flagged -----------------------------------------
       int cbase = 0;
-      int npin = 0;  // this thread's products inside the tile
       for (int c = 0; c < nchunks; ++c) {
-        if (nchunks > 1 || (tile == 0 && !pre)) {
+        if (nchunks > 1 || tile == 0) {
           gather(c);
           if constexpr (CACHED) fill_cache();
         }
@@ -244,7 +243,6 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
             const unsigned lc = (unsigned)(cc[s] - lo);
             bool first = false;
             if (j0 + lane < Lt && lc < (unsigned)Wt) {
-              ++npin;
               const int w = lc >> 5;
               const unsigned b = 1u << (lc & 31);
               const unsigned old = atomicOr(&bm[w], b);
@@ -258,7 +256,6 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
           for_products([&](int j, int col) {
             const unsigned lc = (unsigned)(col - lo);
             if (lc < (unsigned)Wt) {
-              ++npin;
               const int w = lc >> 5;
               const unsigned b = 1u << (lc & 31);
               const unsigned old = atomicOr(&bm[w], b);
@@ -318,14 +315,6 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
         pcarry += ptot;
       }
       const int ctile = pcarry;
-      {  // dup slots of the tile: its products minus its distinct columns (one global atomic)
-        const long long ptile = ntiles == 1 ? (long long)f : g.sum((long long)npin);
-        if (tid == 0) {
-          const long long nd = ptile - ctile;
-          s_dbase = nd > 0 ? atomicAdd(P.dupn, (unsigned long long)nd) : 0ull;
-          s_dcnt = 0;
-        }
-      }
       __syncthreads();
       // ---- pass 2: ranks -> gather plan (first claimers) and dup list (the others) ---------------
       cbase = 0;
@@ -340,16 +329,12 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
               const int j = j0 + lane;
               const unsigned lc = (unsigned)(cc[s] - lo);
               const bool in = j < Lt && lc < (unsigned)Wt;
-              bool first = false;
-              int rank = 0, e = 0, q = 0;
               if (in) {
-                rank = out + rank_of(lc);
-                first = (flags[j >> 5] >> (j & 31)) & 1u;
-                q = sbs[r] + (j - seg[r]);
-                e = sae[r];
-                if (first) EQrow[rank] = make_int2(e, q);
+                const bool first = (flags[j >> 5] >> (j & 31)) & 1u;
+                const int o = out + rank_of(lc);
+                if (first) put(o, sae[r] - pa0, j - seg[r]);
+                else put_dup(o, sae[r] - pa0, j - seg[r]);
               }
-              dup_push(P, in && !first, li, rank, e, q, s_dbase, &s_dcnt);
             }
           }
         } else {
@@ -362,27 +347,22 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
               rr[u] = 0;
               if (j0 < Lt) {
                 rr[u] = lane_run(j0);
-                if (j0 + lane < Lt) q[u] = sbs[rr[u]] + (j0 + lane - seg[rr[u]]);
+                if (j0 + lane < Lt) q[u] = j0 + lane - seg[rr[u]];
               }
             }
             uint8_t fb[BATCH];
 #pragma unroll
             for (int u = 0; u < BATCH; ++u) {
-              col[u] = q[u] >= 0 ? P.colB[q[u]] : -1;
+              col[u] = q[u] >= 0 ? P.colB[sbs[rr[u]] + q[u]] : -1;
               fb[u] = q[u] >= 0 ? frow8[cbase + j00 + u * NT + lane] : 0;
             }
 #pragma unroll
             for (int u = 0; u < BATCH; ++u) {
-              if (j00 + u * NT < Lt) {  // warp-uniform
-                const unsigned lc = (unsigned)(col[u] - lo);
-                const bool in = q[u] >= 0 && lc < (unsigned)Wt;
-                int rank = 0;
-                const int e = sae[rr[u]];
-                if (in) {
-                  rank = out + rank_of(lc);
-                  if (fb[u]) EQrow[rank] = make_int2(e, q[u]);
-                }
-                dup_push(P, in && !fb[u], li, rank, e, q[u], s_dbase, &s_dcnt);
+              const unsigned lc = (unsigned)(col[u] - lo);
+              if (q[u] >= 0 && lc < (unsigned)Wt) {
+                const int o = out + rank_of(lc);
+                if (fb[u]) put(o, sae[rr[u]] - pa0, q[u]);
+                else put_dup(o, sae[rr[u]] - pa0, q[u]);
               }
             }
           }
@@ -409,7 +389,10 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
         for (int x = tid; x < nfw; x += NT) flags[x] = 0;
       __syncthreads();
     }
-    if (tid == 0) P.crow[li + 1] = out;
+    if (tid == 0) {
+      P.crow[li + 1] = out;
+      if (f > out) atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)(f - out));
+    }
   }
 }
 
@@ -440,11 +423,11 @@ int heavy_occupancy(int bin) {
 }
 
 cudaError_t launch_heavy_rank(int bin, cudaStream_t st, int grid, const SymProb& P, const int* list,
-                              const int* count, long long N, int fallback) {
+                              const int* count, long long N) {
   int lwmax = 10;
   while (lwmax < 20 && ((long long)1 << lwmax) < N) ++lwmax;
   int n32 = (int)N;
-  void* args[] = {(void*)&P, (void*)&list, (void*)&count, (void*)&lwmax, (void*)&n32, (void*)&fallback};
+  void* args[] = {(void*)&P, (void*)&list, (void*)&count, (void*)&lwmax, (void*)&n32};
   return cudaLaunchKernel(bitmap_kernel(bin), dim3(grid), dim3(bitmap_threads(bin)), args, bitmap_smem(bin), st);
 }
 

@@ -1,132 +1,117 @@
 // kernels.cuh — declarations shared by the kernel translation units and the C-ABI layer.
 //
 // Pipeline:
-//   analysis   k_row_flops: f_i, run flags, log2 histogram
-//   classify   k_classify: row path (light tile kernel / heavy bitmap kernel / identity copy),
-//              heavy row lists and their plan (EQ) offsets; scan of light flops -> PL; k_tiles:
-//              tile cut points in light-product space, plan offsets of light rows
-//   symbolic   k_light_rank (tiles of light rows) and k_bitmap_rank (heavy rows) sort every row's
-//              products by column and emit the gather plan: for the first product of each
-//              distinct column of row i, EQ[Ro_i + rank] = {A entry, B entry}; every other
-//              product goes to the dup list.  c_i = #distinct.
-//   plan       k_plan: per-row EQ-to-C offset (or the SINGLE row's run), chunk -> first row
-//   numeric    k_numeric: C in chunks of NUM_CH outputs, one coalesced pass — C(i, r) =
-//              valA[e]·valB[q] from EQ (Phase IV of PAPER.md L154-156: the sort moved to the
-//              symbolic phase, so numeric re-runs are a stream); k_numeric_dup adds the dup list.
+//   analysis   k_row_flops: f_i, run count and size flags per row, log2 histogram
+//   classify   k_classify: heavy rows (f_i > light_max, or long A rows) go to a bitmap bin list;
+//              every other row belongs to a tile; plan words per row (scanned into Ro)
+//   items      k_tile_flags + scan + k_items: the ordered list of items — a heavy row, or a tile
+//              of consecutive non-heavy rows (<= TILE_RM rows, < TILE_PMAX products,
+//              < 2 TILE_EC A entries)
+//   symbolic   k_tile_rank (tiles) and k_bitmap_rank (heavy rows) sort every item's products by
+//              (row, column), count c_i and write the plan: the item's outputs in C order as
+//              {A entry, B offset} words, then its repeated products (dups)
+//   units      k_unit_count + scan + k_unit_fill: numeric work units — segments of an item's
+//              outputs
+//   numeric    k_numeric: persistent warps take units from a queue — C(i, j) = valA[e]·valB[q]
+//              streamed in C order (coalesced plan read, coalesced C write; A/B from L2); then,
+//              once every unit of the item has stored, a share of the item's repeated products
+//              is added with RED (Phase IV of PAPER.md L154-156: the sort moved to symbolic, so
+//              numeric re-runs on new values are a stream)
 #pragma once
 #include "common.cuh"
 
 namespace spg {
 
 struct ClassParams {
-  int light_max;   // f <= light_max -> light (tile) kernel
-  int heavy_max;   // f <= heavy_max -> register-cached bitmap kernel, else HUGE (uncached)
+  int light_max;   // f <= light_max -> tile path
+  int heavy_max;   // heavy rows with f <= heavy_max -> register-cached bitmap kernel, else HUGE
   int tile_cap;    // nominal products per tile; rows above TILE_PMAX - tile_cap are solo tiles
   int force;       // -1 or a class id >= CLS_TINY
-  int single_ok;   // B rows canonical -> SINGLE (identity) shortcut allowed
-  int warp_max;    // light rows with f <= warp_max -> warp-per-row kernel (0: none)
+  int single_ok;   // B rows canonical -> SINGLE (copy) shortcut allowed
 };
 
 struct HeavyLists {
-  int* rows[NUM_LISTS];
+  int* rows[NUM_BINS];
 };
 
 // Small per-call device scratch (zeroed at the start of every symbolic call).
 struct Small {
   int counts[8];            // per bitmap bin: rows
   int qhead[8];             // per bitmap bin: dynamic row-queue heads (counts + 8)
-  int fb[16];               // fallback rows from the light kernel: [0] rows, [8] queue head
-  int ntiles;
+  int nitems;               // items (tiles + heavy rows)
   int err;
-  int r_ok;                 // EQ capacity sufficient (written by k_tiles)
   int amax;                 // longest row of A
-  int nch_need;             // numeric chunks (+1) the plan needed
-  int tqhead;               // light tiles: dynamic queue head
-  unsigned long long dupn;  // non-first products (dup list entries)
-  long long heavy_total;    // products of heavy rows (EQ offsets of heavy rows, relative)
-  long long fr;             // products of rows with a gather plan (light + heavy)
+  int tqhead;               // tiles: dynamic queue head
+  long long dups;           // repeated products (statistics)
+  long long nunits;         // numeric work units
   unsigned long long hist[65];
   unsigned long long cstats[2 * NUM_CLS + 2];
 };
 
 // Problem view passed to the symbolic kernels.  Row indices in lists / cls / Ro / crow are
 // local (i - row_begin).
-//
-// Gather plan (the symbolic phase's output, consumed by numeric): row i's distinct columns, in
-// ascending order, are described by EQ[Ro_i + r] = {A entry e, B entry q} of the first product
-// (in the kernel's visiting order) that produced the column of rank r; every other product of
-// the column is a dup entry {li, r, e, q}.  Numeric is then C(i, r) = valA[e]·valB[q] (+ dups):
-// a coalesced stream in output order (Phase IV's "sort, mark, add like-tuples, compact" of
-// PAPER.md L154-156 with the sort moved to symbolic, so numeric re-runs on new values are cheap).
 struct SymProb {
   const int* __restrict__ rpA;
   const int* __restrict__ colA;
   const int* __restrict__ rpB;
   const int* __restrict__ colB;
+  const int* __restrict__ Tb;   // per A entry: start of its B row (rpB[colA[e]])
+  const int* __restrict__ Tl;   // per A entry: length of its B row
   const int* frow;          // f_i (global row index)
-  const uint8_t* cls;       // path per local row
-  const long long* Ro;      // EQ offset per local row (-1: no plan: empty / SINGLE)
-  int2* EQ;                 // gather plan, indexed Ro_i + rank
-  int4* dup;                // dup list
-  unsigned long long* dupn; // its length (may exceed dupcap: then the host grows it and reruns)
-  long long dupcap;
+  const uint8_t* cls;       // class and path flags per local row
+  const long long* Ro;      // plan word offset per local row (exclusive prefix, [Mloc + 1])
+  unsigned* plan;           // the plan (capacity r_cap words)
   uint8_t* fl8;             // uncached bitmap rows: first-claim flag per product (Ro_i + offset)
   long long* crow;          // C row offsets (local); symbolic writes counts at [li + 1]
-  const int* r_ok;
-  const long long* heavy_total;  // heavy rows' plan size (final after k_classify)
-  long long r_cap;               // plan capacity (entries)
+  unsigned* D;              // item-relative output of the repeated product whose plan entry starts
+                            // at the same word (sized like the plan, written only for repeats)
+  long long* dups;          // repeated-product counter (statistics)
+  long long r_cap;          // plan capacity (words); the kernels do nothing if Ro[Mloc] > r_cap
   int row_begin, row_end;
-  int lgN;                  // ceil(log2 N), N = columns of B
 };
 
-// Append a non-first product to the dup list (all 32 lanes must call).  The caller reserved the
-// slots [base, base + n) of its row / tile / batch with one global atomic (the count is known before
-// the ranks are written: products - distinct columns); *s_cnt (shared) hands them out per warp.
-__device__ __forceinline__ void dup_push(const SymProb& P, bool d, int li, int rank, int e, int q,
-                                         unsigned long long base, int* s_cnt) {
-  const unsigned m = __ballot_sync(FULL, d);
-  if (!m) return;
-  const int lane = threadIdx.x & 31, leader = __ffs(m) - 1;
-  int o = 0;
-  if (lane == leader) o = atomicAdd(s_cnt, __popc(m));
-  const unsigned long long b = base + (unsigned long long)(__shfl_sync(FULL, o, leader) + __popc(m & lanemask_lt()));
-  if (d && (long long)b < P.dupcap) P.dup[b] = make_int4(li, rank, e, q);
-}
+// Numeric work units: item t has hs_t = ceil(c_t / NUM_SH) units; unit {t, k} stores outputs
+// [k NUM_SH, (k + 1) NUM_SH) of the item, then adds the k-th of hs_t equal shares of its
+// repeated products (d_t = f_t - c_t) once all hs_t units have stored.
+constexpr int NUM_SH = 1024;
 
-// Numeric phase: chunks of NUM_CH consecutive outputs of C (one block each).
-constexpr int NUM_CH = 2048;
-constexpr int NUM_NT = 256;
-
+// Numeric phase.
 template <typename V>
 struct NumProb {
+  const int* __restrict__ rpA;
   const V* __restrict__ valA;
+  const int* __restrict__ Tb;           // per A entry: start of its B row
   const int* __restrict__ colB;
   const V* __restrict__ valB;
-  const int2* __restrict__ EQ;
-  const int4* __restrict__ dup;
+  const unsigned* __restrict__ plan;
+  const long long* __restrict__ Ro;
   const long long* __restrict__ crow;   // C row offsets (local)
-  const long long* __restrict__ nd;     // per local row: EQ index (or B index, SINGLE) minus C offset
-  const int* __restrict__ ne;           // per local row: -1, or the A entry of a SINGLE row
-  const int* __restrict__ chunk_row;    // row holding the first output of each chunk
-  long long nnz;                        // outputs (this rank)
-  long long ndup;
-  void* packB;                          // optional packed {column, value} copy of B (one gather)
-  long long nB;
-  int nch;
-  int mloc;
+  const uint8_t* __restrict__ cls;
+  const int* __restrict__ items;        // ordered item starts (local rows) + sentinel
+  const int2* __restrict__ units;
+  const long long* __restrict__ nunits;
+  const unsigned* __restrict__ D;
+  int* hd;                              // per item: finished output segments (all calls)
+  int* ticket;                          // work-unit queue head (zeroed before the launch)
+  int epoch;                            // numeric calls since symbolic (1, 2, ...)
+  int row_begin;
   int* ccol;
   V* cval;
 };
 
 // analysis.cu
 cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB, int* f,
-                             uint8_t* nz, unsigned long long* hist, int* err, int* amax);
+                             uint8_t* nz, int* Tb, int* Tl, unsigned long long* hist, int* err, int* amax);
+cudaError_t launch_unit_count(cudaStream_t st, int sms, const int* items, const long long* crow, const long long* Ro,
+                              const uint8_t* cls, int mloc, int* ucnt, int* hd);
+cudaError_t launch_unit_fill(cudaStream_t st, int sms, const int* ucnt, const long long* uscan, int mloc,
+                             int2* units, Small* small, const int* items, const long long* crow);
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
-                            const ClassParams& prm, uint8_t* cls, int* fl, long long* Ro, const HeavyLists& lists,
-                            Small* small, long long* crow, long long* PL);
-cudaError_t launch_tiles(cudaStream_t st, int sms, const int* f, int rb, int re, int tile_cap, const uint8_t* cls,
-                         const long long* PL, long long* Ro, uint8_t* tflag, int* tiles, Small* small,
-                         long long r_cap);
+                            const ClassParams& prm, uint8_t* cls, int* pw, const HeavyLists& lists, Small* small);
+cudaError_t launch_tile_flags(cudaStream_t st, int sms, const int* f, const int* rpA, int rb, int re, int tile_cap,
+                              const uint8_t* cls, const long long* Ro, int* tflag);
+cudaError_t launch_items(cudaStream_t st, int sms, const int* tflag, const long long* tscan, int mloc, int* items,
+                         Small* small);
 cudaError_t launch_sort_list(cudaStream_t st, const HeavyLists& lists, int bin, const int* f, int rb,
                              const Small* small);
 size_t scan_tmp_elems(long long n);
@@ -142,28 +127,19 @@ template <typename V>
 cudaError_t launch_fill(cudaStream_t st, V* p, long long n, V v);
 cudaError_t launch_narrow(cudaStream_t st, const long long* in, int* out, long long n);
 
-// k_light.cu — symbolic ranks of the light rows, one tile per block iteration.
-cudaError_t light_configure();
-int light_occupancy();
-cudaError_t launch_light_rank(cudaStream_t st, int grid, const SymProb& P, const int* tiles, const int* ntiles, int* tqhead,
-                              const uint8_t* tflag, const long long* PL, int* fb_list, int* fb_count);
+// k_light.cu — symbolic sort of the tiles, one tile per block iteration.
+cudaError_t tile_configure();
+int tile_occupancy();
+cudaError_t launch_tile_rank(cudaStream_t st, int grid, const SymProb& P, const int* items, const int* nitems,
+                             int* tqhead);
 
-// k_warp.cu — symbolic plan of the smallest light rows, one warp per row.
-int warp_occupancy();
-cudaError_t launch_warp_rank(cudaStream_t st, int grid, const SymProb& P, const int* list, const int* count);
-
-// k_heavy.cu — symbolic ranks of heavy rows (column bitmap), per bin or over an explicit list.
+// k_heavy.cu — symbolic sort of the heavy rows (column bitmap), one row per block iteration.
 cudaError_t heavy_configure();
 int heavy_occupancy(int bin);
 cudaError_t launch_heavy_rank(int bin, cudaStream_t st, int grid, const SymProb& P, const int* list,
-                              const int* count, long long N, int fallback);
+                              const int* count, long long N);
 
-// k_numeric.cu — numeric plan (end of symbolic) and numeric phase.
-cudaError_t launch_plan(cudaStream_t st, int sms, const long long* crow, int mloc, const int* rpA, const int* colA,
-                        const int* rpB, const uint8_t* cls, const long long* Ro, int rb, long long* nd, int* ne,
-                        int* chunk_row, int chcap, Small* small);
-template <typename V>
-cudaError_t numeric_configure();
+// k_numeric.cu — numeric phase.
 template <typename V>
 int numeric_occupancy();
 template <typename V>

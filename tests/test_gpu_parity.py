@@ -81,14 +81,6 @@ def test_thresholds_do_not_change_result(heavy_max, tile, light_max):
     compare(A, B, got, ref=ref)
 
 
-@pytest.mark.parametrize("warp_max", [0, 1, 32, 33, 64, 100, 128, 256])
-def test_warp_rows_threshold(warp_max):
-    """k_warp.cu (one warp per light row, f <= warp_max) against the oracle; every register-sort
-    width (1, 2, 4, 8 keys per lane) and the boundaries between them; 0 = all light rows in tiles."""
-    A, B = W.make("cl10k")
-    compare(A, B, run_gpu(A, B, warp_max_flops=warp_max))
-
-
 def test_fp32_power_law():
     A = W.chung_lu(20000, 20000, 2.1, 80000, 3000, 3000, 6.0, 1.1, 5, np.float32)
     B = W.chung_lu(20000, 20000, 3.0, 160000, 1000, 1000, -1.0, 1.0, 6, np.float32)

@@ -227,27 +227,129 @@ __global__ void __launch_bounds__(256) k_items(const int* __restrict__ tflag, co
   }
 }
 
-// Numeric work units per item t (unit counts ucnt[t]; hd[t] = 0: no output unit done yet).
+// Numeric work units per item t: ceil(c_t / NUM_SH).
 __global__ void __launch_bounds__(256) k_unit_count(const int* __restrict__ items, const long long* __restrict__ crow,
-                                                    const long long* __restrict__ Ro, const uint8_t* __restrict__ cls,
-                                                    int n, int* __restrict__ ucnt, int* __restrict__ hd) {
-  for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < n; t += (long long)gridDim.x * blockDim.x) {
-    const int r = items[t], r2 = items[t + 1];
-    const long long c = crow[r2] - crow[r];
-    ucnt[t] = (int)((c + NUM_SH - 1) / NUM_SH);
-    hd[t] = 0;
-  }
+                                                    int n, int* __restrict__ ucnt) {
+  for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < n; t += (long long)gridDim.x * blockDim.x)
+    ucnt[t] = (int)((crow[items[t + 1]] - crow[items[t]] + NUM_SH - 1) / NUM_SH);
 }
 
 __global__ void __launch_bounds__(256) k_unit_fill(const int* __restrict__ ucnt, const long long* __restrict__ uscan,
-                                                   int n, int2* __restrict__ units, Small* __restrict__ sm,
-                                                   const int* __restrict__ items, const long long* __restrict__ crow) {
+                                                   int n, NumUnit* __restrict__ units, Small* __restrict__ sm,
+                                                   const int* __restrict__ items, const long long* __restrict__ crow,
+                                                   const long long* __restrict__ Ro, const uint8_t* __restrict__ cls,
+                                                   const int* __restrict__ rpA, int rb, const int* __restrict__ dub) {
   for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < n; t += (long long)gridDim.x * blockDim.x) {
     const int u = ucnt[t];
     const long long b = uscan[t] - u;
-    for (int k = 0; k < u; ++k) units[b + k] = make_int2((int)t, k);
+    const int r = items[t], r2 = items[t + 1];
+    const long long o0 = crow[r], c = crow[r2] - o0, P0 = Ro[r];
+    const bool wide = (cls[r] & CLS_HEAVY_PATH) && (cls[r] & CLS_WIDE);
+    const int sw = wide ? 2 : 1;
+    const long long f = (Ro[r2] - P0) / sw;
+    const int e0 = rpA[rb + r];
+    const int* db = dub + dub_index(P0, t);
+    const bool sorted = (cls[r] & CLS_HEAVY_PATH) && f > c && db[0] >= 0;  // heavy rows: k_dup_sort
+    for (int k = 0; k < u; ++k) {
+      NumUnit v;
+      v.pw = P0 + (long long)k * NUM_SH * sw;
+      v.oc = o0 + (long long)k * NUM_SH;
+      v.dw = P0 + (c + (sorted ? db[k] : 0)) * sw;
+      v.d = sorted ? db[k + 1] - db[k] : (int)(f - c);
+      v.n = (int)min((long long)NUM_SH, c - (long long)k * NUM_SH);
+      v.e0 = e0;
+      v.ob = k * NUM_SH | (wide ? UNIT_WIDE : 0);
+      units[b + k] = v;
+    }
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) sm->nunits = n > 0 ? uscan[n - 1] : 0;
+}
+
+// Repeats of a heavy row bucketed by numeric unit (counting sort on o / NUM_SH): one block per
+// heavy row, a scratch copy of the (word, output) pairs, then written back in bucket order.
+// dub[dub_index(P0, t) + k] = first repeat of unit k (relative to the row's repeats), k <= hs;
+// dub[...] = -1: not sorted (no repeats, a wide row, more than DUP_SORT_UNITS units, or so few
+// units and repeats that filtering is cheaper).
+constexpr int DS_NT = 512;
+__global__ void __launch_bounds__(DS_NT) k_dup_sort(HeavyLists lists, int c0, int c1, int c2,
+                                                    const long long* __restrict__ crow,
+                                                    const long long* __restrict__ Ro, const uint8_t* __restrict__ cls,
+                                                    const long long* __restrict__ tscan, unsigned* __restrict__ plan,
+                                                    unsigned* __restrict__ D, uint2* __restrict__ scratch,
+                                                    unsigned long long* __restrict__ scratch_head,
+                                                    int* __restrict__ dub) {
+  __shared__ int s_cnt[DUP_SORT_UNITS + 1];
+  __shared__ int scratch_s[DS_NT / 32 + 1];
+  __shared__ unsigned long long s_base;
+  const Group<DS_NT> g{(int)threadIdx.x, scratch_s};
+  const int tid = threadIdx.x;
+  int b = blockIdx.x, bin = 0;
+  const int cnts[3] = {c0, c1, c2};
+  while (b >= cnts[bin]) b -= cnts[bin++];
+  const int li = lists.rows[bin][b];
+  const long long t = tscan[li] - 1;
+  const long long o0 = crow[li], c = crow[li + 1] - o0, P0 = Ro[li];
+  int* db = dub + dub_index(P0, t);
+  const bool wide = cls[li] & CLS_WIDE;
+  const long long f = (Ro[li + 1] - P0) >> (wide ? 1 : 0);
+  const long long d = f - c;
+  const long long hs = (c + NUM_SH - 1) / NUM_SH;
+  // (few units x few repeats: numeric filters the unsorted list more cheaply than this sorts it)
+  if (d <= 0 || wide || hs > DUP_SORT_UNITS || hs * d <= 8192) {
+    if (tid == 0) db[0] = -1;
+    return;
+  }
+  for (int k = tid; k <= hs; k += DS_NT) s_cnt[k] = 0;
+  __syncthreads();
+  const long long w0 = P0 + c;  // first repeat's word
+  for (long long j = tid; j < d; j += DS_NT) atomicAdd(&s_cnt[D[w0 + j] / NUM_SH], 1);
+  __syncthreads();
+  {  // exclusive scan of the bucket sizes (contiguous ownership)
+    const int per = (int)((hs + DS_NT) / DS_NT);
+    int mine = 0;
+    for (int x = 0; x < per; ++x) {
+      const long long k = (long long)tid * per + x;
+      if (k < hs) mine += s_cnt[k];
+    }
+    int tot;
+    int run = g.excl_scan(mine, tot);
+    for (int x = 0; x < per; ++x) {
+      const long long k = (long long)tid * per + x;
+      if (k < hs) {
+        const int v = s_cnt[k];
+        s_cnt[k] = run;
+        db[k] = run;
+        run += v;
+      }
+    }
+    if (tid == 0) {
+      db[hs] = tot;
+      s_base = atomicAdd(scratch_head, (unsigned long long)d);
+    }
+  }
+  __syncthreads();
+  uint2* tmp = scratch + s_base;
+  for (long long j = tid; j < d; j += DS_NT) {
+    const unsigned o = D[w0 + j];
+    const int pos = atomicAdd(&s_cnt[o / NUM_SH], 1);
+    tmp[pos] = make_uint2(plan[w0 + j], o);
+  }
+  __syncthreads();
+  for (long long j = tid; j < d; j += DS_NT) {
+    const uint2 x = tmp[j];
+    plan[w0 + j] = x.x;
+    D[w0 + j] = x.y;
+  }
+}
+
+cudaError_t launch_dup_sort(cudaStream_t st, const HeavyLists& lists, const int* counts_host, const long long* crow,
+                            const long long* Ro, const uint8_t* cls, const long long* tscan, unsigned* plan,
+                            unsigned* D, uint2* scratch, unsigned long long* scratch_head, int* dub) {
+  const long long n = (long long)counts_host[0] + counts_host[1] + counts_host[2];
+  if (n <= 0) return cudaSuccess;
+  k_dup_sort<<<(unsigned)n, DS_NT, 0, st>>>(lists, counts_host[0], counts_host[1], counts_host[2], crow, Ro, cls, tscan,
+                                           plan, D, scratch, scratch_head, dub);
+  return cudaGetLastError();
 }
 
 // ---- inclusive scan to int64 (three passes: tile scan, tile-sum scan, add) -------------------
@@ -416,16 +518,17 @@ cudaError_t launch_tile_flags(cudaStream_t st, int sms, const int* f, const int*
   return cudaGetLastError();
 }
 
-cudaError_t launch_unit_count(cudaStream_t st, int sms, const int* items, const long long* crow, const long long* Ro,
-                              const uint8_t* cls, int n, int* ucnt, int* hd) {
+cudaError_t launch_unit_count(cudaStream_t st, int sms, const int* items, const long long* crow, int n, int* ucnt) {
   if (n <= 0) return cudaSuccess;
-  k_unit_count<<<grid_for_rows(n, sms), 256, 0, st>>>(items, crow, Ro, cls, n, ucnt, hd);
+  k_unit_count<<<grid_for_rows(n, sms), 256, 0, st>>>(items, crow, n, ucnt);
   return cudaGetLastError();
 }
 
-cudaError_t launch_unit_fill(cudaStream_t st, int sms, const int* ucnt, const long long* uscan, int n, int2* units,
-                             Small* small, const int* items, const long long* crow) {
-  k_unit_fill<<<grid_for_rows(n, sms), 256, 0, st>>>(ucnt, uscan, n, units, small, items, crow);
+cudaError_t launch_unit_fill(cudaStream_t st, int sms, const int* ucnt, const long long* uscan, int n,
+                             NumUnit* units, Small* small, const int* items, const long long* crow,
+                             const long long* Ro, const uint8_t* cls, const int* rpA, int rb, const int* dub) {
+  k_unit_fill<<<grid_for_rows(n, sms), 256, 0, st>>>(ucnt, uscan, n, units, small, items, crow, Ro, cls, rpA, rb,
+                                                     dub);
   return cudaGetLastError();
 }
 

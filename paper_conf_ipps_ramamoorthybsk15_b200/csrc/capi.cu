@@ -82,7 +82,7 @@ struct spg_ctx {
   int thresholds_set = 0;  // light_max / tile_cap set by the caller (else N-dependent defaults)
   // workspace: analysis (all rows), classification and items (this rank's rows), the plan
   DevBuf f, nz, Tb, Tl, cls, pw, Ro, tflag, tscan, items, lists, small, scan_tmp, plan, fl8, D, ucnt, uscan,
-      units, hd, ticket, Pf, splits, canonB[4], iota, ones, crow_tmp;
+      units, ticket, dub, dscratch, Pf, splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
   long long iota_n = -1, ones_n = -1;
@@ -92,7 +92,6 @@ struct spg_ctx {
   cudaEvent_t ev_t[8] = {};
   cudaEvent_t ev_p[4] = {};  // tile path start/end, heavy path start/end
   int occ_tile = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1;
-  int epoch = 0;  // numeric calls since the last symbolic
   // cached symbolic state
   bool sym_ok = false;
   SymKey key{};
@@ -252,7 +251,6 @@ spg_status ensure_ws(spg_handle h, int M, long long nnzA) {
   CK(h->Tl.ensure(na * sizeof(int)));
   CK(h->ucnt.ensure((m + 1) * sizeof(int)));
   CK(h->uscan.ensure((m + 1) * sizeof(long long)));
-  CK(h->hd.ensure((m + 1) * sizeof(int)));
   CK(h->ticket.ensure(sizeof(int)));
   CK(h->f.ensure(m * sizeof(int)));
   CK(h->nz.ensure(m));
@@ -443,17 +441,32 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   const Small& hs = h->hr->small;
   h->nnzC = h->hr->nnz;
   h->nitems = hs.nitems;
-  {  // numeric work units (structure only: built once, reused by every numeric call)
+  {  // repeats of heavy rows bucketed by numeric unit, then the numeric work units (structure
+     // only: built once, reused by every numeric call)
+    const Small* dsm = h->small.as<Small>();
+    CK(h->dub.ensure((size_t)(h->plan_words / NUM_SH + 2LL * hs.nitems + 4) * sizeof(int)));
+    CK(h->dscratch.ensure((size_t)(hs.dups + 1) * sizeof(uint2)));
+    CK(cudaMemsetAsync(&ds->scratch_head, 0, sizeof(unsigned long long), h->stream));
+    HeavyLists HL;
+    int hc[NUM_BINS];
+    for (int b = 0; b < NUM_BINS; ++b) {
+      HL.rows[b] = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
+      hc[b] = hs.counts[b];
+    }
+    CK(launch_dup_sort(h->stream, HL, hc, crow, h->Ro.as<long long>(), h->cls.as<uint8_t>(), h->tscan.as<long long>(),
+                       h->plan.as<unsigned>(), h->D.as<unsigned>(), h->dscratch.as<uint2>(), &ds->scratch_head,
+                       h->dub.as<int>()));
+    h->launches += 2;
+    (void)dsm;
     const long long ucap = (long long)hs.nitems + h->nnzC / NUM_SH + 2;
-    CK(h->units.ensure((size_t)ucap * sizeof(int2)));
+    CK(h->units.ensure((size_t)ucap * sizeof(NumUnit)));
     const int n = hs.nitems;
-    CK(launch_unit_count(h->stream, h->sms, h->items.as<int>(), crow, h->Ro.as<long long>(), h->cls.as<uint8_t>(), n,
-                         h->ucnt.as<int>(), h->hd.as<int>()));
+    CK(launch_unit_count(h->stream, h->sms, h->items.as<int>(), crow, n, h->ucnt.as<int>()));
     CK(launch_incl_scan<int>(h->stream, h->ucnt.as<int>(), h->uscan.as<long long>(), n, h->scan_tmp.as<long long>()));
-    CK(launch_unit_fill(h->stream, h->sms, h->ucnt.as<int>(), h->uscan.as<long long>(), n, h->units.as<int2>(), ds,
-                        h->items.as<int>(), crow));
+    CK(launch_unit_fill(h->stream, h->sms, h->ucnt.as<int>(), h->uscan.as<long long>(), n, h->units.as<NumUnit>(), ds,
+                        h->items.as<int>(), crow, h->Ro.as<long long>(), h->cls.as<uint8_t>(), A->row_ptr, h->rb,
+                        h->dub.as<int>()));
     h->launches += 2 + scan_launches(n);
-    h->epoch = 0;
   }
   for (int b = 0; b < NUM_BINS; ++b) h->counts[b] = hs.counts[b];
   spg_stats& st = h->stats;
@@ -511,12 +524,10 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
     P.crow = reinterpret_cast<const long long*>(C_row_ptr);
     P.cls = h->cls.as<uint8_t>();
     P.items = h->items.as<int>();
-    P.units = h->units.as<int2>();
+    P.units = h->units.as<NumUnit>();
     P.nunits = &h->small.as<Small>()->nunits;
     P.D = h->D.as<unsigned>();
-    P.hd = h->hd.as<int>();
     P.ticket = h->ticket.as<int>();
-    P.epoch = ++h->epoch;
     P.row_begin = h->rb;
     P.ccol = C_col;
     P.cval = (V*)C_val;
@@ -605,7 +616,7 @@ spg_status spg_spgemm_free(spg_handle h) {
     cudaStreamSynchronize(h->stream);
     DevBuf* bufs[] = {&h->f,     &h->nz,    &h->Tb,    &h->Tl,    &h->cls,    &h->pw,   &h->Ro,    &h->tflag,
                       &h->tscan, &h->items, &h->lists, &h->small, &h->scan_tmp, &h->plan, &h->fl8, &h->D,
-                      &h->ucnt,  &h->uscan, &h->units, &h->hd,    &h->ticket, &h->Pf,     &h->splits,
+                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->dscratch, &h->Pf,     &h->splits,
                       &h->iota,  &h->ones,  &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();

@@ -4,89 +4,131 @@
 // The symbolic phase sorted every item's products by (row, column) and left the plan: for an
 // item (a tile of consecutive rows, or one heavy row) with plan region [P0, P0 + f) and outputs
 // [o0, o0 + c), plan word P0 + o describes output o0 + o — {e_rel, qoff}: the A entry e0 + e_rel
-// and the offset of the B entry inside that entry's B row — and the words from the end of the
-// region backwards are the item's repeated products (dups), each with its output in D at the
-// same word.
+// and the offset of the B entry inside that entry's B row — and words c..f-1 of the region are
+// the item's repeated products (dups), each with its item-relative output in D at the same word.
 //
 // So numeric is a stream in C order (Phase IV of PAPER.md L154-156, "add like-tuples and
 // compact", with the sort done once in symbolic).  Persistent warps take work units (NUM_SH
-// consecutive outputs of one item) from a queue built in item order at the end of symbolic:
-//   outputs   per output one coalesced plan word, the A entry's B-row start Tb[e] and value
+// consecutive outputs of one item) from a queue built in item order at the end of symbolic;
+// while a unit is processed, one lane has already put the next unit's plan words in flight into
+// the warp's other shared-memory buffer with a TMA bulk copy (cp.async.bulk + mbarrier), so the
+// plan stream from HBM is never on the dependent path:
+//   outputs   per output one plan word (shared memory), the A entry's B-row start Tb[e] and value
 //             valA[e] (the item's A entries: L1), the B gather (column and value, L2: B rows are
-//             consumed in ascending order), one multiply, two coalesced streaming stores; then
-//             hd[t] += 1 (release).
-//   repeats   the unit's share of the item's repeated products waits (relaxed polling, no L1
-//             invalidation) until hd[t] says every unit of the item has stored — they were
-//             dequeued no later than the item's last unit, so they are running or done — then
-//             adds a·b into its output with RED.ADD.F64/F32 (the lines are still in L2).
+//             consumed in ascending order), one multiply, two coalesced streaming stores.
+//   repeats   the unit scans the item's dup outputs in D (a few KB, L1/L2) and adds a·b for those
+//             inside its own outputs with RED.ADD.F64/F32 — into lines it just wrote (L2), ordered
+//             after its stores by __syncwarp; no unit ever waits for another.
 // HBM traffic per output: 4 B of plan read + (4 + sizeof(V)) B of C written; A and B once.
 #include "kernels.cuh"
 
 namespace spg {
 
-constexpr int NUM_NT = 256;            // threads per block (8 independent warps)
+constexpr int NUM_NT = 128;            // threads per block: 4 independent warps
+constexpr int NUM_W = NUM_NT / 32;
 constexpr int NUM_U = 4;               // outputs per lane in flight
+constexpr int NUM_BUFW = NUM_SH + 8;   // plan words per staging buffer (16-byte alignment slack)
 
 __device__ __forceinline__ void st_cs(int* p, int v) { __stcs(p, v); }
 __device__ __forceinline__ void st_cs(double* p, double v) { __stcs(p, v); }
 __device__ __forceinline__ void st_cs(float* p, float v) { __stcs(p, v); }
 
-// Release increment: MEMBAR + RED (no L1 invalidation, unlike __threadfence()).
-__device__ __forceinline__ void red_release(int* p, int v) {
-  asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+
+// ---- TMA (cp.async.bulk) staging of a unit's plan words with an mbarrier ------------------------
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long* bar) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
 }
-__device__ __forceinline__ int ld_relaxed(const int* p) {
-  int v;
-  asm volatile("ld.relaxed.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
+__device__ __forceinline__ void tma_plan(unsigned* dst, const unsigned* src, unsigned bytes, unsigned long long* bar) {
+  asm volatile(
+      "fence.proxy.async.shared::cta;\n\t"  // earlier generic reads of dst before the async write
+      "mbarrier.arrive.expect_tx.shared::cta.b64 _, [%3], %2;\n\t"
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned phase) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(phase)
+      : "memory");
 }
 
 template <typename V>
 __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
-  const int lane = threadIdx.x & 31;
+  __shared__ __align__(16) unsigned s_buf[NUM_W][2][NUM_BUFW];
+  __shared__ __align__(8) unsigned long long s_bar[NUM_W][2];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const long long nunits = *P.nunits;
-  for (;;) {
+  if (lane == 0) {
+    mbar_init(&s_bar[w][0]);
+    mbar_init(&s_bar[w][1]);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+  auto grab = [&]() -> long long {
     long long u = 0;
     if (lane == 0) u = atomicAdd(P.ticket, 1);
-    u = __shfl_sync(FULL, u, 0);
-    if (u >= nunits) break;
-    const int2 un = P.units[u];
-    const int t = un.x, k = un.y;
-    // ---- the item ----------------------------------------------------------------------------
-    const int r = P.items[t], r2 = P.items[t + 1];
-    const long long o0 = P.crow[r];
-    const int c = (int)(P.crow[r2] - o0);
-    const long long P0 = P.Ro[r];
-    const uint8_t cl = P.cls[r];
-    const bool wide = (cl & CLS_HEAVY_PATH) && (cl & CLS_WIDE);
-    const int e0 = P.rpA[P.row_begin + r];
-    const unsigned* __restrict__ plan = P.plan + P0;
-    // plan position x -> A entry e, B entry q
-    auto decode = [&](long long x, int& e, int& q) {
-      unsigned er, qo;
-      if (wide) {
-        er = __ldcs(plan + 2 * x);
-        qo = __ldcs(plan + 2 * x + 1);
-      } else {
-        const unsigned w = __ldcs(plan + x);
-        er = w & 0xffffu;
-        qo = w >> 16;
-      }
-      e = e0 + (int)er;
-      q = __ldg(P.Tb + e) + (int)qo;
-    };
-    int* __restrict__ ccol = P.ccol + o0;
-    V* __restrict__ cval = P.cval + o0;
+    return __shfl_sync(FULL, u, 0);
+  };
+  // stage the plan words of unit x into buffer b (narrow units; wide ones read the plan
+  // directly); returns the word offset of the unit's first word inside the buffer
+  auto staged = [](const NumUnit& x) { return !(x.ob & UNIT_WIDE); };
+  auto stage = [&](const NumUnit& x, int b) -> int {
+    if (!staged(x)) return 0;
+    const long long a0 = x.pw & ~3LL, a1 = (x.pw + x.n + 3) & ~3LL;
+    if (lane == 0) tma_plan(s_buf[w][b], P.plan + a0, (unsigned)(a1 - a0) * 4u, &s_bar[w][b]);
+    return (int)(x.pw - a0);
+  };
 
-    // ---- outputs [k NUM_SH, ...) in C order ------------------------------------------------
-    const int ob = k * NUM_SH, oe = min(c, ob + NUM_SH);
-    for (int o00 = ob + lane; o00 < oe; o00 += 32 * NUM_U) {
+  long long u = grab();
+  if (u >= nunits) return;
+  NumUnit cur = P.units[u];
+  int cur_sh = stage(cur, 0);
+  unsigned phases = 0u;  // bit b: parity of buffer b's next completion
+  int cb = 0;
+  for (;;) {
+    // prefetch the next unit's plan while this one is processed
+    const long long un = grab();
+    const bool more = un < nunits;
+    NumUnit nxt;
+    int nxt_sh = 0;
+    if (more) {
+      nxt = P.units[un];
+      nxt_sh = stage(nxt, cb ^ 1);
+    }
+    const bool wide = cur.ob & UNIT_WIDE;
+    const int e0 = cur.e0, n = cur.n;
+    // ---- outputs in C order -----------------------------------------------------------------------
+    int* __restrict__ ccol = P.ccol + cur.oc;
+    V* __restrict__ cval = P.cval + cur.oc;
+    const unsigned* pb = s_buf[w][cb] + cur_sh;
+    if (!wide) {
+      mbar_wait(&s_bar[w][cb], (phases >> cb) & 1u);
+      phases ^= 1u << cb;
+    }
+    for (int o00 = lane; o00 < n; o00 += 32 * NUM_U) {
       int e[NUM_U], q[NUM_U];
 #pragma unroll
       for (int x = 0; x < NUM_U; ++x) {
         const int o = o00 + 32 * x;
         q[x] = -1;
-        if (o < oe) decode(o, e[x], q[x]);
+        if (o < n) {
+          unsigned er, qo;
+          if (!wide) {
+            const unsigned wd = pb[o];
+            er = wd & 0xffffu;
+            qo = wd >> 16;
+          } else {
+            er = __ldcs(P.plan + cur.pw + 2 * (long long)o);
+            qo = __ldcs(P.plan + cur.pw + 2 * (long long)o + 1);
+          }
+          e[x] = e0 + (int)er;
+          q[x] = __ldg(P.Tb + e[x]) + (int)qo;
+        }
       }
       int col[NUM_U];
       V a[NUM_U], b[NUM_U];
@@ -105,31 +147,34 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
           st_cs(cval + o, a[x] * b[x]);
         }
     }
-    // ---- this unit's share of the repeated products ---------------------------------------------
-    const int f = (int)((P.Ro[r2] - P0) >> (wide ? 1 : 0));
-    if (f > c) {
-      const int hs = (c + NUM_SH - 1) / NUM_SH, d = f - c;
-      const int jb = (int)((long long)d * k / hs), je = (int)((long long)d * (k + 1) / hs);
-      __syncwarp();
-      if (lane == 0) {
-        red_release(P.hd + t, 1);  // this warp's outputs are in L2 before the count
-        if (je > jb) {
-          // The adds below are L2 atomics issued only after the loop exits (control dependency;
-          // no speculative stores), so they land after every counted unit's outputs.
-          const int need = P.epoch * hs;
-          while (ld_relaxed(P.hd + t) < need) __nanosleep(100);
+    __syncwarp();  // every lane is done with buffer cb, and its stores precede the adds below
+    // ---- repeated products of the item that land in this unit's outputs ------------------------
+    if (cur.d > 0) {
+      const int ob = cur.ob & (UNIT_WIDE - 1);
+      const int sw = wide ? 2 : 1;
+      V* __restrict__ cv0 = cval - ob;
+      for (int j = lane; j < cur.d; j += 32) {
+        const long long x = cur.dw + (long long)j * sw;
+        const int o = (int)__ldg(P.D + x);
+        if ((unsigned)(o - ob) >= (unsigned)n) continue;
+        unsigned er, qo;
+        if (!wide) {
+          const unsigned wd = __ldg(P.plan + x);
+          er = wd & 0xffffu;
+          qo = wd >> 16;
+        } else {
+          er = __ldg(P.plan + x);
+          qo = __ldg(P.plan + x + 1);
         }
-      }
-      __syncwarp();
-      for (int j = jb + lane; j < je; j += 32) {
-        const long long x = f - 1 - j;
-        int e, q;
-        decode(x, e, q);
-        const V v = __ldg(P.valA + e) * __ldg(P.valB + q);
-        const int o = (int)__ldcs(P.D + P0 + (wide ? 2 * x : x));
-        atomicAdd(cval + o, v);
+        const int e = e0 + (int)er;
+        const int q = __ldg(P.Tb + e) + (int)qo;
+        atomicAdd(cv0 + o, __ldg(P.valA + e) * __ldg(P.valB + q));
       }
     }
+    if (!more) break;
+    cur = nxt;
+    cur_sh = nxt_sh;
+    if (staged(cur)) cb ^= 1;
   }
 }
 

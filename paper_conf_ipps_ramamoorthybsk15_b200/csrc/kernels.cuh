@@ -13,10 +13,10 @@
 //   units      k_unit_count + scan + k_unit_fill: numeric work units — segments of an item's
 //              outputs
 //   numeric    k_numeric: persistent warps take units from a queue — C(i, j) = valA[e]·valB[q]
-//              streamed in C order (coalesced plan read, coalesced C write; A/B from L2); then,
-//              once every unit of the item has stored, a share of the item's repeated products
-//              is added with RED (Phase IV of PAPER.md L154-156: the sort moved to symbolic, so
-//              numeric re-runs on new values are a stream)
+//              streamed in C order (TMA-staged plan words, coalesced C write; A/B from L2); then
+//              the unit adds the item's repeated products that land in its outputs with RED
+//              (Phase IV of PAPER.md L154-156: the sort moved to symbolic, so numeric re-runs on
+//              new values are a stream)
 #pragma once
 #include "common.cuh"
 
@@ -44,6 +44,7 @@ struct Small {
   int tqhead;               // tiles: dynamic queue head
   long long dups;           // repeated products (statistics)
   long long nunits;         // numeric work units
+  unsigned long long scratch_head;  // k_dup_sort scratch reservation
   unsigned long long hist[65];
   unsigned long long cstats[2 * NUM_CLS + 2];
 };
@@ -70,10 +71,26 @@ struct SymProb {
   int row_begin, row_end;
 };
 
-// Numeric work units: item t has hs_t = ceil(c_t / NUM_SH) units; unit {t, k} stores outputs
-// [k NUM_SH, (k + 1) NUM_SH) of the item, then adds the k-th of hs_t equal shares of its
-// repeated products (d_t = f_t - c_t) once all hs_t units have stored.
-constexpr int NUM_SH = 1024;
+// Numeric work units, in a list built in item order: item t has ceil(c_t / NUM_SH) units, unit k
+// owning outputs [k NUM_SH, (k + 1) NUM_SH) of the item.  A unit stores its outputs, then adds
+// the item's repeated products (d_t = f_t - c_t plan entries after the outputs, each with its
+// output in D) that land in its own outputs: a warp only ever adds into outputs it stored
+// itself, so no unit waits for another.  Heavy rows' repeats are bucketed by unit after symbolic
+// (k_dup_sort: bucket starts in dub[dub_index(P0, t) + k]), so a unit reads only its bucket;
+// tiles (few repeats) and wide rows keep them unsorted and every unit filters the list.
+constexpr int NUM_SH = 512;
+constexpr int DUP_SORT_UNITS = 8192;   // heavy rows with more units keep their repeats unsorted
+__host__ __device__ __forceinline__ long long dub_index(long long P0, long long t) { return P0 / NUM_SH + 2 * t; }
+struct NumUnit {
+  long long pw;   // plan word of the unit's first output
+  long long oc;   // C offset (local) of the unit's first output
+  long long dw;   // plan word of the item's first repeated product
+  int d;          // repeated products of the item
+  int n;          // outputs of the unit
+  int e0;         // first A entry of the item
+  int ob;         // item-relative output of the unit's first output | UNIT_WIDE
+};
+constexpr int UNIT_WIDE = 1 << 30;   // two plan words per entry
 
 // Numeric phase.
 template <typename V>
@@ -88,12 +105,10 @@ struct NumProb {
   const long long* __restrict__ crow;   // C row offsets (local)
   const uint8_t* __restrict__ cls;
   const int* __restrict__ items;        // ordered item starts (local rows) + sentinel
-  const int2* __restrict__ units;
+  const NumUnit* __restrict__ units;
   const long long* __restrict__ nunits;
   const unsigned* __restrict__ D;
-  int* hd;                              // per item: finished output segments (all calls)
   int* ticket;                          // work-unit queue head (zeroed before the launch)
-  int epoch;                            // numeric calls since symbolic (1, 2, ...)
   int row_begin;
   int* ccol;
   V* cval;
@@ -102,10 +117,13 @@ struct NumProb {
 // analysis.cu
 cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* colA, int K, const int* rpB, int* f,
                              uint8_t* nz, int* Tb, int* Tl, unsigned long long* hist, int* err, int* amax);
-cudaError_t launch_unit_count(cudaStream_t st, int sms, const int* items, const long long* crow, const long long* Ro,
-                              const uint8_t* cls, int mloc, int* ucnt, int* hd);
-cudaError_t launch_unit_fill(cudaStream_t st, int sms, const int* ucnt, const long long* uscan, int mloc,
-                             int2* units, Small* small, const int* items, const long long* crow);
+cudaError_t launch_unit_count(cudaStream_t st, int sms, const int* items, const long long* crow, int n, int* ucnt);
+cudaError_t launch_unit_fill(cudaStream_t st, int sms, const int* ucnt, const long long* uscan, int n,
+                             NumUnit* units, Small* small, const int* items, const long long* crow,
+                             const long long* Ro, const uint8_t* cls, const int* rpA, int rb, const int* dub);
+cudaError_t launch_dup_sort(cudaStream_t st, const HeavyLists& lists, const int* counts_host, const long long* crow,
+                            const long long* Ro, const uint8_t* cls, const long long* tscan, unsigned* plan,
+                            unsigned* D, uint2* scratch, unsigned long long* scratch_head, int* dub);
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
                             const ClassParams& prm, uint8_t* cls, int* pw, const HeavyLists& lists, Small* small);
 cudaError_t launch_tile_flags(cudaStream_t st, int sms, const int* f, const int* rpA, int rb, int re, int tile_cap,

@@ -249,7 +249,7 @@ __global__ void __launch_bounds__(256) k_unit_fill(const int* __restrict__ ucnt,
     const long long f = (Ro[r2] - P0) / sw;
     const int e0 = rpA[rb + r];
     const int* db = dub + dub_index(P0, t);
-    const bool sorted = (cls[r] & CLS_HEAVY_PATH) && f > c && db[0] >= 0;  // heavy rows: k_dup_sort
+    const bool sorted = f > c && db[0] >= 0;  // bucketed repeats (k_tile_rank / k_dup_sort)
     for (int k = 0; k < u; ++k) {
       NumUnit v;
       v.pw = P0 + (long long)k * NUM_SH * sw;
@@ -268,9 +268,8 @@ __global__ void __launch_bounds__(256) k_unit_fill(const int* __restrict__ ucnt,
 // Repeats of a heavy row bucketed by numeric unit (counting sort on o / NUM_SH): one block per
 // heavy row, a scratch copy of the (word, output) pairs, then written back in bucket order.
 // dub[dub_index(P0, t) + k] = first repeat of unit k (relative to the row's repeats), k <= hs;
-// dub[...] = -1: not sorted (no repeats, a wide row, more than DUP_SORT_UNITS units, or so few
-// units and repeats that filtering is cheaper).
-constexpr int DS_NT = 512;
+// dub[...] = -1: not sorted (no repeats, a wide row, or more than DUP_SORT_UNITS units).
+constexpr int DS_NT = 128;
 __global__ void __launch_bounds__(DS_NT) k_dup_sort(HeavyLists lists, int c0, int c1, int c2,
                                                     const long long* __restrict__ crow,
                                                     const long long* __restrict__ Ro, const uint8_t* __restrict__ cls,
@@ -294,9 +293,15 @@ __global__ void __launch_bounds__(DS_NT) k_dup_sort(HeavyLists lists, int c0, in
   const long long f = (Ro[li + 1] - P0) >> (wide ? 1 : 0);
   const long long d = f - c;
   const long long hs = (c + NUM_SH - 1) / NUM_SH;
-  // (few units x few repeats: numeric filters the unsorted list more cheaply than this sorts it)
-  if (d <= 0 || wide || hs > DUP_SORT_UNITS || hs * d <= 8192) {
+  if (d <= 0 || wide || hs > DUP_SORT_UNITS) {
     if (tid == 0) db[0] = -1;
+    return;
+  }
+  if (hs == 1) {  // one unit: already its own bucket
+    if (tid == 0) {
+      db[0] = 0;
+      db[1] = (int)d;
+    }
     return;
   }
   for (int k = tid; k <= hs; k += DS_NT) s_cnt[k] = 0;

@@ -186,6 +186,7 @@ SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* cr
   P.fl8 = h->fl8.as<uint8_t>();
   P.crow = crow;
   P.D = h->D.as<unsigned>();
+  P.dub = h->dub.as<int>();
   P.dups = &h->small.as<Small>()->dups;
   long long r_cap = h->plan_cap();
   P.r_cap = r_cap;
@@ -407,6 +408,8 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(launch_classify(h->stream, h->sms, h->f.as<int>(), h->nz.as<uint8_t>(), h->rb, h->re, prm,
                        h->cls.as<uint8_t>(), h->pw.as<int>(), L3, ds));
     CK(launch_incl_scan<int>(h->stream, h->pw.as<int>(), Ro + 1, Mloc, h->scan_tmp.as<long long>()));
+    // repeats' bucket starts: index < plan words / NUM_SH + 2 items + 2
+    CK(h->dub.ensure((size_t)(h->plan_cap() / NUM_SH + 2LL * (Mloc + 1) + 4) * sizeof(int)));
     CK(launch_tile_flags(h->stream, h->sms, h->f.as<int>(), A->row_ptr, h->rb, h->re, tile_cap, h->cls.as<uint8_t>(),
                          Ro, h->tflag.as<int>()));
     CK(launch_incl_scan<int>(h->stream, h->tflag.as<int>(), h->tscan.as<long long>(), Mloc,
@@ -444,7 +447,6 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   {  // repeats of heavy rows bucketed by numeric unit, then the numeric work units (structure
      // only: built once, reused by every numeric call)
     const Small* dsm = h->small.as<Small>();
-    CK(h->dub.ensure((size_t)(h->plan_words / NUM_SH + 2LL * hs.nitems + 4) * sizeof(int)));
     CK(h->dscratch.ensure((size_t)(hs.dups + 1) * sizeof(uint2)));
     CK(cudaMemsetAsync(&ds->scratch_head, 0, sizeof(unsigned long long), h->stream));
     HeavyLists HL;

@@ -20,9 +20,9 @@
 //   6. offsets   block scan of c_j: the output offset of every row inside the tile.
 //   7. ranks     rank = heads of the row's earlier buckets + distinct smaller columns in the own
 //                bucket; a head writes its plan word at P0 + out_j + rank (C order), every other
-//                product at the end of the tile's plan region (the dups, each with its output
-//                out_j + rank in D at the same word).  SINGLE rows (one non-empty B row,
-//                already sorted) write their products in order.
+//                product after the tile's outputs (the dups, each with its output out_j + rank
+//                in D at the same word), bucketed by the numeric unit that owns that output.
+//                SINGLE rows (one non-empty B row, already sorted) write their products in order.
 // This is Phase IV's "sort, mark like-tuples, scan, compact", done per tile in
 // shared memory.
 #include "kernels.cuh"
@@ -98,7 +98,9 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
   int* sae = reinterpret_cast<int*>(sm + TileSmem::sae);
   uint8_t* srw = reinterpret_cast<uint8_t*>(sm + TileSmem::srw);
   __shared__ int scratch[TILE_NT / 32 + 1];
-  __shared__ int s_tile, s_dn;
+  __shared__ int s_tile;
+  constexpr int TU = TILE_PMAX / NUM_SH;  // numeric units of a tile
+  __shared__ int s_uc[TU + 1], s_us[TU + 1];
   constexpr int NT = TILE_NT, NW = NT / 32;
   const Group<NT> g{(int)threadIdx.x, scratch};
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -325,13 +327,13 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
       if (tid < nr) s_out[tid] = ex;
       if (tid == 0) {
         s_out[nr] = tot;
-        s_dn = 0;
         if (PT > tot) atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)(PT - tot));
       }
+      if (tid <= TU) s_uc[tid] = 0;
     }
     __syncthreads();
 
-    // ---- 7. ranks -> plan: heads in C order, the others at the end of the region -----------------
+    // ---- 7. ranks -> plan: heads in C order; repeats after them, bucketed by numeric unit --------
     unsigned* plan = P.plan + P0;
     for (int x = tid; x < Pg; x += NT) {
       const int b = sbk[x];
@@ -344,15 +346,36 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
         u += (ky >= 0 && ky < k);
       }
       const int jr = brow[b];
-      const unsigned w = pay[sidx[x]];
       const int o = s_out[jr] + hc[b] - hc[s_bb[jr]] + u;  // output of the product's column
       if (kx >= 0) {
-        plan[o] = w;
-      } else {  // a repeat: slot from the end of the region, its output in D at the same word
-        const int x2 = PT - 1 - atomicAdd(&s_dn, 1);
-        plan[x2] = w;
-        P.D[P0 + x2] = (unsigned)o;
+        plan[o] = pay[sidx[x]];
+      } else {  // a repeat: its output parked in sbk (read above, own slot only)
+        sbk[x] = (unsigned short)o;
+        atomicAdd(&s_uc[o / NUM_SH], 1);
       }
+    }
+    const int Ct = s_out[nr];
+    __syncthreads();
+    if (PT > Ct) {
+      if (tid == 0) {  // bucket starts, also for numeric (dub)
+        int* db = P.dub + dub_index(P0, t);
+        const int hs = (Ct + NUM_SH - 1) / NUM_SH;
+        int run = 0;
+        for (int k = 0; k < hs; ++k) {
+          s_us[k] = run;
+          db[k] = run;
+          run += s_uc[k];
+        }
+        db[hs] = run;
+      }
+      __syncthreads();
+      for (int x = tid; x < Pg; x += NT)
+        if (keys[x] < 0) {
+          const int o = sbk[x];
+          const int pos = Ct + atomicAdd(&s_us[o / NUM_SH], 1);
+          plan[pos] = pay[sidx[x]];
+          P.D[P0 + pos] = (unsigned)o;
+        }
     }
     for (int idx = tid; idx < PT; idx += NT)  // SINGLE rows: products already in column order
       if (exb[idx] == NOBUCKET) {

@@ -66,6 +66,7 @@ struct SymProb {
   long long* crow;          // C row offsets (local); symbolic writes counts at [li + 1]
   unsigned* D;              // item-relative output of the repeated product whose plan entry starts
                             // at the same word (sized like the plan, written only for repeats)
+  int* dub;                 // repeats' bucket starts per numeric unit (dub_index(P0, t) + k)
   long long* dups;          // repeated-product counter (statistics)
   long long r_cap;          // plan capacity (words); the kernels do nothing if Ro[Mloc] > r_cap
   int row_begin, row_end;
@@ -75,11 +76,12 @@ struct SymProb {
 // owning outputs [k NUM_SH, (k + 1) NUM_SH) of the item.  A unit stores its outputs, then adds
 // the item's repeated products (d_t = f_t - c_t plan entries after the outputs, each with its
 // output in D) that land in its own outputs: a warp only ever adds into outputs it stored
-// itself, so no unit waits for another.  Heavy rows' repeats are bucketed by unit after symbolic
-// (k_dup_sort: bucket starts in dub[dub_index(P0, t) + k]), so a unit reads only its bucket;
-// tiles (few repeats) and wide rows keep them unsorted and every unit filters the list.
+// itself, so no unit waits for another.  The repeats are bucketed by unit (tiles: in k_tile_rank;
+// heavy rows: k_dup_sort after symbolic), bucket starts in dub[dub_index(P0, t) + k], so a unit
+// reads only its bucket; rows with dub[...] = -1 (wide, or more than DUP_SORT_UNITS units) keep
+// them unsorted and every unit of the row filters the list.
 constexpr int NUM_SH = 512;
-constexpr int DUP_SORT_UNITS = 8192;   // heavy rows with more units keep their repeats unsorted
+constexpr int DUP_SORT_UNITS = 1024;   // heavy rows with more units keep their repeats unsorted
 __host__ __device__ __forceinline__ long long dub_index(long long P0, long long t) { return P0 / NUM_SH + 2 * t; }
 struct NumUnit {
   long long pw;   // plan word of the unit's first output

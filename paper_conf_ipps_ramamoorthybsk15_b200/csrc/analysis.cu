@@ -269,7 +269,7 @@ __global__ void __launch_bounds__(256) k_unit_fill(const int* __restrict__ ucnt,
 // heavy row, a scratch copy of the (word, output) pairs, then written back in bucket order.
 // dub[dub_index(P0, t) + k] = first repeat of unit k (relative to the row's repeats), k <= hs;
 // dub[...] = -1: not sorted (no repeats, a wide row, or more than DUP_SORT_UNITS units).
-constexpr int DS_NT = 128;
+constexpr int DS_NT = 1024;
 __global__ void __launch_bounds__(DS_NT) k_dup_sort(HeavyLists lists, int c0, int c1, int c2,
                                                     const long long* __restrict__ crow,
                                                     const long long* __restrict__ Ro, const uint8_t* __restrict__ cls,

@@ -185,6 +185,7 @@ SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* cr
   P.plan = h->plan.as<unsigned>();
   P.fl8 = h->fl8.as<uint8_t>();
   P.crow = crow;
+  P.tscan = h->tscan.as<long long>();
   P.D = h->D.as<unsigned>();
   P.dub = h->dub.as<int>();
   P.dups = &h->small.as<Small>()->dups;
@@ -451,9 +452,9 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(cudaMemsetAsync(&ds->scratch_head, 0, sizeof(unsigned long long), h->stream));
     HeavyLists HL;
     int hc[NUM_BINS];
-    for (int b = 0; b < NUM_BINS; ++b) {
+    for (int b = 0; b < NUM_BINS; ++b) {  // (register-cached bins bucket their repeats themselves)
       HL.rows[b] = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
-      hc[b] = hs.counts[b];
+      hc[b] = b == BIN_HUGE ? hs.counts[b] : 0;
     }
     CK(launch_dup_sort(h->stream, HL, hc, crow, h->Ro.as<long long>(), h->cls.as<uint8_t>(), h->tscan.as<long long>(),
                        h->plan.as<unsigned>(), h->D.as<unsigned>(), h->dscratch.as<uint2>(), &ds->scratch_head,

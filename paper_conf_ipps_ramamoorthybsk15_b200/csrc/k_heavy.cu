@@ -15,8 +15,10 @@
 //           output in D at the same word).
 //   c_i     = claimed bits (summed over column tiles).
 // HEAVY rows (f <= 8192, one gather chunk) keep their products (column) in registers across
-// the passes and their head flags in a shared bit array; HUGE rows re-gather columns per pass
-// and keep the flag in a global byte per product (fl8) between pass 1 and pass 2.  Products are
+// the passes and their head flags in a shared bit array, and place their repeats after the
+// outputs bucketed by numeric unit at the end of the row; HUGE rows re-gather columns per pass,
+// keep the flag in a global byte per product (fl8) between pass 1 and pass 2, and leave their
+// repeats unsorted at the end of the region (k_dup_sort buckets them after symbolic).  Products are
 // visited in 32-product warp windows (coalesced within a B row); the run of each lane comes from
 // a REDUX.OR mask of run starts.  SINGLE rows (one non-empty B row) only copy their run.
 #include "kernels.cuh"
@@ -75,6 +77,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
   const int n = count[0];
   __shared__ int s_next;
   __shared__ int s_dcnt, s_single;
+  __shared__ int s_uc[HEAVY_CAP / NUM_SH + 2];  // cached rows: repeats per numeric unit
   for (;;) {
     if (tid == 0) s_next = atomicAdd(const_cast<int*>(count) + 8, 1);
     __syncthreads();
@@ -132,6 +135,8 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
     int out = 0;
     int nz = 0, Lt = 0;  // current chunk: runs, products
     int cc[BMP_SLOTS];   // cached mode: this lane's product columns
+    int oo[BMP_SLOTS];   // ... and the outputs of those that repeat a column (bit s of dmask)
+    unsigned dmask = 0;
 
     auto gather = [&](int c) {
       const int p = pa0 + c * RCAP + tid;
@@ -332,8 +337,12 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
               if (in) {
                 const bool first = (flags[j >> 5] >> (j & 31)) & 1u;
                 const int o = out + rank_of(lc);
-                if (first) put(o, sae[r] - pa0, j - seg[r]);
-                else put_dup(o, sae[r] - pa0, j - seg[r]);
+                if (first) {
+                  put(o, sae[r] - pa0, j - seg[r]);
+                } else {  // placed after the row's outputs once c_i is known (below)
+                  oo[s] = o;
+                  dmask |= 1u << s;
+                }
               }
             }
           }
@@ -389,10 +398,46 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
         for (int x = tid; x < nfw; x += NT) flags[x] = 0;
       __syncthreads();
     }
+    if constexpr (CACHED) {
+      if (f > out) {  // repeats after the outputs, bucketed by the numeric unit owning their output
+        const int hs = (out + NUM_SH - 1) / NUM_SH;
+        if (tid <= hs) s_uc[tid] = 0;
+        __syncthreads();
+#pragma unroll
+        for (int s = 0; s < BMP_SLOTS; ++s)
+          if (dmask >> s & 1u) atomicAdd(&s_uc[oo[s] / NUM_SH], 1);
+        __syncthreads();
+        if (tid == 0) {
+          int* db = P.dub + dub_index(ro, P.tscan[li] - 1);
+          int run = 0;
+          for (int k = 0; k < hs; ++k) {
+            const int v = s_uc[k];
+            s_uc[k] = run;
+            db[k] = run;
+            run += v;
+          }
+          db[hs] = run;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int s = 0; s < BMP_SLOTS; ++s) {
+          const int j0 = warp * 32 + s * NT;
+          if (j0 < Lt) {  // warp-uniform
+            const int r = lane_run(j0);
+            if (dmask >> s & 1u) {
+              const int pos = out + atomicAdd(&s_uc[oo[s] / NUM_SH], 1);
+              put(pos, sae[r] - pa0, j0 + lane - seg[r]);
+              P.D[ro + pos] = (unsigned)oo[s];
+            }
+          }
+        }
+      }
+    }
     if (tid == 0) {
       P.crow[li + 1] = out;
       if (f > out) atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)(f - out));
     }
+    __syncthreads();
   }
 }
 

@@ -64,6 +64,7 @@ struct SymProb {
   unsigned* plan;           // the plan (capacity r_cap words)
   uint8_t* fl8;             // uncached bitmap rows: first-claim flag per product (Ro_i + offset)
   long long* crow;          // C row offsets (local); symbolic writes counts at [li + 1]
+  const long long* tscan;   // inclusive scan of the item-start flags: item of row li = tscan[li] - 1
   unsigned* D;              // item-relative output of the repeated product whose plan entry starts
                             // at the same word (sized like the plan, written only for repeats)
   int* dub;                 // repeats' bucket starts per numeric unit (dub_index(P0, t) + k)

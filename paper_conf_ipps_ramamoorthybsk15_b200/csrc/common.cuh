@@ -40,7 +40,6 @@ constexpr int TILE_EC = 1024;         // entries: a tile never crosses a multipl
 constexpr int TILE_RM = 256;          // rows per tile (tiles never cross a multiple of TILE_RM)
 constexpr int TILE_NT = 512;          // threads per symbolic tile block
 constexpr int TILE_BK = 2;            // expected products per bucket
-constexpr int TILE_NBMAX = TILE_PMAX / TILE_BK + TILE_RM;  // buckets per tile (ceil per row)
 // Heavy (bitmap) kernel geometry.
 constexpr int HEAVY_CAP = 8192;       // largest f of the register-cached bitmap mode (1024 threads)
 constexpr int HEAVY1_CAP = 4096;      // ... 512-thread blocks, two per SM

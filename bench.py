@@ -7,7 +7,12 @@ One step = the whole hot path on one input: row analysis + classification + symb
 resident in HBM before timing; L2 is flushed (256 MiB memset) between timed steps.  N > 1:
 rows are flop-partitioned across ranks (a5), B resident on every rank (replicated with an NCCL
 broadcast before timing), each rank times its block, the max over ranks is the step time and
-`value` is 2 * F_total / that time (strong scaling: total work fixed).
+`value` is 2 * F_total / that time (strong scaling: total work fixed).  `python bench.py
+--gpus N` outside torchrun re-launches itself under torch.distributed.run with N ranks.
+
+The roofline object is the numeric phase's HBM roofline on SURVEY.md §8(d)'s compulsory bytes
+(A + B + C); the plan the symbolic phase leaves (4 bytes per product) is reported next to it as
+`plan_bytes` / `with_plan_frac`, not counted as algorithmic.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config webbase1m] [--impl ours|reference]
 """
@@ -53,6 +58,36 @@ def dist_env():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     return ws, rank, local
+
+
+def relaunch_if_needed(args) -> bool:
+    """--gpus N (N > 1) outside torchrun: run this script under torch.distributed.run with N ranks.
+    Returns True if this process only supervised the child launcher."""
+    if "WORLD_SIZE" in os.environ:
+        ws = int(os.environ["WORLD_SIZE"])
+        if ws != args.gpus and not args.virtual:
+            sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={ws}")
+        return False
+    if args.gpus <= 1:
+        return False
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    sys.exit(subprocess.call(cmd))
+
+
+def cpu_model() -> str:
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name:"):
+                return line.split(":", 1)[1].strip()
+    except (OSError, subprocess.TimeoutExpired):
+        pass
+    return "unknown"
 
 
 def load_peaks():
@@ -292,17 +327,15 @@ def run_ours(args):
     F_total = int(st["flops_total"])
     value = 2.0 * F_total / (ms_step * 1e-3) / 1e9
 
-    # roofline of the numeric phase (the dominant stage: class kernels forked on streams and joined)
+    # roofline of the numeric phase (k_numeric, one launch per step): SURVEY.md §8(d)'s compulsory
+    # bytes A + B + C of this rank's rows; the plan read is this design's overhead, reported apart
     nnzA_loc = int(A.row_ptr[re]) - int(A.row_ptr[rb])
-    # A + B + C + intermediate, the intermediate being the read of the symbolic
-    # phase's output (the gather plan: EQ entries of non-SINGLE outputs + the dup list)
     abc_bytes = (csr_bytes(re - rb, nnzA_loc, vb) + csr_bytes(B.nrows, B.nnz, vb)
                  + csr_bytes(re - rb, nnz, vb, rp_bytes=8))
     plan_bytes = int(st["plan_bytes"])
-    alg_bytes = abc_bytes + plan_bytes
     num_ms = float(np.mean(num))
     peak, peak_src = load_peaks()
-    achieved = alg_bytes / (num_ms * 1e-3) / 1e9
+    achieved = abc_bytes / (num_ms * 1e-3) / 1e9
     traffic = None
     tpath = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
     if os.path.exists(tpath):
@@ -351,9 +384,16 @@ def run_ours(args):
         t0 = time.perf_counter()
         oracle.spgemm(A, B, 0, r1, nthreads=T, with_abs=False)
         dt = time.perf_counter() - t0
+        s1, Fs1, _ = oracle_sample(A, B, 8.0, 1)  # single-thread leg
+        t1 = time.perf_counter()
+        oracle.spgemm(A, B, 0, s1, nthreads=1, with_abs=False)
+        dt1 = time.perf_counter() - t1
         cpu = {"value": 2.0 * Fs / dt / 1e9, "unit": UNIT, "cores": T, "kind": "oracle",
+               "cpu_model": cpu_model(),
                "sample": f"rows [0, {r1}) of {args.config}: {Fs} of {F} products ({100.0 * Fs / F:.1f}%), "
-                         f"{dt:.1f} s on {T} threads (std::map Gustavson, as it stands)"}
+                         f"{dt:.1f} s on {T} threads (std::map Gustavson, as it stands)",
+               "single_thread": {"value": 2.0 * Fs1 / dt1 / 1e9, "unit": UNIT, "cores": 1,
+                                 "sample": f"rows [0, {s1}): {Fs1} products, {dt1:.1f} s on 1 thread"}}
 
     clocks = sampler.summary(t_wall0, t_wall1) if sampler else None
     stl = st
@@ -361,7 +401,7 @@ def run_ours(args):
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": ws, "steps": K, "warmup": args.warmup,
-            "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong" if ws > 1 else "weak",
+            "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64" if vb == 8 else "f32", "data": "synthetic",
             "config": {"workload": args.config, "rows": A.nrows, "nnzA": A.nnz, "nnzB": B.nnz, "flops": F_total,
                        "nnzC": int(st["nnz_c"]) if ws == 1 else None,
@@ -369,7 +409,10 @@ def run_ours(args):
                        "parallelism": (f"rows flop-partitioned over {ws} GPU(s)" + (" (virtual ranks on one GPU)"
                                        if args.virtual else "")) if ws > 1 else "1 GPU",
                        "options": args.opt},
+            "ms_per_step_median": float(np.median(sym + num)), "ms_per_step_min": float(np.min(sym + num)),
             "phases": {"symbolic_ms": float(np.mean(sym)), "numeric_ms": num_ms,
+                       "symbolic_ms_median": float(np.median(sym)), "numeric_ms_median": float(np.median(num)),
+                       "numeric_ms_min": float(np.min(num)),
                        "numeric_gflops": 2.0 * int(st["flops"]) / (num_ms * 1e-3) / 1e9,
                        "symbolic_path_ms": dict(zip(["analysis", "light", "heavy"], (path_ms / K).round(4).tolist())),
                        "tiles": int(st["tiles"]), "heavy_rows": int(st["heavy_rows"]), "dup_products": int(st["dup_products"]),
@@ -378,10 +421,10 @@ def run_ours(args):
                        "class_flops": dict(zip(spg.CLASS_NAMES, stl["class_flops"]))},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                         "kernel": "numeric phase (k_numeric gather stream + k_numeric_dup)",
-                         "algorithmic_bytes": int(alg_bytes), "abc_bytes": int(abc_bytes),
+                         "kernel": "k_numeric (numeric phase: one launch per step)",
+                         "algorithmic_bytes": int(abc_bytes), "bytes_def": "A + B + C (SURVEY.md 8d)",
                          "plan_bytes": plan_bytes,
-                         "abc_frac": abc_bytes / (num_ms * 1e-3) / 1e9 / peak},
+                         "with_plan_frac": (abc_bytes + plan_bytes) / (num_ms * 1e-3) / 1e9 / peak},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clocks,
         }
         emit(line, args)
@@ -392,6 +435,7 @@ def run_ours(args):
 
 def main():
     args = parse()
+    relaunch_if_needed(args)
     if args.impl == "reference":
         run_reference(args)
     else:

@@ -102,10 +102,11 @@ typedef enum {
 typedef enum {
   SPG_OPT_LIGHT_MAX_FLOPS = 0,  /* heavy/light threshold t: 0..4096; light rows
                                    above 4096 - TILE_FLOPS are tiles of their own;
-                                   default 1024 with tile 3072 (tools/sweep.py, profiles/); when
-                                   B has > 2^22 columns and neither option was set: 3072 with
-                                   tile 1024.  0 sends every non-SINGLE row to the heavy path  */
-  SPG_OPT_TILE_FLOPS = 1,       /* nominal products per light tile, default 3072               */
+                                   default 2048 with tile 2048 (tools/sweep_quick.sh, profiles/);
+                                   when B has > 2^22 columns and neither option was set: 3072
+                                   with tile 1024.  0 sends every non-SINGLE row to the heavy
+                                   path                                                         */
+  SPG_OPT_TILE_FLOPS = 1,       /* nominal products per light tile, default 2048               */
   SPG_OPT_HEAVY_MAX_FLOPS = 2,  /* 0..8192, default 8192; heavy rows above are HUGE            */
   SPG_OPT_FORCE_CLASS = 3,      /* -1 (default) or a class id c >= TINY: the SINGLE shortcut is
                                    off, and c >= HEAVY sends every non-empty row to the heavy

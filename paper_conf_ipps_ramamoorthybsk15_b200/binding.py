@@ -309,7 +309,17 @@ class SpGEMM:
     def set_option(self, name, value):
         spg_set_option(self.h, name, value)
 
+    def _check(self, *mats):
+        """The C side reads every value array as the handle's dtype: reject anything else."""
+        for m in mats:
+            for t in (m.row_ptr, m.col_idx):
+                if t.dtype != torch.int32 or not t.is_contiguous():
+                    raise TypeError("row_ptr / col_idx must be contiguous int32 tensors")
+            if m.vals.numel() and (m.vals.dtype != self.dtype or not m.vals.is_contiguous()):
+                raise TypeError(f"values must be contiguous {self.dtype}, got {m.vals.dtype}")
+
     def symbolic(self, A: DeviceCSR, B: DeviceCSR) -> DeviceCSR64:
+        self._check(A, B)
         rp = torch.empty(A.nrows + 1, dtype=torch.int64, device=A.row_ptr.device)
         nnz, rb, re = spg_spgemm_symbolic(self.h, A, B, rp)
         n = re - rb
@@ -318,6 +328,9 @@ class SpGEMM:
         return DeviceCSR64(n, B.ncols, rp[: n + 1], col, val, rb)
 
     def numeric(self, A: DeviceCSR, B: DeviceCSR, C: DeviceCSR64) -> DeviceCSR64:
+        self._check(A, B)
+        if C.vals.numel() and (C.vals.dtype != self.dtype or not C.vals.is_contiguous()):
+            raise TypeError(f"C values must be contiguous {self.dtype}")
         spg_spgemm_numeric(self.h, A, B, C.row_ptr, C.col_idx, C.vals)
         return C
 

@@ -32,8 +32,8 @@ constexpr uint8_t NZ_ALEN1K = 0x80;     // ... more than 1024
 constexpr int TINY_MAX = 32;          // class boundaries for statistics only (same kernel)
 constexpr int LIGHTC_MAX = 256;
 constexpr int TILE_PMAX = 4096;       // products per tile: tile capacity + light threshold <= this
-constexpr int TILE_CAP_DEFAULT = 3072;
-constexpr int LIGHT_MAX_DEFAULT = 1024;
+constexpr int TILE_CAP_DEFAULT = 2048;
+constexpr int LIGHT_MAX_DEFAULT = 2048;
 constexpr int TILE_EC = 1024;         // entries: a tile never crosses a multiple of TILE_EC in A's
                                       // entry space, so with rows of <= TILE_EC entries it has
                                       // < 2 * TILE_EC entries

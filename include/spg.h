@@ -116,7 +116,11 @@ typedef enum {
                                    0: the library canonicalises a copy of B                   */
   SPG_OPT_TIMING = 6,           /* 1: record per-phase CUDA-event times into the stats        */
   SPG_OPT_HUGE_SLOTS = 7,       /* max concurrent heavy-row blocks per bin (0 = full occupancy) */
-  SPG_OPT_CONCURRENT = 8        /* 1 (default): light and heavy kernels on concurrent streams  */
+  SPG_OPT_CONCURRENT = 8,       /* 1 (default): light and heavy kernels on concurrent streams  */
+  SPG_OPT_AUTOTUNE = 9          /* 1: the first symbolic call on a new A/B structure times five
+                                   (LIGHT_MAX_FLOPS, TILE_FLOPS) candidates and keeps the fastest
+                                   (spg_stats.light_max / tile_flops report the choice); 0
+                                   (default): the fixed defaults above                         */
 } spg_option;
 
 typedef struct {
@@ -139,6 +143,8 @@ typedef struct {
   float ms_numeric;                       /*   numeric (last numeric call)                */
   float ms_light;                         /*   symbolic light-tile kernel                 */
   float ms_heavy;                         /*   symbolic heavy-row kernels                 */
+  int32_t light_max;                      /* thresholds the last symbolic call used      */
+  int32_t tile_flops;
   int32_t launches_symbolic;              /* kernels launched by the last symbolic call  */
   int32_t launches_numeric;               /* kernels launched by the last numeric call   */
 } spg_stats;
@@ -198,6 +204,23 @@ spg_status spg_create_dist(spg_handle* h, int device, void* cuda_stream, spg_dty
 /* In-place broadcast of a device CSR (row_ptr, col_idx, vals) whose buffers are already
  * allocated with the right sizes on every rank. */
 spg_status spg_broadcast_csr(spg_handle h, spg_csr* m, int root);
+/* As spg_broadcast_csr, but only the structure (row_ptr, col_idx) is broadcast on the handle's
+ * stream; the values go over an internal communication stream, so a following
+ * spg_spgemm_symbolic (structure only) overlaps them.  The next spg_spgemm_numeric on this
+ * handle waits for the values (valB broadcast overlapped with symbolic). */
+spg_status spg_broadcast_csr_async(spg_handle h, spg_csr* m, int root);
+/* A != B (the paper ships A's row blocks to its devices): A lives on `root` only.
+ * Every rank passes A's dimensions (pointers may be NULL off the root) and the replicated B.
+ * The root computes the flop-balanced split points (same formula as above) and broadcasts them;
+ * every rank learns its rows [row_begin, row_end) and their entry count.  Synchronous. */
+spg_status spg_scatter_plan(spg_handle h, const spg_csr* A, const spg_csr* B, int root, int32_t* row_begin,
+                            int32_t* row_end, int64_t* nnz_local);
+/* After spg_scatter_plan: the root sends every rank its row block (ncclSend / ncclRecv group).
+ * A_local: device buffers allocated by the caller for (row_end - row_begin) rows and nnz_local
+ * entries; its row offsets come out starting at 0.  The rank then multiplies A_local x B with a
+ * single-GPU handle; the row blocks of C concatenate in rank order.  Stream-ordered. */
+spg_status spg_scatter_rows(spg_handle h, const spg_csr* A, int root, spg_csr* A_local);
+
 /* Gathers every rank's C row block into full C on every rank (allgatherv through grouped
  * ncclBroadcast).  C_row_ptr_full: device int64[M+1]; C_col_full/C_val_full sized for
  * the total nnz (= sum of all ranks' nnzC; query with spg_allgather_nnz). */

@@ -26,12 +26,13 @@ CLASS_NAMES = ["empty", "single", "tiny", "light", "medium", "heavy", "huge"]
 NUM_CLASSES = 7
 # options
 OPTIONS = {"light_max_flops": 0, "tile_flops": 1, "heavy_max_flops": 2, "force_class": 3, "validate": 4,
-           "input_canonical": 5, "timing": 6, "huge_slots": 7, "concurrent": 8}
+           "input_canonical": 5, "timing": 6, "huge_slots": 7, "concurrent": 8, "autotune": 9}
 
 EXPORTED = ["spg_create", "spg_set_option", "spg_get_option", "spg_spgemm_free", "spg_last_error", "spg_get_stats",
             "spg_version", "spg_spgemm_symbolic", "spg_spgemm_numeric", "spg_spgemm_host_symbolic",
             "spg_spgemm_host_numeric", "spg_get_unique_id", "spg_create_dist", "spg_broadcast_csr",
-            "spg_allgather_nnz", "spg_allgatherv_c", "spg_split_points"]
+            "spg_allgather_nnz", "spg_allgatherv_c", "spg_split_points", "spg_broadcast_csr_async",
+            "spg_scatter_plan", "spg_scatter_rows"]
 
 
 class spg_csr(ctypes.Structure):
@@ -46,6 +47,7 @@ class spg_stats(ctypes.Structure):
                 ("bin_hist", c_int64 * 65), ("tiles", c_int64), ("heavy_rows", c_int64),
                 ("dup_products", c_int64), ("plan_bytes", c_int64), ("ms_analysis", c_float), ("ms_symbolic", c_float),
                 ("ms_numeric", c_float), ("ms_light", c_float), ("ms_heavy", c_float),
+                ("light_max", c_int32), ("tile_flops", c_int32),
                 ("launches_symbolic", c_int32), ("launches_numeric", c_int32)]
 
     def to_dict(self) -> dict:
@@ -100,6 +102,10 @@ def load(build_if_missing: bool = True):
         "spg_allgather_nnz": [H, c_int64, POINTER(c_int64)],
         "spg_allgatherv_c": [H, P, P, P, P, P, P],
         "spg_split_points": [H, POINTER(spg_csr), POINTER(spg_csr), c_int32, P],
+        "spg_broadcast_csr_async": [H, POINTER(spg_csr), c_int],
+        "spg_scatter_plan": [H, POINTER(spg_csr), POINTER(spg_csr), c_int, POINTER(c_int32), POINTER(c_int32),
+                             POINTER(c_int64)],
+        "spg_scatter_rows": [H, POINTER(spg_csr), c_int, POINTER(spg_csr)],
     }
     for name, args in sig.items():
         fn = getattr(lib, name)
@@ -273,6 +279,27 @@ def spg_create_dist(device: int, stream, dtype, uid, rank: int, nranks: int) -> 
 def spg_broadcast_csr(h, m: DeviceCSR, root: int):
     c = m.c()
     _check(h, load().spg_broadcast_csr(h, byref(c), root))
+
+
+def spg_broadcast_csr_async(h, m: DeviceCSR, root: int):
+    c = m.c()
+    _check(h, load().spg_broadcast_csr_async(h, byref(c), root))
+
+
+def spg_scatter_plan(h, A, B: DeviceCSR, root: int):
+    """A: DeviceCSR on the root; elsewhere any object with nrows/ncols (its tensors are not read).
+    Returns (row_begin, row_end, nnz_local)."""
+    a = A.c() if isinstance(A, DeviceCSR) else spg_csr(int(A.nrows), int(A.ncols), 0, None, None, None)
+    b = B.c()
+    rb, re, nz = c_int32(), c_int32(), c_int64()
+    _check(h, load().spg_scatter_plan(h, byref(a), byref(b), root, byref(rb), byref(re), byref(nz)))
+    return rb.value, re.value, nz.value
+
+
+def spg_scatter_rows(h, A, root: int, A_local: DeviceCSR):
+    a = A.c() if isinstance(A, DeviceCSR) else spg_csr(int(A.nrows), int(A.ncols), 0, None, None, None)
+    loc = A_local.c()
+    _check(h, load().spg_scatter_rows(h, byref(a), root, byref(loc)))
 
 
 def spg_allgather_nnz(h, nnz_local: int) -> int:

@@ -475,6 +475,21 @@ __global__ void k_rebase(long long* __restrict__ rp, int M, int P, const int* __
   }
 }
 
+// Scatter of A's row blocks: rp[i] -= rp[0] (a received block's row offsets start at 0), and the
+// per-rank row / entry counts of a split: out[r] = s[r+1]-s[r], out[P+r] = rpA[s[r+1]]-rpA[s[r]].
+__global__ void k_rebase32(int* __restrict__ rp, long long n, const int* __restrict__ first) {
+  const int b = *first;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+    rp[i] -= b;
+}
+__global__ void k_split_sizes(const int* __restrict__ s, const int* __restrict__ rpA, int P, long long* __restrict__ out) {
+  for (int r = threadIdx.x; r < P; r += blockDim.x) {
+    out[r] = s[r + 1] - s[r];
+    out[P + r] = (long long)rpA[s[r + 1]] - rpA[s[r]];
+    out[2 * P + r] = rpA[s[r]];
+  }
+}
+
 // Canonicalisation helpers (SPG_OPT_INPUT_CANONICAL = 0): iota, constant fill, narrowing copy.
 __global__ void k_iota(int* __restrict__ p, long long n) {
   for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
@@ -622,6 +637,14 @@ cudaError_t launch_rebase(cudaStream_t st, long long* rp_full, int M, int P, con
 }
 
 static int grid_for(long long n) { long long g = (n + 255) / 256; return (int)(g < 1 ? 1 : (g > 4096 ? 4096 : g)); }
+cudaError_t launch_rebase32(cudaStream_t st, int* rp, long long n, const int* first) {
+  if (n > 0) k_rebase32<<<grid_for(n), 256, 0, st>>>(rp, n, first);
+  return cudaGetLastError();
+}
+cudaError_t launch_split_sizes(cudaStream_t st, const int* s, const int* rpA, int P, long long* out) {
+  k_split_sizes<<<1, 256, 0, st>>>(s, rpA, P, out);
+  return cudaGetLastError();
+}
 cudaError_t launch_iota(cudaStream_t st, int* p, long long n) {
   if (n > 0) k_iota<<<grid_for(n), 256, 0, st>>>(p, n);
   return cudaGetLastError();

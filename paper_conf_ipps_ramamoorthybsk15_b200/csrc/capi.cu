@@ -80,6 +80,10 @@ struct spg_ctx {
   int light_max = LIGHT_MAX_DEFAULT, tile_cap = TILE_CAP_DEFAULT, heavy_max = HEAVY_CAP, force = -1;
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
   int thresholds_set = 0;  // light_max / tile_cap set by the caller (else N-dependent defaults)
+  int autotune = 0;        // SPG_OPT_AUTOTUNE: time candidate thresholds on a new structure
+  bool tuned = false;
+  SymKey tuned_key{};
+  int tuned_light = 0, tuned_tile = 0;
   // workspace: analysis (all rows), classification and items (this rank's rows), the plan
   DevBuf f, nz, Tb, Tl, cls, pw, Ro, tflag, tscan, items, lists, small, scan_tmp, plan, fl8, D, ucnt, uscan,
       units, ticket, dub, dscratch, Pf, splits, canonB[4], iota, ones, crow_tmp;
@@ -91,6 +95,9 @@ struct spg_ctx {
   cudaEvent_t ev_fork = nullptr, ev_fork2 = nullptr, ev_join[6] = {};
   cudaEvent_t ev_t[8] = {};
   cudaEvent_t ev_p[4] = {};  // tile path start/end, heavy path start/end
+  cudaEvent_t ev_bval = nullptr;  // values of an asynchronous broadcast are in (numeric waits)
+  bool bval_pending = false;
+  std::vector<long long> scat;  // scatter plan: rows, nnz, first entry per rank (root-side offsets)
   int occ_tile = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1;
   // cached symbolic state
   bool sym_ok = false;
@@ -373,6 +380,7 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   h->host_sym_ok = false;
   long long F_total = -1;
   long long Mloc = 0;
+  int used_light = 0, used_tile = 0;
   Small* ds = h->small.as<Small>();
   long long* crow = reinterpret_cast<long long*>(C_row_ptr);
   for (int attempt = 0;; ++attempt) {
@@ -401,6 +409,8 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
       tile_cap = 1024;
     }
     ClassParams prm{light_max, h->heavy_max, tile_cap, h->force, h->canonical ? 1 : 0};
+    used_light = light_max;
+    used_tile = tile_cap;
     HeavyLists L3;
     for (int b = 0; b < NUM_BINS; ++b) L3.rows[b] = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
     long long* Ro = h->Ro.as<long long>();
@@ -474,6 +484,8 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   for (int b = 0; b < NUM_BINS; ++b) h->counts[b] = hs.counts[b];
   spg_stats& st = h->stats;
   std::memset(&st, 0, sizeof st);
+  st.light_max = used_light;
+  st.tile_flops = used_tile;
   st.flops = 0;
   for (int c = 0; c < NUM_CLS; ++c) st.flops += (int64_t)hs.cstats[NUM_CLS + c];
   st.flops_total = F_total >= 0 ? F_total : st.flops;
@@ -581,6 +593,7 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
   }
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_fork2, cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_bval, cudaEventDisableTiming);
   for (int k = 0; k < 8 && e == cudaSuccess; ++k) e = cudaEventCreate(&h->ev_t[k]);
   if (e != cudaSuccess) {
     h->err = cudaGetErrorString(e);
@@ -632,6 +645,7 @@ spg_status spg_spgemm_free(spg_handle h) {
     }
     if (h->ev_fork) cudaEventDestroy(h->ev_fork);
     if (h->ev_fork2) cudaEventDestroy(h->ev_fork2);
+    if (h->ev_bval) cudaEventDestroy(h->ev_bval);
     for (auto& e : h->ev_t)
       if (e) cudaEventDestroy(e);
     if (h->hr) cudaFreeHost(h->hr);
@@ -676,6 +690,10 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
       h->huge_slots_opt = (int)v;
       break;
     case SPG_OPT_CONCURRENT: h->concurrent = v != 0; break;
+    case SPG_OPT_AUTOTUNE:
+      h->autotune = v != 0;
+      h->tuned = false;
+      break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   h->sym_ok = false;
@@ -694,6 +712,7 @@ spg_status spg_get_option(spg_handle h, spg_option opt, int64_t* v) {
     case SPG_OPT_TIMING: *v = h->timing; break;
     case SPG_OPT_HUGE_SLOTS: *v = h->huge_slots_opt; break;
     case SPG_OPT_CONCURRENT: *v = h->concurrent; break;
+    case SPG_OPT_AUTOTUNE: *v = h->autotune; break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   return SPG_OK;
@@ -724,8 +743,49 @@ spg_status spg_spgemm_symbolic(spg_handle h, const spg_csr* A, const spg_csr* B,
     if (s != SPG_OK) return s;
     Bx = &h->Bc;
   }
+  const SymKey key = make_key(A, B);
+  if (h->autotune && !(h->tuned && h->tuned_key == key)) {
+    // f1 (the threshold is chosen empirically; the paper leaves an
+    // automatic choice to future work): time symbolic + numeric-plan construction for a few
+    // (light_max, tile) candidates on this structure and keep the fastest.  Only the first call
+    // with a new structure pays for it.
+    static const int cand[][2] = {{1024, 3072}, {2048, 2048}, {3072, 1024}, {4096, 2048}, {512, 3584}};
+    const int saved_set = h->thresholds_set, saved_timing = h->timing;
+    float best = 1e30f;
+    int bl = h->light_max, bt = h->tile_cap;
+    h->thresholds_set = 1;
+    h->timing = 0;
+    for (const auto& c : cand) {
+      h->light_max = c[0];
+      h->tile_cap = c[1];
+      float ms = 0.f;
+      for (int rep = 0; rep < 2; ++rep) {  // the first run may size the plan: time the second
+        CK(cudaEventRecord(h->ev_t[5], h->stream));
+        if ((s = symbolic_impl(h, A, Bx, C_row_ptr, nnzC, row_begin, row_end)) != SPG_OK) {
+          h->thresholds_set = saved_set;
+          h->timing = saved_timing;
+          return s;
+        }
+        CK(cudaEventRecord(h->ev_t[6], h->stream));
+        CK(cudaEventSynchronize(h->ev_t[6]));
+        cudaEventElapsedTime(&ms, h->ev_t[5], h->ev_t[6]);
+      }
+      if (ms < best) {
+        best = ms;
+        bl = c[0];
+        bt = c[1];
+      }
+    }
+    h->light_max = bl;
+    h->tile_cap = bt;
+    h->timing = saved_timing;
+    h->tuned = true;
+    h->tuned_key = key;
+    h->tuned_light = bl;
+    h->tuned_tile = bt;
+  }
   s = symbolic_impl(h, A, Bx, C_row_ptr, nnzC, row_begin, row_end);
-  if (s == SPG_OK) h->key = make_key(A, B);
+  if (s == SPG_OK) h->key = key;
   return s;
 }
 
@@ -745,6 +805,10 @@ spg_status spg_spgemm_numeric(spg_handle h, const spg_csr* A, const spg_csr* B, 
     s = h->dtype == SPG_FP64 ? canonicalize<double>(h, B, true) : canonicalize<float>(h, B, true);
     if (s != SPG_OK) return s;
     Bx = &h->Bc;
+  }
+  if (h->bval_pending) {  // values of an asynchronous broadcast: numeric needs them
+    CK(cudaStreamWaitEvent(h->stream, h->ev_bval, 0));
+    h->bval_pending = false;
   }
   return h->dtype == SPG_FP64 ? numeric_impl<double>(h, A, Bx, C_row_ptr, C_col_idx, C_vals)
                               : numeric_impl<float>(h, A, Bx, C_row_ptr, C_col_idx, C_vals);
@@ -868,6 +932,99 @@ spg_status spg_broadcast_csr(spg_handle h, spg_csr* m, int root) {
     NK(ncclBroadcast(m->vals, (void*)m->vals, (size_t)m->nnz, vt, root, h->comm, h->stream));
   }
   NK(ncclGroupEnd());
+  return SPG_OK;
+}
+
+spg_status spg_broadcast_csr_async(spg_handle h, spg_csr* m, int root) {
+  if (!h || !m) return SPG_ERR_INVALID_ARGUMENT;
+  if (!h->comm) return setf(h, SPG_ERR_BAD_STATE, "handle has no communicator (use spg_create_dist)");
+  spg_status s = check_csr(h, m, "matrix", true);
+  if (s != SPG_OK) return s;
+  DeviceGuard g(h->device);
+  const ncclDataType_t vt = h->dtype == SPG_FP64 ? ncclFloat64 : ncclFloat32;
+  // structure on the handle stream (symbolic needs it), values on the communication stream
+  cudaStream_t cs = h->aux[5];
+  NK(ncclGroupStart());
+  NK(ncclBroadcast(m->row_ptr, (void*)m->row_ptr, (size_t)m->nrows + 1, ncclInt32, root, h->comm, h->stream));
+  if (m->nnz) NK(ncclBroadcast(m->col_idx, (void*)m->col_idx, (size_t)m->nnz, ncclInt32, root, h->comm, h->stream));
+  NK(ncclGroupEnd());
+  if (m->nnz) {
+    CK(cudaEventRecord(h->ev_bval, h->stream));  // (NCCL calls of one comm are ordered: after the structure)
+    CK(cudaStreamWaitEvent(cs, h->ev_bval, 0));
+    NK(ncclBroadcast(m->vals, (void*)m->vals, (size_t)m->nnz, vt, root, h->comm, cs));
+    CK(cudaEventRecord(h->ev_bval, cs));
+    h->bval_pending = true;
+  }
+  return SPG_OK;
+}
+
+spg_status spg_scatter_plan(spg_handle h, const spg_csr* A, const spg_csr* B, int root, int32_t* row_begin,
+                            int32_t* row_end, int64_t* nnz_local) {
+  if (!h || !A || !B || !row_begin || !row_end || !nnz_local) return SPG_ERR_INVALID_ARGUMENT;
+  if (!h->comm) return setf(h, SPG_ERR_BAD_STATE, "handle has no communicator (use spg_create_dist)");
+  if (root < 0 || root >= h->nranks) return setf(h, SPG_ERR_INVALID_ARGUMENT, "bad root");
+  if (A->ncols != B->nrows) return setf(h, SPG_ERR_DIMENSION_MISMATCH, "A.ncols (%d) != B.nrows (%d)", A->ncols, B->nrows);
+  DeviceGuard g(h->device);
+  const int P = h->nranks;
+  CK(h->crow_tmp.ensure(sizeof(long long) * (size_t)(3 * P + 1)));
+  long long* d = h->crow_tmp.as<long long>();
+  spg_status s;
+  if (h->rank == root) {  // split points and block sizes from A (root only) and the replicated B
+    if ((s = validate_pair(h, A, B, false)) != SPG_OK) return s;
+    if ((s = ensure_ws(h, A->nrows, A->nnz)) != SPG_OK) return s;
+    if ((s = analysis(h, A, B)) != SPG_OK) return s;
+    if ((s = split_points(h, A->nrows, P)) != SPG_OK) return s;
+    CK(launch_split_sizes(h->stream, h->splits.as<int>(), A->row_ptr, P, d));
+  }
+  NK(ncclBroadcast(d, d, (size_t)(3 * P), ncclInt64, root, h->comm, h->stream));
+  h->scat.assign((size_t)(3 * P), 0);
+  CK(cudaMemcpyAsync(h->scat.data(), d, sizeof(long long) * (size_t)(3 * P), cudaMemcpyDeviceToHost, h->stream));
+  CK(cudaStreamSynchronize(h->stream));
+  long long rb = 0;
+  for (int r = 0; r < h->rank; ++r) rb += h->scat[r];
+  *row_begin = (int32_t)rb;
+  *row_end = (int32_t)(rb + h->scat[h->rank]);
+  *nnz_local = h->scat[P + h->rank];
+  h->sym_ok = false;
+  return SPG_OK;
+}
+
+spg_status spg_scatter_rows(spg_handle h, const spg_csr* A, int root, spg_csr* A_local) {
+  if (!h || !A || !A_local) return SPG_ERR_INVALID_ARGUMENT;
+  if (!h->comm) return setf(h, SPG_ERR_BAD_STATE, "handle has no communicator (use spg_create_dist)");
+  const int P = h->nranks;
+  if ((int)h->scat.size() != 3 * P) return setf(h, SPG_ERR_BAD_STATE, "spg_scatter_rows needs spg_scatter_plan first");
+  const long long rows = h->scat[h->rank], nnz = h->scat[P + h->rank];
+  if (A_local->nrows != rows || A_local->nnz != nnz || !A_local->row_ptr || (nnz && (!A_local->col_idx || !A_local->vals)))
+    return setf(h, SPG_ERR_INVALID_ARGUMENT, "A_local must hold %lld rows and %lld entries", rows, nnz);
+  if (h->rank == root && (!A->row_ptr || (A->nnz && (!A->col_idx || !A->vals))))
+    return setf(h, SPG_ERR_INVALID_ARGUMENT, "A is NULL on the root");
+  DeviceGuard g(h->device);
+  const size_t vb = h->dtype == SPG_FP64 ? 8 : 4;
+  const ncclDataType_t vt = h->dtype == SPG_FP64 ? ncclFloat64 : ncclFloat32;
+  NK(ncclGroupStart());
+  if (h->rank == root) {
+    long long r0 = 0;
+    for (int r = 0; r < P; ++r) {
+      const long long nr = h->scat[r], nz = h->scat[P + r], e0 = h->scat[2 * P + r];
+      NK(ncclSend(A->row_ptr + r0, (size_t)nr + 1, ncclInt32, r, h->comm, h->stream));
+      if (nz) {
+        NK(ncclSend(A->col_idx + e0, (size_t)nz, ncclInt32, r, h->comm, h->stream));
+        NK(ncclSend((const char*)A->vals + (size_t)e0 * vb, (size_t)nz, vt, r, h->comm, h->stream));
+      }
+      r0 += nr;
+    }
+  }
+  NK(ncclRecv((void*)A_local->row_ptr, (size_t)rows + 1, ncclInt32, root, h->comm, h->stream));
+  if (nnz) {
+    NK(ncclRecv((void*)A_local->col_idx, (size_t)nnz, ncclInt32, root, h->comm, h->stream));
+    NK(ncclRecv((void*)A_local->vals, (size_t)nnz, vt, root, h->comm, h->stream));
+  }
+  NK(ncclGroupEnd());
+  // the block's offsets start at rpA[s_rank]: rebase to 0 (the first element is read on the device)
+  CK(h->Pf.ensure(sizeof(int)));
+  CK(cudaMemcpyAsync(h->Pf.p, A_local->row_ptr, sizeof(int), cudaMemcpyDeviceToDevice, h->stream));
+  CK(launch_rebase32(h->stream, (int*)A_local->row_ptr, rows + 1, h->Pf.as<int>()));
   return SPG_OK;
 }
 

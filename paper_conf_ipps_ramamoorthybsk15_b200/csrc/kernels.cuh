@@ -144,6 +144,8 @@ cudaError_t launch_validate(cudaStream_t st, int sms, int M, const int* rp, cons
                             int check_sorted, int* err);
 cudaError_t launch_rebase(cudaStream_t st, long long* rp_full, int M, int P, const int* splits, const long long* off);
 cudaError_t launch_iota(cudaStream_t st, int* p, long long n);
+cudaError_t launch_rebase32(cudaStream_t st, int* rp, long long n, const int* first);
+cudaError_t launch_split_sizes(cudaStream_t st, const int* s, const int* rpA, int P, long long* out);
 template <typename V>
 cudaError_t launch_fill(cudaStream_t st, V* p, long long n, V v);
 cudaError_t launch_narrow(cudaStream_t st, const long long* in, int* out, long long n);

@@ -81,6 +81,16 @@ def test_thresholds_do_not_change_result(heavy_max, tile, light_max):
     compare(A, B, got, ref=ref)
 
 
+def test_autotune_picks_a_candidate_and_keeps_the_result():
+    """SPG_OPT_AUTOTUNE (f1): the first symbolic call on a structure times the candidate
+    thresholds; whichever wins, C is the oracle's (thresholds never change C)."""
+    A, B = W.make("cl10k")
+    got = run_gpu(A, B, autotune=1)
+    compare(A, B, got)
+    st = got[3]
+    assert (st["light_max"], st["tile_flops"]) in [(1024, 3072), (2048, 2048), (3072, 1024), (4096, 2048), (512, 3584)]
+
+
 def test_fp32_power_law():
     A = W.chung_lu(20000, 20000, 2.1, 80000, 3000, 3000, 6.0, 1.1, 5, np.float32)
     B = W.chung_lu(20000, 20000, 3.0, 160000, 1000, 1000, -1.0, 1.0, 6, np.float32)
@@ -194,6 +204,11 @@ def test_error_paths():
         plan.set_option("force_class", 1)
     with pytest.raises(spg.SpgError, match="INVALID_ARGUMENT"):
         plan.set_option("light_max_flops", 5000)  # > TILE_PMAX (4096)
+    # value arrays of another dtype are rejected before they reach the C side (it would read
+    # fp32 data as fp64)
+    dA32 = spg.DeviceCSR(dA.nrows, dA.ncols, dA.row_ptr, dA.col_idx, dA.vals.float())
+    with pytest.raises(TypeError):
+        plan.symbolic(dA32, dB2)
     # validation: unsorted B rows and out-of-range columns are reported, not executed
     plan.set_option("validate", 1)
     Bu = W.random_csr(8, 8, 0.5, 3)
@@ -367,6 +382,95 @@ def test_nccl_single_rank_broadcast_allgatherv():
         compare(A, B, (full.row_ptr.cpu().numpy(), full.col_idx.cpu().numpy(), full.vals.cpu().numpy()))
     finally:
         spg.spg_spgemm_free(h)
+
+
+def test_nccl_single_rank_async_broadcast_and_scatter():
+    """One real NCCL rank: B replicated with the asynchronous broadcast (values overlap symbolic),
+    A != B row blocks scattered from the root (ncclSend/Recv to itself), C = A_local x B."""
+    A = W.chung_lu(6000, 5000, 2.1, 30000, 1500, 1500, 6.0, 1.1, 21)
+    B = W.chung_lu(5000, 7000, 3.0, 40000, 800, 800, -1.0, 1.0, 22)
+    ref = oracle.spgemm(A, B, nthreads=8)
+    uid = spg.spg_get_unique_id()
+    h = spg.spg_create_dist(0, None, torch.float64, uid, 0, 1)
+    try:
+        dA, dB = to_dev(A), to_dev(B)
+        spg.spg_broadcast_csr_async(h, dB, 0)
+        rb, re, nz = spg.spg_scatter_plan(h, dA, dB, 0)
+        assert (rb, re, nz) == (0, A.nrows, A.nnz)
+        loc = spg.DeviceCSR(re - rb, A.ncols, torch.empty(re - rb + 1, dtype=torch.int32, device="cuda"),
+                            torch.empty(nz, dtype=torch.int32, device="cuda"),
+                            torch.empty(nz, dtype=torch.float64, device="cuda"))
+        spg.spg_scatter_rows(h, dA, 0, loc)
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(loc.row_ptr.cpu().numpy(), A.row_ptr)
+        np.testing.assert_array_equal(loc.col_idx.cpu().numpy(), A.col_idx)
+        # symbolic on the dist handle (one rank: all rows), numeric after the async values
+        rp = torch.empty(A.nrows + 1, dtype=torch.int64, device="cuda")
+        nnz, _, _ = spg.spg_spgemm_symbolic(h, loc, dB, rp)
+        col = torch.empty(nnz, dtype=torch.int32, device="cuda")
+        val = torch.empty(nnz, dtype=torch.float64, device="cuda")
+        spg.spg_spgemm_numeric(h, loc, dB, rp, col, val)
+        torch.cuda.synchronize()
+        compare(A, B, (rp.cpu().numpy(), col.cpu().numpy(), val.cpu().numpy()), ref=ref)
+    finally:
+        spg.spg_spgemm_free(h)
+
+
+def _two_process_worker(rank, world, port, out_q):
+    """One process per rank on the SAME GPU: virtual-rank handles (the library's partitioned
+    pipeline) with the process group on gloo; C blocks gathered by dist.allgatherv_c."""
+    import os
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    import torch.distributed as tdist
+    import oracle as O
+    import workloads as WW
+    import paper_conf_ipps_ramamoorthybsk15_b200 as S
+    from paper_conf_ipps_ramamoorthybsk15_b200 import dist as D
+    tdist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    try:
+        A, B = WW.make("cl10k")
+        dA = S.DeviceCSR.from_host(A, "cuda")
+        h = S.spg_create_dist(0, None, torch.float64, None, rank, world)
+        rp = torch.empty(A.nrows + 1, dtype=torch.int64, device="cuda")
+        nnz, rb, re = S.spg_spgemm_symbolic(h, dA, dA, rp)
+        col = torch.empty(max(nnz, 1), dtype=torch.int32, device="cuda")
+        val = torch.empty(max(nnz, 1), dtype=torch.float64, device="cuda")
+        S.spg_spgemm_numeric(h, dA, dA, rp, col, val)
+        torch.cuda.synchronize()
+        splits = S.spg_split_points(h, dA, dA, world)
+        frp, fcol, fval = D.allgatherv_c(rp[: re - rb + 1].cpu().numpy(), col[:nnz].cpu().numpy(),
+                                         val[:nnz].cpu().numpy(), splits)
+        S.spg_spgemm_free(h)
+        t = D.max_over_ranks(float(rank + 1))
+        if rank == 0:
+            ref = O.spgemm(A, B, nthreads=4)
+            err = np.abs(fval - ref[2]) <= 1e-12 * ref[3] if frp[-1] == ref[0][-1] else False
+            out_q.put((np.array_equal(frp, ref[0]), np.array_equal(fcol, ref[1]), bool(np.all(err)), t,
+                       [int(x) for x in splits]))
+    finally:
+        tdist.destroy_process_group()
+
+
+def test_two_processes_virtual_ranks_gloo():
+    import socket
+    import torch.multiprocessing as mp
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_two_process_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(timeout=600)
+        assert p.exitcode == 0
+    rp_ok, col_ok, val_ok, t, splits = q.get(timeout=10)
+    assert rp_ok and col_ok and val_ok and t == 2.0
+    A, B = W.make("cl10k")
+    np.testing.assert_array_equal(splits, oracle.split_points(oracle.row_flops(A, B), 2))
 
 
 # ---- light/medium kernels hand rows to the general kernel: many runs, clustered columns -----

@@ -238,7 +238,8 @@ __global__ void __launch_bounds__(256) k_unit_fill(const int* __restrict__ ucnt,
                                                    int n, NumUnit* __restrict__ units, Small* __restrict__ sm,
                                                    const int* __restrict__ items, const long long* __restrict__ crow,
                                                    const long long* __restrict__ Ro, const uint8_t* __restrict__ cls,
-                                                   const int* __restrict__ rpA, int rb, const int* __restrict__ dub) {
+                                                   const int* __restrict__ rpA, int rb,
+                                                   const long long* __restrict__ dub) {
   for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < n; t += (long long)gridDim.x * blockDim.x) {
     const int u = ucnt[t];
     const long long b = uscan[t] - u;
@@ -248,14 +249,14 @@ __global__ void __launch_bounds__(256) k_unit_fill(const int* __restrict__ ucnt,
     const int sw = wide ? 2 : 1;
     const long long f = (Ro[r2] - P0) / sw;
     const int e0 = rpA[rb + r];
-    const int* db = dub + dub_index(P0, t);
-    const bool sorted = f > c && db[0] >= 0;  // bucketed repeats (k_tile_rank / k_dup_sort)
+    const long long* db = dub + dub_index(P0, t);
+    const bool rep = f > c;
     for (int k = 0; k < u; ++k) {
       NumUnit v;
       v.pw = P0 + (long long)k * NUM_SH * sw;
       v.oc = o0 + (long long)k * NUM_SH;
-      v.dw = P0 + (c + (sorted ? db[k] : 0)) * sw;
-      v.d = sorted ? db[k + 1] - db[k] : (int)(f - c);
+      v.dw = rep ? db[k] : 0;
+      v.d = rep ? (int)(db[k + 1] - db[k]) : 0;
       v.n = (int)min((long long)NUM_SH, c - (long long)k * NUM_SH);
       v.e0 = e0;
       v.ob = k * NUM_SH | (wide ? UNIT_WIDE : 0);
@@ -265,50 +266,45 @@ __global__ void __launch_bounds__(256) k_unit_fill(const int* __restrict__ ucnt,
   if (blockIdx.x == 0 && threadIdx.x == 0) sm->nunits = n > 0 ? uscan[n - 1] : 0;
 }
 
-// Repeats of a heavy row bucketed by numeric unit (counting sort on o / NUM_SH): one block per
-// heavy row, a scratch copy of the (word, output) pairs, then written back in bucket order.
-// dub[dub_index(P0, t) + k] = first repeat of unit k (relative to the row's repeats), k <= hs;
-// dub[...] = -1: not sorted (no repeats, a wide row, or more than DUP_SORT_UNITS units).
+// Repeats of a HUGE (uncached bitmap) row, left unsorted at the end of its plan region with their
+// outputs in D, become R records bucketed by numeric unit (counting sort on o / NUM_SH): one block
+// per row; dub[dub_index(P0, t) + k] = first R record of unit k, k <= hs.
 constexpr int DS_NT = 1024;
-__global__ void __launch_bounds__(DS_NT) k_dup_sort(HeavyLists lists, int c0, int c1, int c2,
-                                                    const long long* __restrict__ crow,
-                                                    const long long* __restrict__ Ro, const uint8_t* __restrict__ cls,
-                                                    const long long* __restrict__ tscan, unsigned* __restrict__ plan,
-                                                    unsigned* __restrict__ D, uint2* __restrict__ scratch,
-                                                    unsigned long long* __restrict__ scratch_head,
-                                                    int* __restrict__ dub) {
-  __shared__ int s_cnt[DUP_SORT_UNITS + 1];
+__global__ void __launch_bounds__(DS_NT) k_dup_sort(HeavyLists lists, int c0, int c1, int c2, SymProb P) {
+  extern __shared__ int s_cnt[];  // [hs + 1]
   __shared__ int scratch_s[DS_NT / 32 + 1];
-  __shared__ unsigned long long s_base;
+  __shared__ long long s_base;
   const Group<DS_NT> g{(int)threadIdx.x, scratch_s};
   const int tid = threadIdx.x;
   int b = blockIdx.x, bin = 0;
   const int cnts[3] = {c0, c1, c2};
   while (b >= cnts[bin]) b -= cnts[bin++];
   const int li = lists.rows[bin][b];
-  const long long t = tscan[li] - 1;
-  const long long o0 = crow[li], c = crow[li + 1] - o0, P0 = Ro[li];
-  int* db = dub + dub_index(P0, t);
-  const bool wide = cls[li] & CLS_WIDE;
-  const long long f = (Ro[li + 1] - P0) >> (wide ? 1 : 0);
+  const long long t = P.tscan[li] - 1;
+  const long long o0 = P.crow[li], c = P.crow[li + 1] - o0, P0 = P.Ro[li];
+  const bool wide = P.cls[li] & CLS_WIDE;
+  const int sw = wide ? 2 : 1;
+  const long long f = (P.Ro[li + 1] - P0) / sw;
   const long long d = f - c;
   const long long hs = (c + NUM_SH - 1) / NUM_SH;
-  if (d <= 0 || wide || hs > DUP_SORT_UNITS) {
-    if (tid == 0) db[0] = -1;
+  if (d <= 0) return;
+  if (hs > DUP_SORT_UNITS) {
+    if (tid == 0) atomicOr(P.err, 4);
     return;
   }
-  if (hs == 1) {  // one unit: already its own bucket
-    if (tid == 0) {
-      db[0] = 0;
-      db[1] = (int)d;
-    }
-    return;
+  long long* db = P.dub + dub_index(P0, t);
+  const int e0 = P.rpA[P.row_begin + li];
+  for (long long k = tid; k <= hs; k += DS_NT) s_cnt[k] = 0;
+  __syncthreads();
+  const long long w0 = P0 + c * sw;  // first repeat's entry
+  for (long long j = tid; j < d; j += DS_NT) atomicAdd(&s_cnt[P.D[w0 + j * sw] / NUM_SH], 1);
+  if (tid == 0) {
+    long long base = (long long)atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)d);
+    if (base + d > P.r_dcap) base = -1;  // too small: the host grows R and reruns
+    s_base = base;
   }
-  for (int k = tid; k <= hs; k += DS_NT) s_cnt[k] = 0;
   __syncthreads();
-  const long long w0 = P0 + c;  // first repeat's word
-  for (long long j = tid; j < d; j += DS_NT) atomicAdd(&s_cnt[D[w0 + j] / NUM_SH], 1);
-  __syncthreads();
+  const long long base = s_base;
   {  // exclusive scan of the bucket sizes (contiguous ownership)
     const int per = (int)((hs + DS_NT) / DS_NT);
     int mine = 0;
@@ -323,37 +319,42 @@ __global__ void __launch_bounds__(DS_NT) k_dup_sort(HeavyLists lists, int c0, in
       if (k < hs) {
         const int v = s_cnt[k];
         s_cnt[k] = run;
-        db[k] = run;
+        db[k] = base + run;
         run += v;
       }
     }
-    if (tid == 0) {
-      db[hs] = tot;
-      s_base = atomicAdd(scratch_head, (unsigned long long)d);
+    if (tid == 0) db[hs] = base + tot;
+  }
+  __syncthreads();
+  if (base < 0) return;
+  for (long long j = tid; j < d; j += DS_NT) {
+    const long long x = w0 + j * sw;
+    const unsigned o = P.D[x];
+    unsigned er, qo;
+    if (wide) {
+      er = P.plan[x];
+      qo = P.plan[x + 1];
+    } else {
+      const unsigned w = P.plan[x];
+      er = w & 0xffffu;
+      qo = w >> 16;
     }
-  }
-  __syncthreads();
-  uint2* tmp = scratch + s_base;
-  for (long long j = tid; j < d; j += DS_NT) {
-    const unsigned o = D[w0 + j];
+    const int e = e0 + (int)er;
     const int pos = atomicAdd(&s_cnt[o / NUM_SH], 1);
-    tmp[pos] = make_uint2(plan[w0 + j], o);
-  }
-  __syncthreads();
-  for (long long j = tid; j < d; j += DS_NT) {
-    const uint2 x = tmp[j];
-    plan[w0 + j] = x.x;
-    D[w0 + j] = x.y;
+    P.R[base + pos] = make_int4(P.Tb[e] + (int)qo, e, (int)o, 0);
   }
 }
 
-cudaError_t launch_dup_sort(cudaStream_t st, const HeavyLists& lists, const int* counts_host, const long long* crow,
-                            const long long* Ro, const uint8_t* cls, const long long* tscan, unsigned* plan,
-                            unsigned* D, uint2* scratch, unsigned long long* scratch_head, int* dub) {
+cudaError_t dup_sort_configure() {
+  return cudaFuncSetAttribute(k_dup_sort, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (DUP_SORT_UNITS + 1) * (int)sizeof(int));
+}
+
+cudaError_t launch_dup_sort(cudaStream_t st, const HeavyLists& lists, const int* counts_host, const SymProb& P) {
   const long long n = (long long)counts_host[0] + counts_host[1] + counts_host[2];
   if (n <= 0) return cudaSuccess;
-  k_dup_sort<<<(unsigned)n, DS_NT, 0, st>>>(lists, counts_host[0], counts_host[1], counts_host[2], crow, Ro, cls, tscan,
-                                           plan, D, scratch, scratch_head, dub);
+  k_dup_sort<<<(unsigned)n, DS_NT, (DUP_SORT_UNITS + 1) * sizeof(int), st>>>(lists, counts_host[0], counts_host[1],
+                                                                             counts_host[2], P);
   return cudaGetLastError();
 }
 
@@ -546,7 +547,7 @@ cudaError_t launch_unit_count(cudaStream_t st, int sms, const int* items, const 
 
 cudaError_t launch_unit_fill(cudaStream_t st, int sms, const int* ucnt, const long long* uscan, int n,
                              NumUnit* units, Small* small, const int* items, const long long* crow,
-                             const long long* Ro, const uint8_t* cls, const int* rpA, int rb, const int* dub) {
+                             const long long* Ro, const uint8_t* cls, const int* rpA, int rb, const long long* dub) {
   k_unit_fill<<<grid_for_rows(n, sms), 256, 0, st>>>(ucnt, uscan, n, units, small, items, crow, Ro, cls, rpA, rb,
                                                      dub);
   return cudaGetLastError();

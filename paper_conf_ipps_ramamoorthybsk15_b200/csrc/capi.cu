@@ -86,7 +86,7 @@ struct spg_ctx {
   int tuned_light = 0, tuned_tile = 0;
   // workspace: analysis (all rows), classification and items (this rank's rows), the plan
   DevBuf f, nz, Tb, Tl, cls, pw, Ro, tflag, tscan, items, lists, small, scan_tmp, plan, fl8, D, ucnt, uscan,
-      units, ticket, dub, dscratch, Pf, splits, canonB[4], iota, ones, crow_tmp;
+      units, ticket, dub, R, Pf, splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
   long long iota_n = -1, ones_n = -1;
@@ -194,8 +194,12 @@ SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* cr
   P.crow = crow;
   P.tscan = h->tscan.as<long long>();
   P.D = h->D.as<unsigned>();
-  P.dub = h->dub.as<int>();
+  P.dub = h->dub.as<long long>();
+  P.R = h->R.as<int4>();
+  P.r_dcap = h->R.p ? (long long)(h->R.cap / sizeof(int4)) : 0;
   P.dups = &h->small.as<Small>()->dups;
+  P.dups_all = &h->small.as<Small>()->dups_all;
+  P.err = &h->small.as<Small>()->err;
   long long r_cap = h->plan_cap();
   P.r_cap = r_cap;
   P.row_begin = h->rb;
@@ -420,7 +424,7 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
                        h->cls.as<uint8_t>(), h->pw.as<int>(), L3, ds));
     CK(launch_incl_scan<int>(h->stream, h->pw.as<int>(), Ro + 1, Mloc, h->scan_tmp.as<long long>()));
     // repeats' bucket starts: index < plan words / NUM_SH + 2 items + 2
-    CK(h->dub.ensure((size_t)(h->plan_cap() / NUM_SH + 2LL * (Mloc + 1) + 4) * sizeof(int)));
+    CK(h->dub.ensure((size_t)(h->plan_cap() / NUM_SH + 2LL * (Mloc + 1) + 4) * sizeof(long long)));
     CK(launch_tile_flags(h->stream, h->sms, h->f.as<int>(), A->row_ptr, h->rb, h->re, tile_cap, h->cls.as<uint8_t>(),
                          Ro, h->tflag.as<int>()));
     CK(launch_incl_scan<int>(h->stream, h->tflag.as<int>(), h->tscan.as<long long>(), Mloc,
@@ -442,35 +446,36 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     if (hs.err & 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "A has a column index outside [0, B.nrows)");
     if (hs.err & 2) return setf(h, SPG_ERR_INDEX_OVERFLOW, "a row of A has too many intermediate products (>= 2^31, or >= 2^30 with 64-bit plan entries)");
     const long long words = h->hr->ncut;
-    if (words <= h->plan_cap()) {
+    const long long rcap = h->R.p ? (long long)(h->R.cap / sizeof(int4)) : 0;
+    if (words <= h->plan_cap() && hs.dups_all <= rcap) {
       h->plan_words = words;
       break;
     }
-    if (attempt > 0) return setf(h, SPG_ERR_OUT_OF_MEMORY, "plan could not be sized");
-    // too small: nothing ran; grow to the exact size and rerun
+    if (attempt > 1) return setf(h, SPG_ERR_OUT_OF_MEMORY, "plan could not be sized");
+    // too small: grow to the exact size and rerun (the first call on a structure)
     CK(h->plan.ensure((size_t)words * sizeof(unsigned)));
     CK(h->D.ensure((size_t)words * sizeof(unsigned)));
     CK(h->fl8.ensure((size_t)words));
+    // repeats: at most the products; the exact count once the plan fitted
+    const long long want = words <= h->plan_cap() && attempt == 0 && hs.dups_all > 0 ? hs.dups_all : words / 16;
+    CK(h->R.ensure((size_t)((want > hs.dups_all ? want : hs.dups_all) + 1024) * sizeof(int4)));
   }
   const Small& hs = h->hr->small;
+  if ((long long)hs.cstats[2 * NUM_CLS] > (long long)NUM_SH * DUP_SORT_UNITS)
+    return setf(h, SPG_ERR_NOT_SUPPORTED, "a row has more than %lld intermediate products",
+                (long long)NUM_SH * DUP_SORT_UNITS);
   h->nnzC = h->hr->nnz;
   h->nitems = hs.nitems;
-  {  // repeats of heavy rows bucketed by numeric unit, then the numeric work units (structure
-     // only: built once, reused by every numeric call)
-    const Small* dsm = h->small.as<Small>();
-    CK(h->dscratch.ensure((size_t)(hs.dups + 1) * sizeof(uint2)));
-    CK(cudaMemsetAsync(&ds->scratch_head, 0, sizeof(unsigned long long), h->stream));
+  {  // repeats of HUGE rows as R records bucketed by numeric unit, then the numeric work units
+     // (structure only: built once, reused by every numeric call)
     HeavyLists HL;
     int hc[NUM_BINS];
     for (int b = 0; b < NUM_BINS; ++b) {  // (register-cached bins bucket their repeats themselves)
       HL.rows[b] = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
       hc[b] = b == BIN_HUGE ? hs.counts[b] : 0;
     }
-    CK(launch_dup_sort(h->stream, HL, hc, crow, h->Ro.as<long long>(), h->cls.as<uint8_t>(), h->tscan.as<long long>(),
-                       h->plan.as<unsigned>(), h->D.as<unsigned>(), h->dscratch.as<uint2>(), &ds->scratch_head,
-                       h->dub.as<int>()));
-    h->launches += 2;
-    (void)dsm;
+    CK(launch_dup_sort(h->stream, HL, hc, make_sym(h, A, B, crow)));
+    h->launches += 1;
     const long long ucap = (long long)hs.nitems + h->nnzC / NUM_SH + 2;
     CK(h->units.ensure((size_t)ucap * sizeof(NumUnit)));
     const int n = hs.nitems;
@@ -478,7 +483,7 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(launch_incl_scan<int>(h->stream, h->ucnt.as<int>(), h->uscan.as<long long>(), n, h->scan_tmp.as<long long>()));
     CK(launch_unit_fill(h->stream, h->sms, h->ucnt.as<int>(), h->uscan.as<long long>(), n, h->units.as<NumUnit>(), ds,
                         h->items.as<int>(), crow, h->Ro.as<long long>(), h->cls.as<uint8_t>(), A->row_ptr, h->rb,
-                        h->dub.as<int>()));
+                        h->dub.as<long long>()));
     h->launches += 2 + scan_launches(n);
   }
   for (int b = 0; b < NUM_BINS; ++b) h->counts[b] = hs.counts[b];
@@ -502,7 +507,7 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
   for (int b = 0; b < NUM_BINS; ++b) nheavy += hs.counts[b];
   st.heavy_rows = nheavy;
   st.tiles = hs.nitems - nheavy;
-  st.dup_products = hs.dups;
+  st.dup_products = hs.dups_all;
   st.plan_bytes = h->plan_words * (int64_t)sizeof(unsigned);
   st.launches_symbolic = h->launches;
   if (h->timing) {
@@ -541,7 +546,7 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
     P.items = h->items.as<int>();
     P.units = h->units.as<NumUnit>();
     P.nunits = &h->small.as<Small>()->nunits;
-    P.D = h->D.as<unsigned>();
+    P.R = h->R.as<int4>();
     P.ticket = h->ticket.as<int>();
     P.row_begin = h->rb;
     P.ccol = C_col;
@@ -585,6 +590,7 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
   cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, device);
   e = tile_configure();
   if (e == cudaSuccess) e = heavy_configure();
+  if (e == cudaSuccess) e = dup_sort_configure();
   if (e == cudaSuccess) e = cudaHostAlloc((void**)&h->hr, sizeof(HostRead), cudaHostAllocDefault);
   for (int c = 0; c < 6 && e == cudaSuccess; ++c) {
     e = cudaStreamCreateWithFlags(&h->aux[c], cudaStreamNonBlocking);
@@ -632,7 +638,7 @@ spg_status spg_spgemm_free(spg_handle h) {
     cudaStreamSynchronize(h->stream);
     DevBuf* bufs[] = {&h->f,     &h->nz,    &h->Tb,    &h->Tl,    &h->cls,    &h->pw,   &h->Ro,    &h->tflag,
                       &h->tscan, &h->items, &h->lists, &h->small, &h->scan_tmp, &h->plan, &h->fl8, &h->D,
-                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->dscratch, &h->Pf,     &h->splits,
+                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->R, &h->Pf,     &h->splits,
                       &h->iota,  &h->ones,  &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();

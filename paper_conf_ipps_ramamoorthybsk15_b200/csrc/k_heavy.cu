@@ -15,10 +15,11 @@
 //           output in D at the same word).
 //   c_i     = claimed bits (summed over column tiles).
 // HEAVY rows (f <= 8192, one gather chunk) keep their products (column) in registers across
-// the passes and their head flags in a shared bit array, and place their repeats after the
-// outputs bucketed by numeric unit at the end of the row; HUGE rows re-gather columns per pass,
-// keep the flag in a global byte per product (fl8) between pass 1 and pass 2, and leave their
-// repeats unsorted at the end of the region (k_dup_sort buckets them after symbolic).  Products are
+// the passes and their head flags in a shared bit array, and write their repeats as R records
+// {B entry, A entry, output} bucketed by numeric unit at the end of the row; HUGE rows re-gather
+// columns per pass, keep the flag in a global byte per product (fl8) between pass 1 and pass 2,
+// and leave their repeats unsorted at the end of the plan region with the outputs in D
+// (k_dup_sort turns them into R records after symbolic).  Products are
 // visited in 32-product warp windows (coalesced within a B row); the run of each lane comes from
 // a REDUX.OR mask of run starts.  SINGLE rows (one non-empty B row) only copy their run.
 #include "kernels.cuh"
@@ -78,6 +79,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
   __shared__ int s_next;
   __shared__ int s_dcnt, s_single;
   __shared__ int s_uc[HEAVY_CAP / NUM_SH + 2];  // cached rows: repeats per numeric unit
+  __shared__ long long s_rbase;
   for (;;) {
     if (tid == 0) s_next = atomicAdd(const_cast<int*>(count) + 8, 1);
     __syncthreads();
@@ -407,27 +409,31 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
         for (int s = 0; s < BMP_SLOTS; ++s)
           if (dmask >> s & 1u) atomicAdd(&s_uc[oo[s] / NUM_SH], 1);
         __syncthreads();
-        if (tid == 0) {
-          int* db = P.dub + dub_index(ro, P.tscan[li] - 1);
+        if (tid == 0) {  // R records, first one per numeric unit in dub
+          long long base = (long long)atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)(f - out));
+          if (base + (f - out) > P.r_dcap) base = -1;  // too small: the host grows R and reruns
+          s_rbase = base;
+          long long* db = P.dub + dub_index(ro, P.tscan[li] - 1);
           int run = 0;
           for (int k = 0; k < hs; ++k) {
             const int v = s_uc[k];
             s_uc[k] = run;
-            db[k] = run;
+            db[k] = base + run;
             run += v;
           }
-          db[hs] = run;
+          db[hs] = base + run;
         }
         __syncthreads();
+        const long long rbase = s_rbase;
 #pragma unroll
         for (int s = 0; s < BMP_SLOTS; ++s) {
           const int j0 = warp * 32 + s * NT;
           if (j0 < Lt) {  // warp-uniform
             const int r = lane_run(j0);
-            if (dmask >> s & 1u) {
-              const int pos = out + atomicAdd(&s_uc[oo[s] / NUM_SH], 1);
-              put(pos, sae[r] - pa0, j0 + lane - seg[r]);
-              P.D[ro + pos] = (unsigned)oo[s];
+            if ((dmask >> s & 1u) && rbase >= 0) {
+              const int pos = atomicAdd(&s_uc[oo[s] / NUM_SH], 1);
+              const int qo = j0 + lane - seg[r];
+              P.R[rbase + pos] = make_int4(sbs[r] + qo, sae[r], oo[s], 0);
             }
           }
         }
@@ -435,7 +441,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
     }
     if (tid == 0) {
       P.crow[li + 1] = out;
-      if (f > out) atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)(f - out));
+      if (f > out) atomicAdd(reinterpret_cast<unsigned long long*>(P.dups_all), (unsigned long long)(f - out));
     }
     __syncthreads();
   }

@@ -23,10 +23,9 @@
 //   6. offsets   block scan of c_j: the output offset of every row inside its tile.
 //   7. ranks     rank = heads of the row's earlier buckets + distinct smaller columns in the own
 //                bucket; a head writes its plan word at P0_tile + out_j + rank (C order), every
-//                other product after the tile's outputs (the dups, each with its output
-//                out_j + rank in D at the same word), bucketed by the numeric unit that owns that
-//                output.  SINGLE rows (one non-empty B row, already sorted) write their products
-//                in order.
+//                other product (a repeat) an R record {B entry, A entry, output out_j + rank},
+//                bucketed by the numeric unit that owns that output.  SINGLE rows (one non-empty
+//                B row, already sorted) write their products in order.
 // This is Phase IV's "sort, mark like-tuples, scan, compact", done per batch
 // in shared memory.
 #include "kernels.cuh"
@@ -113,7 +112,7 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
   __shared__ int s_t0, s_qr0[BATCH_NI + 1], s_qheavy[BATCH_NI], s_qp[BATCH_NI], s_qe0[BATCH_NI];
   __shared__ long long s_qP0[BATCH_NI + 1];
   __shared__ int s_nb, s_bi[BATCH_NI], s_irb[BATCH_NI + 1], s_ie0[BATCH_NI], s_iub[BATCH_NI + 1], s_inext;
-  __shared__ long long s_iP0[BATCH_NI];
+  __shared__ long long s_iP0[BATCH_NI], s_idb[BATCH_NI];
   __shared__ int s_uc[BATCH_NU];
   constexpr int NT = TILE_NT, NW = NT / 32;
   const Group<NT> g{(int)threadIdx.x, scratch};
@@ -428,7 +427,7 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
           ub += (C + NUM_SH - 1) / NUM_SH;
         }
         s_iub[NI] = ub;
-        if (dups) atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)dups);
+        if (dups) atomicAdd(reinterpret_cast<unsigned long long*>(P.dups_all), (unsigned long long)dups);
       }
       if (tid < BATCH_NU) s_uc[tid] = 0;
       __syncthreads();
@@ -462,21 +461,25 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
           P.plan[s_iP0[it] + s_out[j] - s_out[s_irb[it]] + idx - s_pf[j]] = pay[idx];
         }
       __syncthreads();
-      if (tid < NI) {  // bucket starts of the tile's repeats (also for numeric: dub)
+      if (tid < NI) {  // R records of the tile's repeats, bucketed by numeric unit (dub: first record)
         const int x = tid;
         const int C = s_out[s_irb[x + 1]] - s_out[s_irb[x]];
         const int F = s_pf[s_irb[x + 1]] - s_pf[s_irb[x]];
+        s_idb[x] = -1;
         if (F > C) {
-          int* db = P.dub + dub_index(s_iP0[x], t0 + s_bi[x]);
+          long long base = (long long)atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)(F - C));
+          if (base + (F - C) > P.r_dcap) base = -1;  // too small: the host grows R and reruns
+          s_idb[x] = base;
+          long long* db = P.dub + dub_index(s_iP0[x], t0 + s_bi[x]);
           const int hs = (C + NUM_SH - 1) / NUM_SH;
           int run = 0;
           for (int k = 0; k < hs; ++k) {
             const int v = s_uc[s_iub[x] + k];
             s_uc[s_iub[x] + k] = run;
-            db[k] = run;
+            db[k] = base + run;
             run += v;
           }
-          db[hs] = run;
+          db[hs] = base + run;
         }
       }
       __syncthreads();
@@ -484,10 +487,11 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
         if (keys[x] < 0) {
           const int o = sbk[x], idx = sidx[x];
           const int it = s_item[exrow[idx]];
-          const int C = s_out[s_irb[it + 1]] - s_out[s_irb[it]];
-          const int pos = C + atomicAdd(&s_uc[s_iub[it] + o / NUM_SH], 1);
-          P.plan[s_iP0[it] + pos] = pay[idx];
-          P.D[s_iP0[it] + pos] = (unsigned)o;
+          if (s_idb[it] < 0) continue;
+          const int pos = atomicAdd(&s_uc[s_iub[it] + o / NUM_SH], 1);
+          const unsigned w = pay[idx];
+          const int e = s_ie0[it] + (int)(w & 0xffffu);
+          P.R[s_idb[it] + pos] = make_int4(P.Tb[e] + (int)(w >> 16), e, o, 0);
         }
       __syncthreads();
     }

@@ -4,8 +4,9 @@
 // The symbolic phase sorted every item's products by (row, column) and left the plan: for an
 // item (a tile of consecutive rows, or one heavy row) with plan region [P0, P0 + f) and outputs
 // [o0, o0 + c), plan word P0 + o describes output o0 + o — {e_rel, qoff}: the A entry e0 + e_rel
-// and the offset of the B entry inside that entry's B row — and words c..f-1 of the region are
-// the item's repeated products (dups), each with its item-relative output in D at the same word.
+// and the offset of the B entry inside that entry's B row.  The item's repeated products (a
+// product whose column another product of its row already produced) are 16-byte records
+// {B entry, A entry, item-relative output} in R, bucketed by the numeric unit owning the output.
 //
 // So numeric is a stream in C order (Phase IV of PAPER.md L154-156, "add like-tuples and
 // compact", with the sort done once in symbolic).  Persistent warps take work units (NUM_SH
@@ -16,9 +17,9 @@
 //   outputs   per output one plan word (shared memory), the A entry's B-row start Tb[e] and value
 //             valA[e] (the item's A entries: L1), the B gather (column and value, L2: B rows are
 //             consumed in ascending order), one multiply, two coalesced streaming stores.
-//   repeats   the unit scans the item's dup outputs in D (a few KB, L1/L2) and adds a·b for those
-//             inside its own outputs with RED.ADD.F64/F32 — into lines it just wrote (L2), ordered
-//             after its stores by __syncwarp; no unit ever waits for another.
+//   repeats   the unit's repeat records (16-byte {B entry, A entry, output}, bucketed by unit in
+//             symbolic) add a·b into its own outputs with RED.ADD.F64/F32 — into lines it just
+//             wrote (L2), ordered after its stores by __syncwarp; no unit ever waits for another.
 // HBM traffic per output: 4 B of plan read + (4 + sizeof(V)) B of C written; A and B once.
 #include "kernels.cuh"
 
@@ -148,27 +149,12 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
         }
     }
     __syncwarp();  // every lane is done with buffer cb, and its stores precede the adds below
-    // ---- repeated products of the item that land in this unit's outputs ------------------------
+    // ---- repeated products landing in this unit's outputs (R records: B entry, A entry, output) -
     if (cur.d > 0) {
-      const int ob = cur.ob & (UNIT_WIDE - 1);
-      const int sw = wide ? 2 : 1;
-      V* __restrict__ cv0 = cval - ob;
+      V* __restrict__ cv0 = cval - (cur.ob & (UNIT_WIDE - 1));
       for (int j = lane; j < cur.d; j += 32) {
-        const long long x = cur.dw + (long long)j * sw;
-        const int o = (int)__ldg(P.D + x);
-        if ((unsigned)(o - ob) >= (unsigned)n) continue;
-        unsigned er, qo;
-        if (!wide) {
-          const unsigned wd = __ldg(P.plan + x);
-          er = wd & 0xffffu;
-          qo = wd >> 16;
-        } else {
-          er = __ldg(P.plan + x);
-          qo = __ldg(P.plan + x + 1);
-        }
-        const int e = e0 + (int)er;
-        const int q = __ldg(P.Tb + e) + (int)qo;
-        atomicAdd(cv0 + o, __ldg(P.valA + e) * __ldg(P.valB + q));
+        const int4 x = __ldg(P.R + cur.dw + j);
+        atomicAdd(cv0 + x.z, __ldg(P.valA + x.y) * __ldg(P.valB + x.x));
       }
     }
     if (!more) break;

@@ -42,9 +42,9 @@ struct Small {
   int err;
   int amax;                 // longest row of A
   int tqhead;               // tiles: dynamic queue head
-  long long dups;           // repeated products (statistics)
+  long long dups;           // repeat records reserved (R entries)
+  long long dups_all;       // repeated products (statistics)
   long long nunits;         // numeric work units
-  unsigned long long scratch_head;  // k_dup_sort scratch reservation
   unsigned long long hist[65];
   unsigned long long cstats[2 * NUM_CLS + 2];
 };
@@ -65,30 +65,33 @@ struct SymProb {
   uint8_t* fl8;             // uncached bitmap rows: first-claim flag per product (Ro_i + offset)
   long long* crow;          // C row offsets (local); symbolic writes counts at [li + 1]
   const long long* tscan;   // inclusive scan of the item-start flags: item of row li = tscan[li] - 1
-  unsigned* D;              // item-relative output of the repeated product whose plan entry starts
-                            // at the same word (sized like the plan, written only for repeats)
-  int* dub;                 // repeats' bucket starts per numeric unit (dub_index(P0, t) + k)
-  long long* dups;          // repeated-product counter (statistics)
+  unsigned* D;              // HUGE rows: item-relative output of the repeated product whose plan
+                            // entry starts at the same word (written only for their repeats)
+  long long* dub;           // repeats' first R record per numeric unit (dub_index(P0, t) + k)
+  int4* R;                  // repeat records {B entry, A entry, item-relative output, 0}
+  long long r_dcap;         // R capacity (records); beyond it nothing is written (host grows, reruns)
+  long long* dups;          // R reservation counter
+  long long* dups_all;      // repeated-product counter (statistics)
+  int* err;                 // error bits (Small::err)
   long long r_cap;          // plan capacity (words); the kernels do nothing if Ro[Mloc] > r_cap
   int row_begin, row_end;
 };
 
 // Numeric work units, in a list built in item order: item t has ceil(c_t / NUM_SH) units, unit k
 // owning outputs [k NUM_SH, (k + 1) NUM_SH) of the item.  A unit stores its outputs, then adds
-// the item's repeated products (d_t = f_t - c_t plan entries after the outputs, each with its
-// output in D) that land in its own outputs: a warp only ever adds into outputs it stored
-// itself, so no unit waits for another.  The repeats are bucketed by unit (tiles: in k_tile_rank;
-// heavy rows: k_dup_sort after symbolic), bucket starts in dub[dub_index(P0, t) + k], so a unit
-// reads only its bucket; rows with dub[...] = -1 (wide, or more than DUP_SORT_UNITS units) keep
-// them unsorted and every unit of the row filters the list.
+// the item's repeated products (d_t = f_t - c_t) that land in its own outputs: a warp only ever
+// adds into outputs it stored itself, so no unit waits for another.  The repeats are 16-byte
+// records {B entry, A entry, item-relative output} in R, bucketed by unit (tiles: k_tile_rank;
+// register-cached heavy rows: k_bitmap_rank; HUGE rows: k_dup_sort after symbolic); unit k's
+// records start at R[dub[dub_index(P0, t) + k]].
 constexpr int NUM_SH = 512;
-constexpr int DUP_SORT_UNITS = 1024;   // heavy rows with more units keep their repeats unsorted
+constexpr int DUP_SORT_UNITS = 48 * 1024;   // k_dup_sort's shared counters (rows up to 24M outputs)
 __host__ __device__ __forceinline__ long long dub_index(long long P0, long long t) { return P0 / NUM_SH + 2 * t; }
 struct NumUnit {
   long long pw;   // plan word of the unit's first output
   long long oc;   // C offset (local) of the unit's first output
-  long long dw;   // plan word of the item's first repeated product
-  int d;          // repeated products of the item
+  long long dw;   // first R record of the unit's repeats
+  int d;          // repeats landing in the unit's outputs
   int n;          // outputs of the unit
   int e0;         // first A entry of the item
   int ob;         // item-relative output of the unit's first output | UNIT_WIDE
@@ -110,7 +113,7 @@ struct NumProb {
   const int* __restrict__ items;        // ordered item starts (local rows) + sentinel
   const NumUnit* __restrict__ units;
   const long long* __restrict__ nunits;
-  const unsigned* __restrict__ D;
+  const int4* __restrict__ R;           // repeat records
   int* ticket;                          // work-unit queue head (zeroed before the launch)
   int row_begin;
   int* ccol;
@@ -123,10 +126,9 @@ cudaError_t launch_row_flops(cudaStream_t st, int M, const int* rpA, const int* 
 cudaError_t launch_unit_count(cudaStream_t st, int sms, const int* items, const long long* crow, int n, int* ucnt);
 cudaError_t launch_unit_fill(cudaStream_t st, int sms, const int* ucnt, const long long* uscan, int n,
                              NumUnit* units, Small* small, const int* items, const long long* crow,
-                             const long long* Ro, const uint8_t* cls, const int* rpA, int rb, const int* dub);
-cudaError_t launch_dup_sort(cudaStream_t st, const HeavyLists& lists, const int* counts_host, const long long* crow,
-                            const long long* Ro, const uint8_t* cls, const long long* tscan, unsigned* plan,
-                            unsigned* D, uint2* scratch, unsigned long long* scratch_head, int* dub);
+                             const long long* Ro, const uint8_t* cls, const int* rpA, int rb, const long long* dub);
+cudaError_t dup_sort_configure();
+cudaError_t launch_dup_sort(cudaStream_t st, const HeavyLists& lists, const int* counts_host, const SymProb& P);
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
                             const ClassParams& prm, uint8_t* cls, int* pw, const HeavyLists& lists, Small* small);
 cudaError_t launch_tile_flags(cudaStream_t st, int sms, const int* f, const int* rpA, int rb, int re, int tile_cap,

@@ -103,6 +103,9 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
     }
     const bool wide = cur.ob & UNIT_WIDE;
     const int e0 = cur.e0, n = cur.n;
+    // the first 32 repeat records: fetched now, used after the outputs
+    int4 rec = make_int4(0, 0, 0, 0);
+    if (lane < cur.d) rec = __ldg(P.R + cur.dw + lane);
     // ---- outputs in C order -----------------------------------------------------------------------
     int* __restrict__ ccol = P.ccol + cur.oc;
     V* __restrict__ cval = P.cval + cur.oc;
@@ -152,7 +155,8 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
     // ---- repeated products landing in this unit's outputs (R records: B entry, A entry, output) -
     if (cur.d > 0) {
       V* __restrict__ cv0 = cval - (cur.ob & (UNIT_WIDE - 1));
-      for (int j = lane; j < cur.d; j += 32) {
+      if (lane < cur.d) atomicAdd(cv0 + rec.z, __ldg(P.valA + rec.y) * __ldg(P.valB + rec.x));
+      for (int j = 32 + lane; j < cur.d; j += 32) {
         const int4 x = __ldg(P.R + cur.dw + j);
         atomicAdd(cv0 + x.z, __ldg(P.valA + x.y) * __ldg(P.valB + x.x));
       }

@@ -43,6 +43,7 @@ def _load():
         common = [_I32, _I32, _I32, _P, _P, _P, _I32, _P, _P, _P, ctypes.c_int]
         lib.orc_spgemm_count.argtypes = common + [_P, ctypes.c_int]
         lib.orc_spgemm_fill.argtypes = common + [_P, _P, _P, _P, ctypes.c_int]
+        lib.orc_csrmm.argtypes = [_I32, _P, _P, _P, ctypes.c_int, _P, ctypes.c_int64, _P, _P]
         _lib = lib
     return _lib
 
@@ -113,3 +114,18 @@ def spgemm(A, B, r0: int = 0, r1: int | None = None, nthreads: int = 1, with_abs
     _load().orc_spgemm_fill(*args, rp.ctypes.data, col.ctypes.data, val.ctypes.data,
                             ab.ctypes.data if with_abs else None, nthreads)
     return rp, col, val, ab
+
+
+def csrmm(A, D: np.ndarray):
+    """Sparse x dense C = A x D (PAPER.md L289's CSTMM): (C float64 [M, n], abs float64 [M, n])."""
+    D = np.ascontiguousarray(D, dtype=np.float64)
+    assert D.ndim == 2 and D.shape[0] == A.ncols, "dimension mismatch"
+    is64 = 1 if np.dtype(A.vals.dtype) == np.float64 else 0
+    vdt = np.float64 if is64 else np.float32
+    rp, ci, v = _c(A.row_ptr, np.int32), _c(A.col_idx, np.int32), _c(A.vals, vdt)
+    n = D.shape[1]
+    C = np.empty((A.nrows, n), np.float64)
+    ab = np.empty((A.nrows, n), np.float64)
+    _load().orc_csrmm(A.nrows, rp.ctypes.data, ci.ctypes.data, v.ctypes.data, is64, D.ctypes.data, n,
+                      C.ctypes.data, ab.ctypes.data)
+    return C, ab

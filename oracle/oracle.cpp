@@ -14,6 +14,9 @@
 //   * Multi-GPU split points (reading R10): s_0 = 0, s_P = M,
 //     s_r = min{ i : Pf[i]*P >= r*F }, Pf the exclusive prefix of f.
 //   * Log2 flop bins: bin = -1 if f = 0 else ceil(log2 f).
+//   * Sparse x dense (CSTMM / csrmm, the extension named in PAPER.md L289, §VI):
+//       C(i,:) = sum_k A(i,k) * D(k,:) over the stored entries of row i of A — the same Row-Row
+//     formulation with a dense right operand; C is dense.
 //
 // Values are promoted to double; for each output entry the oracle also returns
 // abs = sum |a*b| so that tests can apply the per-entry bound |gpu - sum| <= rtol * abs.
@@ -147,6 +150,24 @@ void orc_spgemm_fill(int32_t r0, int32_t r1, int32_t M, const int32_t* rpA, cons
       }
     }
   });
+}
+
+// Sparse x dense: C (M x n, row-major, double) = A (CSR) x D (K x n, row-major, double), rows
+// [0, M); absv = sum |A(i,k) * D(k,j)| per entry (tolerance bound).  Plain row loop.
+void orc_csrmm(int32_t M, const int32_t* rpA, const int32_t* colA, const void* valA, int is_f64, const double* D,
+               int64_t n, double* C, double* absv) {
+  Mat A{M, rpA, colA, valA, is_f64};
+  for (int32_t i = 0; i < M; ++i)
+    for (int64_t j = 0; j < n; ++j) {
+      double s = 0.0, t = 0.0;
+      for (int64_t p = A.rp[i]; p < A.rp[i + 1]; ++p) {
+        const double x = A.val(p) * D[(int64_t)A.ci[p] * n + j];
+        s += x;
+        t += x < 0 ? -x : x;
+      }
+      C[(int64_t)i * n + j] = s;
+      absv[(int64_t)i * n + j] = t;
+    }
 }
 
 }  // extern "C"

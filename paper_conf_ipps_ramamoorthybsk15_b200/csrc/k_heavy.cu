@@ -163,8 +163,12 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
 
     // product window [j0, j0+32): run of each lane (runs starting inside the window form a
     // bitmask, REDUX.OR; a lane's run = the window's first run + popcount of starts <= it)
+    // B-side classes (the paper's B_H / B_L split): a window inside one
+    // long B row (B_H: in a heavy row the longest B row holds ~80% of the products) is that row
+    // for every lane; only windows over short B rows (B_L) pay for the run-start mask.
     auto lane_run = [&](int j0) {
       const int rb = (j0 >> 5) < BMP_CTCAP ? (int)ctab[j0 >> 5] : upper_idx(seg, nz, j0);
+      if (seg[rb + 1] >= j0 + 32) return rb;  // warp-uniform
       const int rs = rb + 1 + lane;
       const int d = rs <= nz ? seg[rs] - j0 : 32;
       const unsigned M = __reduce_or_sync(FULL, (d >= 1 && d <= 31) ? (1u << d) : 0u);

@@ -267,3 +267,46 @@ def test_split_points_large_values():
     f = np.array([2**40, 1, 2**40, 3], np.int64)
     s = oracle.split_points(f, 2)
     assert list(s) == [0, 3, 4]   # Pf = [0, 2^40, 2^40+1, 2^41+1, 2^41+4]
+
+
+# --- sparse x dense (csrmm) ------------------------------------------------------
+@pytest.mark.parametrize("seed", range(4))
+@pytest.mark.parametrize("shape", [(7, 5, 3), (12, 12, 33), (1, 9, 1), (9, 1, 4), (20, 16, 70)])
+def test_csrmm_dense_triple_loop(seed, shape):
+    """Against a textbook triple loop over the dense form of A (signed small integers: exact)."""
+    M, K, n = shape
+    A = W.random_csr(M, K, 0.35, seed, values="int", empty_row_frac=0.2)
+    D = np.random.default_rng(seed).integers(-8, 9, size=(K, n)).astype(np.float64)
+    Ad = csr_to_dense(A)
+    ref = np.zeros((M, n))
+    for i in range(M):
+        for j in range(n):
+            for k in range(K):
+                ref[i, j] += Ad[i, k] * D[k, j]
+    C, ab = oracle.csrmm(A, D)
+    np.testing.assert_array_equal(C, ref)
+    np.testing.assert_array_equal(ab, np.abs(Ad) @ np.abs(D))
+
+
+def test_csrmm_identity_and_duplicates():
+    """I x D = D; duplicate stored entries of A add (Gustavson semantics)."""
+    D = np.random.default_rng(3).standard_normal((6, 5))
+    C, _ = oracle.csrmm(identity(6), D)
+    np.testing.assert_array_equal(C, D)
+    A = W.CSR(1, 6, np.array([0, 3], np.int32), np.array([2, 2, 4], np.int32), np.array([1.0, 2.0, -1.0]))
+    C, ab = oracle.csrmm(A, D)
+    np.testing.assert_allclose(C[0], 3.0 * D[2] - D[4], rtol=1e-15)
+    np.testing.assert_allclose(ab[0], 3.0 * np.abs(D[2]) + np.abs(D[4]), rtol=1e-15)
+
+
+def test_csrmm_matches_spgemm_with_dense_b():
+    """A x D equals the SpGEMM oracle's A x B with B the CSR form of D (all entries stored)."""
+    A = W.random_csr(15, 10, 0.3, 4)
+    D = np.random.default_rng(4).uniform(1, 2, size=(10, 7))
+    B = dense_to_csr(D)
+    rp, col, val, _ = oracle.spgemm(A, B)
+    C, _ = oracle.csrmm(A, D)
+    Cs = np.zeros_like(C)
+    for i in range(15):
+        Cs[i, col[rp[i]:rp[i + 1]]] = val[rp[i]:rp[i + 1]]
+    np.testing.assert_allclose(C, Cs, rtol=1e-14)

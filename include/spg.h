@@ -117,10 +117,12 @@ typedef enum {
   SPG_OPT_TIMING = 6,           /* 1: record per-phase CUDA-event times into the stats        */
   SPG_OPT_HUGE_SLOTS = 7,       /* max concurrent heavy-row blocks per bin (0 = full occupancy) */
   SPG_OPT_CONCURRENT = 8,       /* 1 (default): light and heavy kernels on concurrent streams  */
-  SPG_OPT_AUTOTUNE = 9          /* 1: the first symbolic call on a new A/B structure times five
+  SPG_OPT_AUTOTUNE = 9,         /* 1: the first symbolic call on a new A/B structure times five
                                    (LIGHT_MAX_FLOPS, TILE_FLOPS) candidates and keeps the fastest
                                    (spg_stats.light_max / tile_flops report the choice); 0
                                    (default): the fixed defaults above                         */
+  SPG_OPT_CSRMM_LIGHT_NNZ = 10  /* spg_csrmm: rows with more stored entries are heavy (a block
+                                   per row), the rest light (a warp per row); default 256      */
 } spg_option;
 
 typedef struct {
@@ -180,6 +182,15 @@ spg_status spg_spgemm_symbolic(spg_handle h, const spg_csr* A, const spg_csr* B,
  * (re-run numeric on new values with the same structure).  Asynchronous. */
 spg_status spg_spgemm_numeric(spg_handle h, const spg_csr* A, const spg_csr* B, const int64_t* C_row_ptr,
                               int32_t* C_col_idx, void* C_vals);
+
+/* ---- sparse x dense (the CSTMM extension) ------------------------------ */
+/* C = A x D with A CSR (device, the handle's dtype), D dense K x n row-major (leading dimension
+ * ldd >= n), C dense M x n row-major (ldc >= n), both device pointers.  C(i,:) = sum_k
+ * A(i,k) D(k,:) (Row-Row); rows with <= SPG_OPT_CSRMM_LIGHT_NNZ stored entries run
+ * one warp per row, longer rows one thread block per row.  Every C(i,j) is written (0 for empty
+ * rows).  Asynchronous on the handle's stream; the summation order of a heavy row's entries is
+ * fixed (deterministic). */
+spg_status spg_csrmm(spg_handle h, const spg_csr* A, const void* D, int64_t ldd, int32_t n, void* C, int64_t ldc);
 
 /* ---- SpGEMM (host pointers; the end-to-end path) ------------------------------------ */
 /* Copies A and B (host) into handle-owned device buffers, runs symbolic, copies C's row

@@ -26,13 +26,14 @@ CLASS_NAMES = ["empty", "single", "tiny", "light", "medium", "heavy", "huge"]
 NUM_CLASSES = 7
 # options
 OPTIONS = {"light_max_flops": 0, "tile_flops": 1, "heavy_max_flops": 2, "force_class": 3, "validate": 4,
-           "input_canonical": 5, "timing": 6, "huge_slots": 7, "concurrent": 8, "autotune": 9}
+           "input_canonical": 5, "timing": 6, "huge_slots": 7, "concurrent": 8, "autotune": 9,
+           "csrmm_light_nnz": 10}
 
 EXPORTED = ["spg_create", "spg_set_option", "spg_get_option", "spg_spgemm_free", "spg_last_error", "spg_get_stats",
             "spg_version", "spg_spgemm_symbolic", "spg_spgemm_numeric", "spg_spgemm_host_symbolic",
             "spg_spgemm_host_numeric", "spg_get_unique_id", "spg_create_dist", "spg_broadcast_csr",
             "spg_allgather_nnz", "spg_allgatherv_c", "spg_split_points", "spg_broadcast_csr_async",
-            "spg_scatter_plan", "spg_scatter_rows"]
+            "spg_scatter_plan", "spg_scatter_rows", "spg_csrmm"]
 
 
 class spg_csr(ctypes.Structure):
@@ -106,6 +107,7 @@ def load(build_if_missing: bool = True):
         "spg_scatter_plan": [H, POINTER(spg_csr), POINTER(spg_csr), c_int, POINTER(c_int32), POINTER(c_int32),
                              POINTER(c_int64)],
         "spg_scatter_rows": [H, POINTER(spg_csr), c_int, POINTER(spg_csr)],
+        "spg_csrmm": [H, POINTER(spg_csr), P, c_int64, c_int32, P, c_int64],
     }
     for name, args in sig.items():
         fn = getattr(lib, name)
@@ -279,6 +281,32 @@ def spg_create_dist(device: int, stream, dtype, uid, rank: int, nranks: int) -> 
 def spg_broadcast_csr(h, m: DeviceCSR, root: int):
     c = m.c()
     _check(h, load().spg_broadcast_csr(h, byref(c), root))
+
+
+def spg_csrmm(h, A: DeviceCSR, D: torch.Tensor, C: torch.Tensor):
+    """C (M x n) = A x D (K x n); D and C row-major device tensors (strided rows allowed)."""
+    assert D.dim() == 2 and C.dim() == 2 and D.stride(1) == 1 and C.stride(1) == 1
+    assert D.shape[0] == A.ncols and C.shape == (A.nrows, D.shape[1])
+    a = A.c()
+    _check(h, load().spg_csrmm(h, byref(a), c_void_p(D.data_ptr() if D.numel() else None), D.stride(0),
+                               int(D.shape[1]), c_void_p(C.data_ptr() if C.numel() else None), C.stride(0)))
+
+
+def csrmm(A: DeviceCSR, D: torch.Tensor, **options) -> torch.Tensor:
+    """C = A x D (sparse x dense) on A's device (one-shot handle)."""
+    dt = A.vals.dtype
+    if D.dtype != dt:
+        raise TypeError(f"D must be {dt}")
+    h = spg_create(A.row_ptr.device.index or 0, None, dt)
+    try:
+        for k, v in options.items():
+            spg_set_option(h, k, v)
+        C = torch.empty(A.nrows, D.shape[1], dtype=dt, device=A.row_ptr.device)
+        spg_csrmm(h, A, D.contiguous(), C)
+        torch.cuda.current_stream().synchronize()
+        return C
+    finally:
+        spg_spgemm_free(h)
 
 
 def spg_broadcast_csr_async(h, m: DeviceCSR, root: int):

@@ -81,12 +81,13 @@ struct spg_ctx {
   int validate = 0, canonical = 1, timing = 0, huge_slots_opt = 0, concurrent = 1;
   int thresholds_set = 0;  // light_max / tile_cap set by the caller (else N-dependent defaults)
   int autotune = 0;        // SPG_OPT_AUTOTUNE: time candidate thresholds on a new structure
+  int csrmm_light = 256;   // SPG_OPT_CSRMM_LIGHT_NNZ
   bool tuned = false;
   SymKey tuned_key{};
   int tuned_light = 0, tuned_tile = 0;
   // workspace: analysis (all rows), classification and items (this rank's rows), the plan
   DevBuf f, nz, Tb, Tl, cls, pw, Ro, tflag, tscan, items, lists, small, scan_tmp, plan, fl8, D, ucnt, uscan,
-      units, ticket, dub, R, Pf, splits, canonB[4], iota, ones, crow_tmp;
+      units, ticket, dub, R, mmlist, Pf, splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
   long long iota_n = -1, ones_n = -1;
@@ -638,7 +639,7 @@ spg_status spg_spgemm_free(spg_handle h) {
     cudaStreamSynchronize(h->stream);
     DevBuf* bufs[] = {&h->f,     &h->nz,    &h->Tb,    &h->Tl,    &h->cls,    &h->pw,   &h->Ro,    &h->tflag,
                       &h->tscan, &h->items, &h->lists, &h->small, &h->scan_tmp, &h->plan, &h->fl8, &h->D,
-                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->R, &h->Pf,     &h->splits,
+                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->R, &h->mmlist, &h->Pf,     &h->splits,
                       &h->iota,  &h->ones,  &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
@@ -700,6 +701,10 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
       h->autotune = v != 0;
       h->tuned = false;
       break;
+    case SPG_OPT_CSRMM_LIGHT_NNZ:
+      if (v < 0 || v > INT_MAX) return setf(h, SPG_ERR_INVALID_ARGUMENT, "CSRMM_LIGHT_NNZ must be in [0, 2^31)");
+      h->csrmm_light = (int)v;
+      break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   h->sym_ok = false;
@@ -719,6 +724,7 @@ spg_status spg_get_option(spg_handle h, spg_option opt, int64_t* v) {
     case SPG_OPT_HUGE_SLOTS: *v = h->huge_slots_opt; break;
     case SPG_OPT_CONCURRENT: *v = h->concurrent; break;
     case SPG_OPT_AUTOTUNE: *v = h->autotune; break;
+    case SPG_OPT_CSRMM_LIGHT_NNZ: *v = h->csrmm_light; break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   return SPG_OK;
@@ -938,6 +944,23 @@ spg_status spg_broadcast_csr(spg_handle h, spg_csr* m, int root) {
     NK(ncclBroadcast(m->vals, (void*)m->vals, (size_t)m->nnz, vt, root, h->comm, h->stream));
   }
   NK(ncclGroupEnd());
+  return SPG_OK;
+}
+
+spg_status spg_csrmm(spg_handle h, const spg_csr* A, const void* D, int64_t ldd, int32_t n, void* C, int64_t ldc) {
+  if (!h) return SPG_ERR_INVALID_ARGUMENT;
+  spg_status s = check_csr(h, A, "A", true);
+  if (s != SPG_OK) return s;
+  if (n < 0 || ldd < n || ldc < n) return setf(h, SPG_ERR_INVALID_ARGUMENT, "need n >= 0, ldd >= n, ldc >= n");
+  if ((long long)A->nrows * n > 0 && !C) return setf(h, SPG_ERR_INVALID_ARGUMENT, "C is NULL");
+  if ((long long)A->ncols * n > 0 && A->nnz > 0 && !D) return setf(h, SPG_ERR_INVALID_ARGUMENT, "D is NULL");
+  DeviceGuard g(h->device);
+  CK(h->mmlist.ensure(((size_t)(A->nrows > 0 ? A->nrows : 1) + 1) * sizeof(int)));
+  int* hl = h->mmlist.as<int>();
+  CK(h->dtype == SPG_FP64 ? launch_csrmm<double>(h->stream, h->sms, A->nrows, A->row_ptr, A->col_idx, A->vals, D, ldd, n,
+                                                C, ldc, h->csrmm_light, hl + 1, hl)
+                          : launch_csrmm<float>(h->stream, h->sms, A->nrows, A->row_ptr, A->col_idx, A->vals, D, ldd, n,
+                                               C, ldc, h->csrmm_light, hl + 1, hl));
   return SPG_OK;
 }
 

@@ -164,6 +164,12 @@ int heavy_occupancy(int bin);
 cudaError_t launch_heavy_rank(int bin, cudaStream_t st, int grid, const SymProb& P, const int* list,
                               const int* count, long long N);
 
+// k_csrmm.cu — sparse x dense.
+template <typename V>
+cudaError_t launch_csrmm(cudaStream_t st, int sms, int M, const int* rpA, const int* colA, const void* valA,
+                         const void* D, long long ldd, int n, void* C, long long ldc, int light_nnz, int* hlist,
+                         int* hcount);
+
 // k_numeric.cu — numeric phase.
 template <typename V>
 int numeric_occupancy();

@@ -500,3 +500,49 @@ def test_fallback_clustered_columns():
     B = W.CSR(K, N, rp, col, rng.integers(1, 5, K * 40).astype(np.float64))
     A = W.random_csr(200, K, 0.05, 32, values="int")
     compare(A, B, run_gpu(A, B), exact_values=True)
+
+
+# ---- sparse x dense (csrmm) ---------------------------------------------------
+def _csrmm_gpu(A, D, **opts):
+    dA = to_dev(A)
+    Dd = torch.from_numpy(np.ascontiguousarray(D)).to("cuda")
+    return spg.csrmm(dA, Dd, **opts).cpu().numpy()
+
+
+@pytest.mark.parametrize("n", [1, 7, 32, 100, 129])
+@pytest.mark.parametrize("light", [0, 16, 256, 1 << 30])
+def test_csrmm_int_exact(n, light):
+    """Small signed integers: every partial sum exact, so C must equal the oracle bit for bit,
+    whichever rows are light (a warp per row) or heavy (a block per row)."""
+    A = W.random_csr(300, 200, 0.2, 3, values="int", empty_row_frac=0.1)
+    D = np.random.default_rng(n).integers(-8, 9, size=(200, n)).astype(np.float64)
+    C = _csrmm_gpu(A, D, csrmm_light_nnz=light)
+    ref, _ = oracle.csrmm(A, D)
+    np.testing.assert_array_equal(C, ref)
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_csrmm_power_law(dtype):
+    """Chung-Lu rows of 1 .. ~2000 stored entries (light and heavy rows), positive values."""
+    A = W.chung_lu(20000, 15000, 2.1, 90000, 2000, 2000, 6.0, 1.1, 9, dtype)
+    D = np.random.default_rng(1).uniform(1, 2, size=(15000, 48)).astype(dtype)
+    C = _csrmm_gpu(A, D)
+    ref, ab = oracle.csrmm(A, D.astype(np.float64))
+    rtol = 1e-12 if dtype == np.float64 else 1e-5
+    assert np.all(np.abs(C.astype(np.float64) - ref) <= rtol * ab)
+
+
+def test_csrmm_strided_and_empty():
+    A = W.random_csr(50, 40, 0.1, 5, values="int", empty_row_frac=0.5)
+    Dfull = np.random.default_rng(2).integers(-4, 5, size=(40, 20)).astype(np.float64)
+    dA = to_dev(A)
+    Dd = torch.from_numpy(Dfull).to("cuda")[:, 3:14]          # ldd = 20, n = 11
+    C = torch.full((50, 16), -7.0, dtype=torch.float64, device="cuda")[:, :11]
+    h = spg.spg_create(0, None, torch.float64)
+    try:
+        spg.spg_csrmm(h, dA, Dd, C)
+        torch.cuda.synchronize()
+    finally:
+        spg.spg_spgemm_free(h)
+    ref, _ = oracle.csrmm(A, Dfull[:, 3:14])
+    np.testing.assert_array_equal(C.cpu().numpy(), ref)

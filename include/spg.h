@@ -121,8 +121,14 @@ typedef enum {
                                    (LIGHT_MAX_FLOPS, TILE_FLOPS) candidates and keeps the fastest
                                    (spg_stats.light_max / tile_flops report the choice); 0
                                    (default): the fixed defaults above                         */
-  SPG_OPT_CSRMM_LIGHT_NNZ = 10  /* spg_csrmm: rows with more stored entries are heavy (a block
+  SPG_OPT_CSRMM_LIGHT_NNZ = 10, /* spg_csrmm: rows with more stored entries are heavy (a block
                                    per row), the rest light (a warp per row); default 256      */
+  SPG_OPT_HEAVY_ORDER = 11      /* order in which heavy-row blocks take rows from their queues:
+                                   0 natural (row order), 1 (default) largest rows first in the
+                                   HUGE / HEAVY2 bins when they hold <= 2048 rows, 2 largest
+                                   first in every bin (long lists by log2 class) — with
+                                   FORCE_CLASS = HUGE the GPU analogues of the paper's Unsorted-
+                                   and Sorted-Workqueue                    */
 } spg_option;
 
 typedef struct {

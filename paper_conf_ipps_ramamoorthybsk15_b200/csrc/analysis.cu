@@ -598,9 +598,43 @@ __global__ void __launch_bounds__(1024) k_sort_lists(HeavyLists lists, int b, co
   for (int x = threadIdx.x; x < n; x += blockDim.x) list[x] = (int)(unsigned)(key[x] & 0xffffffffu);
 }
 
+// Lists longer than LPT_MAX (SPG_OPT_HEAVY_ORDER = 2): descending log2(f) classes — a one-block
+// counting sort through a scratch copy (order inside a class is arbitrary).
+__global__ void __launch_bounds__(1024) k_sort_lists_bins(HeavyLists lists, int b, const int* __restrict__ f, int rb,
+                                                          const Small* __restrict__ sm, int* __restrict__ tmp) {
+  __shared__ int hist[33];
+  const int n = sm->counts[b];
+  if (n <= LPT_MAX) return;
+  int* list = lists.rows[b];
+  if (threadIdx.x < 33) hist[threadIdx.x] = 0;
+  __syncthreads();
+  for (int x = threadIdx.x; x < n; x += blockDim.x) {
+    const int v = f[rb + list[x]];
+    atomicAdd(&hist[v > 0 ? 31 - __clz(v) : 32], 1);
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {  // exclusive prefix in descending class order
+    int run = 0;
+    for (int c = 31; c >= 0; --c) {
+      const int v = hist[c];
+      hist[c] = run;
+      run += v;
+    }
+    hist[32] = run;
+  }
+  __syncthreads();
+  for (int x = threadIdx.x; x < n; x += blockDim.x) {
+    const int li = list[x], v = f[rb + li];
+    tmp[atomicAdd(&hist[v > 0 ? 31 - __clz(v) : 32], 1)] = li;
+  }
+  __syncthreads();
+  for (int x = threadIdx.x; x < n; x += blockDim.x) list[x] = tmp[x];
+}
+
 cudaError_t launch_sort_list(cudaStream_t st, const HeavyLists& lists, int bin, const int* f, int rb,
-                             const Small* small) {
+                             const Small* small, int* tmp) {
   k_sort_lists<<<1, 1024, 0, st>>>(lists, bin, f, rb, small);
+  if (tmp) k_sort_lists_bins<<<1, 1024, 0, st>>>(lists, bin, f, rb, small, tmp);
   return cudaGetLastError();
 }
 

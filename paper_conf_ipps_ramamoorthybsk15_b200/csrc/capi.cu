@@ -82,12 +82,13 @@ struct spg_ctx {
   int thresholds_set = 0;  // light_max / tile_cap set by the caller (else N-dependent defaults)
   int autotune = 0;        // SPG_OPT_AUTOTUNE: time candidate thresholds on a new structure
   int csrmm_light = 256;   // SPG_OPT_CSRMM_LIGHT_NNZ
+  int heavy_order = 1;     // SPG_OPT_HEAVY_ORDER
   bool tuned = false;
   SymKey tuned_key{};
   int tuned_light = 0, tuned_tile = 0;
   // workspace: analysis (all rows), classification and items (this rank's rows), the plan
   DevBuf f, nz, Tb, Tl, cls, pw, Ro, tflag, tscan, items, lists, small, scan_tmp, plan, fl8, D, ucnt, uscan,
-      units, ticket, dub, R, mmlist, Pf, splits, canonB[4], iota, ones, crow_tmp;
+      units, ticket, dub, R, mmlist, lsort, Pf, splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
   long long iota_n = -1, ones_n = -1;
@@ -229,11 +230,18 @@ spg_status fork_heavy(spg_handle h, const spg_csr* A, const spg_csr* B, long lon
     long long grid = (long long)h->occ_heavy[b] * h->sms;
     if (h->huge_slots_opt > 0 && h->huge_slots_opt < grid) grid = h->huge_slots_opt;
     int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
-    if (b != BIN_HEAVY && Mloc > 0) {  // largest rows first (the HEAVY bin's list is too long to pay)
+    // largest rows first (HEAVY_ORDER 1: the HUGE and HEAVY2 lists when they hold <= 2048 rows;
+    // 2: every list, long ones by log2 class; 0: natural order)
+    if (Mloc > 0 && (h->heavy_order == 2 || (h->heavy_order == 1 && b != BIN_HEAVY))) {
       HeavyLists L3;
       for (int c = 0; c < NUM_BINS; ++c) L3.rows[c] = h->lists.as<int>() + (size_t)c * (size_t)Mloc;
-      CK(launch_sort_list(st, L3, b, h->f.as<int>(), h->rb, ds));
-      h->launches++;
+      int* tmp = nullptr;
+      if (h->heavy_order == 2) {
+        CK(h->lsort.ensure((size_t)NUM_BINS * (size_t)Mloc * sizeof(int)));
+        tmp = h->lsort.as<int>() + (size_t)b * (size_t)Mloc;
+      }
+      CK(launch_sort_list(st, L3, b, h->f.as<int>(), h->rb, ds, tmp));
+      h->launches += tmp ? 2 : 1;
     }
     CK(launch_heavy_rank(b, st, (int)grid, P, list, ds->counts + b, B->ncols));
     h->launches++;
@@ -639,7 +647,7 @@ spg_status spg_spgemm_free(spg_handle h) {
     cudaStreamSynchronize(h->stream);
     DevBuf* bufs[] = {&h->f,     &h->nz,    &h->Tb,    &h->Tl,    &h->cls,    &h->pw,   &h->Ro,    &h->tflag,
                       &h->tscan, &h->items, &h->lists, &h->small, &h->scan_tmp, &h->plan, &h->fl8, &h->D,
-                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->R, &h->mmlist, &h->Pf,     &h->splits,
+                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->R, &h->mmlist, &h->lsort, &h->Pf,     &h->splits,
                       &h->iota,  &h->ones,  &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
@@ -705,6 +713,10 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
       if (v < 0 || v > INT_MAX) return setf(h, SPG_ERR_INVALID_ARGUMENT, "CSRMM_LIGHT_NNZ must be in [0, 2^31)");
       h->csrmm_light = (int)v;
       break;
+    case SPG_OPT_HEAVY_ORDER:
+      if (v < 0 || v > 2) return setf(h, SPG_ERR_INVALID_ARGUMENT, "HEAVY_ORDER must be 0, 1 or 2");
+      h->heavy_order = (int)v;
+      break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   h->sym_ok = false;
@@ -725,6 +737,7 @@ spg_status spg_get_option(spg_handle h, spg_option opt, int64_t* v) {
     case SPG_OPT_CONCURRENT: *v = h->concurrent; break;
     case SPG_OPT_AUTOTUNE: *v = h->autotune; break;
     case SPG_OPT_CSRMM_LIGHT_NNZ: *v = h->csrmm_light; break;
+    case SPG_OPT_HEAVY_ORDER: *v = h->heavy_order; break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   return SPG_OK;

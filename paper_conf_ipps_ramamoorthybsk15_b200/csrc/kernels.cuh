@@ -136,7 +136,7 @@ cudaError_t launch_tile_flags(cudaStream_t st, int sms, const int* f, const int*
 cudaError_t launch_items(cudaStream_t st, int sms, const int* tflag, const long long* tscan, int mloc, int* items,
                          Small* small);
 cudaError_t launch_sort_list(cudaStream_t st, const HeavyLists& lists, int bin, const int* f, int rb,
-                             const Small* small);
+                             const Small* small, int* tmp);
 size_t scan_tmp_elems(long long n);
 int scan_launches(long long n);
 template <typename Tin>

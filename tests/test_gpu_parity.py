@@ -91,6 +91,21 @@ def test_autotune_picks_a_candidate_and_keeps_the_result():
     assert (st["light_max"], st["tile_flops"]) in [(1024, 3072), (2048, 2048), (3072, 1024), (4096, 2048), (512, 3584)]
 
 
+@pytest.mark.parametrize("alpha", [3.0, 6.5])
+def test_alpha_sweep_pair_variants(alpha):
+    """The f3 alpha-sweep workload (two distinct Chung-Lu matrices with the same exponent, n =
+    100K) through compare() with the default split and every baseline the
+    sweep times: block per row ([13]-style one path), max tiles, and the Unsorted- / Sorted-
+    Workqueue analogues (FORCE_CLASS = HUGE, HEAVY_ORDER 0 / 2)."""
+    n = 100000
+    A = W.chung_lu(n, n, alpha, 8 * n, 2000.0, 2000.0, 6.0, 1.1, 101)
+    B = W.chung_lu(n, n, alpha, 8 * n, 2000.0, 2000.0, 6.0, 1.1, 202)
+    ref = oracle.spgemm(A, B, nthreads=8)
+    for opts in ({}, {"force_class": 5}, {"light_max_flops": 4096, "tile_flops": 1024},
+                 {"force_class": 6, "heavy_order": 0}, {"force_class": 6, "heavy_order": 2}):
+        compare(A, B, run_gpu(A, B, **opts), ref=ref)
+
+
 def test_fp32_power_law():
     A = W.chung_lu(20000, 20000, 2.1, 80000, 3000, 3000, 6.0, 1.1, 5, np.float32)
     B = W.chung_lu(20000, 20000, 3.0, 160000, 1000, 1000, -1.0, 1.0, 6, np.float32)

@@ -7,14 +7,22 @@ sys.path.insert(0, ".")
 import paper_conf_ipps_ramamoorthybsk15_b200 as spg, workloads as W
 A, _ = W.make("cl10k")
 dA = spg.DeviceCSR.from_host(A, "cuda:0")
-for opts in ({}, {"warp_max_flops": 256}, {"force_class": 6}, {"light_max_flops": 0}):
+for opts in ({}, {"force_class": 6}, {"force_class": 5}, {"light_max_flops": 0}, {"light_max_flops": 4096, "tile_flops": 1024}):
     plan = spg.SpGEMM(0, torch.float64)
     for k, v in opts.items():
         plan.set_option(k, v)
     C = plan(dA, dA)
     torch.cuda.synchronize()
     plan.close()
-print("case ok", int(C.row_ptr[-1]))
+D = torch.rand(A.ncols, 40, dtype=torch.float64, device="cuda:0")
+spg.csrmm(dA, D, csrmm_light_nnz=16)
+B = W.random_csr(A.ncols, 3000, 0.002, 4, canonical=False)
+dB = spg.DeviceCSR.from_host(B, "cuda:0")
+plan = spg.SpGEMM(0, torch.float64, input_canonical=0)
+C2 = plan(dA, dB)
+torch.cuda.synchronize()
+plan.close()
+print("case ok", int(C.row_ptr[-1]), int(C2.row_ptr[-1]))
 PY
 for tool in memcheck racecheck synccheck; do
   timeout 1500 compute-sanitizer --tool $tool --error-exitcode 9 python /tmp/san_case.py > gpurun_out/san_$tool.log 2>&1

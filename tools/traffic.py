@@ -1,5 +1,6 @@
-"""Per-launch DRAM traffic of the numeric phase (k_numeric + k_numeric_dup [+ k_pack_b]) from an
-ncu launch list (tools/gpu_iter.sh metrics) -> profiles/traffic_<config>.json, read by bench.py."""
+"""Per-launch DRAM traffic of the numeric phase (k_numeric) from an ncu launch list
+(tools/round_capture.sh metrics) -> <out dir>/traffic_<config>.json (copied to profiles/, where
+bench.py reads it).   python tools/traffic.py launches.csv webbase1m [out_dir]"""
 import csv
 import json
 import re
@@ -21,5 +22,6 @@ tot = sum(m['dram__bytes_read.sum'] + m['dram__bytes_write.sum'] for _, m in num
 out = {"numeric_dram_bytes_per_launch": tot / n, "launches": n, "source": src,
        "kernels": sorted({k[1] for k, _ in num}),
        "how": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum --clock-control none, python bench.py --profile"}
-json.dump(out, open(f"profiles/traffic_{config}.json", "w"), indent=1)
+odir = sys.argv[3] if len(sys.argv) > 3 else "profiles"
+json.dump(out, open(f"{odir}/traffic_{config}.json", "w"), indent=1)
 print(json.dumps(out))

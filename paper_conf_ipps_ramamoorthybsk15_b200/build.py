@@ -43,7 +43,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     logs = []
     for src in sources():
         obj = os.path.join(BUILD, os.path.basename(src) + ".o")
-        extra = os.environ.get("SPG_NVCC_FLAGS", "").split()  # experiments only (e.g. -DSPG_PHASE_PROF)
+        extra = os.environ.get("SPG_NVCC_FLAGS", "").split()  # experiments only (variant builds for tools/so_ab.sh)
         cmd = [nvcc, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xptxas", "-v", "-Xcompiler", "-fPIC", *extra,
                "-I", os.path.join(ROOT, "include"), "-I", CSRC, "-I", inc, "-c", src, "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)

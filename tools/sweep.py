@@ -53,7 +53,7 @@ def time_plan(dA, dB, steps, **opts):
 LIGHT = [int(x) for x in os.environ.get("SWEEP_LIGHT", "0,256,512,1024,2048").split(",")]
 TILE = [int(x) for x in os.environ.get("SWEEP_TILE", "1024,2048").split(",")]
 HEAVY = [int(x) for x in os.environ.get("SWEEP_HEAVY", "4096,8192").split(",")]
-PMAX = int(os.environ.get("SWEEP_PMAX", "3072"))
+PMAX = int(os.environ.get("SWEEP_PMAX", "6144"))
 
 
 def main():
@@ -67,7 +67,8 @@ def main():
     dA = spg.DeviceCSR.from_host(A, "cuda")
     dB = dA if B is A else spg.DeviceCSR.from_host(B, "cuda")
     # (light_max, tile_flops, heavy_max): light rows (f <= light_max) go to the tile kernel,
-    # light_max + tile_flops <= TILE_PMAX (3072); heavy rows up to heavy_max to the cached bitmap
+    # light_max + tile_flops <= SWEEP_PMAX (rows above TILE_PMAX - tile_flops are solo tiles);
+    # heavy rows up to heavy_max to the cached bitmap
     grid = [(lm, tf, hm) for lm in LIGHT for tf in TILE for hm in HEAVY if lm + tf <= PMAX]
     ref = None
     for lm, tf, hm in grid:

@@ -123,12 +123,17 @@ typedef enum {
                                    (default): the fixed defaults above                         */
   SPG_OPT_CSRMM_LIGHT_NNZ = 10, /* spg_csrmm: rows with more stored entries are heavy (a block
                                    per row), the rest light (a warp per row); default 256      */
-  SPG_OPT_HEAVY_ORDER = 11      /* order in which heavy-row blocks take rows from their queues:
+  SPG_OPT_HEAVY_ORDER = 11,     /* order in which heavy-row blocks take rows from their queues:
                                    0 natural (row order), 1 (default) largest rows first in the
                                    HUGE / HEAVY2 bins when they hold <= 2048 rows, 2 largest
                                    first in every bin (long lists by log2 class) — with
                                    FORCE_CLASS = HUGE the GPU analogues of the paper's Unsorted-
                                    and Sorted-Workqueue                    */
+  SPG_OPT_PACK_B = 12           /* numeric gathers B through a packed {column, value} copy (one
+                                   sector per output instead of two; the copy is made by every
+                                   numeric call, 16 B per B entry for fp64): -1 (default) when
+                                   B's columns + values exceed 64 MB (B not L2-resident), 0 never,
+                                   1 always                                                     */
 } spg_option;
 
 typedef struct {

@@ -83,12 +83,13 @@ struct spg_ctx {
   int autotune = 0;        // SPG_OPT_AUTOTUNE: time candidate thresholds on a new structure
   int csrmm_light = 256;   // SPG_OPT_CSRMM_LIGHT_NNZ
   int heavy_order = 1;     // SPG_OPT_HEAVY_ORDER
+  int pack_b = -1;         // SPG_OPT_PACK_B
   bool tuned = false;
   SymKey tuned_key{};
   int tuned_light = 0, tuned_tile = 0;
   // workspace: analysis (all rows), classification and items (this rank's rows), the plan
   DevBuf f, nz, Tb, Tl, cls, pw, Ro, tflag, tscan, items, lists, small, scan_tmp, plan, fl8, D, ucnt, uscan,
-      units, ticket, dub, R, mmlist, lsort, Pf, splits, canonB[4], iota, ones, crow_tmp;
+      units, ticket, dub, R, mmlist, lsort, Bp, Pf, splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
   long long iota_n = -1, ones_n = -1;
@@ -100,7 +101,7 @@ struct spg_ctx {
   cudaEvent_t ev_bval = nullptr;  // values of an asynchronous broadcast are in (numeric waits)
   bool bval_pending = false;
   std::vector<long long> scat;  // scatter plan: rows, nnz, first entry per rank (root-side offsets)
-  int occ_tile = 1, occ_heavy[NUM_BINS] = {}, occ_num = 1;
+  int occ_tile = 1, occ_heavy[NUM_BINS] = {};
   // cached symbolic state
   bool sym_ok = false;
   SymKey key{};
@@ -548,6 +549,15 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
     P.Tb = h->Tb.as<int>();
     P.colB = B->col_idx;
     P.valB = (const V*)B->vals;
+    P.Bp = nullptr;
+    // packed B when it does not stay in L2 (auto: columns + values above 64 MB)
+    const long long bbytes = (long long)B->nnz * (4 + (long long)sizeof(V));
+    if (B->nnz > 0 && (h->pack_b > 0 || (h->pack_b < 0 && bbytes > (64LL << 20)))) {
+      CK(h->Bp.ensure((size_t)B->nnz * (sizeof(V) == 8 ? 16 : 8)));
+      CK(launch_pack_b<V>(h->stream, h->sms, B->col_idx, (const V*)B->vals, B->nnz, h->Bp.p));
+      P.Bp = h->Bp.p;
+      h->launches += 1;
+    }
     P.plan = h->plan.as<unsigned>();
     P.Ro = h->Ro.as<long long>();
     P.crow = reinterpret_cast<const long long*>(C_row_ptr);
@@ -561,7 +571,7 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
     P.ccol = C_col;
     P.cval = (V*)C_val;
     CK(cudaMemsetAsync(P.ticket, 0, sizeof(int), h->stream));
-    CK(launch_numeric<V>(h->stream, h->occ_num * h->sms, P));
+    CK(launch_numeric<V>(h->stream, h->sms, P));
     h->launches += 1;
   }
   h->stats.launches_numeric = h->launches;
@@ -616,7 +626,6 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     return SPG_ERR_CUDA;
   }
   h->occ_tile = tile_occupancy();
-  h->occ_num = dtype == SPG_FP64 ? numeric_occupancy<double>() : numeric_occupancy<float>();
   for (int b = 0; b < NUM_BINS; ++b) h->occ_heavy[b] = heavy_occupancy(b);
   cudaGetLastError();
   *out = h;
@@ -647,7 +656,7 @@ spg_status spg_spgemm_free(spg_handle h) {
     cudaStreamSynchronize(h->stream);
     DevBuf* bufs[] = {&h->f,     &h->nz,    &h->Tb,    &h->Tl,    &h->cls,    &h->pw,   &h->Ro,    &h->tflag,
                       &h->tscan, &h->items, &h->lists, &h->small, &h->scan_tmp, &h->plan, &h->fl8, &h->D,
-                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->R, &h->mmlist, &h->lsort, &h->Pf,     &h->splits,
+                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->R, &h->mmlist, &h->lsort, &h->Bp, &h->Pf,     &h->splits,
                       &h->iota,  &h->ones,  &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
@@ -717,6 +726,10 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
       if (v < 0 || v > 2) return setf(h, SPG_ERR_INVALID_ARGUMENT, "HEAVY_ORDER must be 0, 1 or 2");
       h->heavy_order = (int)v;
       break;
+    case SPG_OPT_PACK_B:
+      if (v < -1 || v > 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "PACK_B must be -1, 0 or 1");
+      h->pack_b = (int)v;
+      break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   h->sym_ok = false;
@@ -738,6 +751,7 @@ spg_status spg_get_option(spg_handle h, spg_option opt, int64_t* v) {
     case SPG_OPT_AUTOTUNE: *v = h->autotune; break;
     case SPG_OPT_CSRMM_LIGHT_NNZ: *v = h->csrmm_light; break;
     case SPG_OPT_HEAVY_ORDER: *v = h->heavy_order; break;
+    case SPG_OPT_PACK_B: *v = h->pack_b; break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   return SPG_OK;

@@ -58,8 +58,35 @@ __device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned phas
       : "memory");
 }
 
+// Packed B: {column, value} in one 16-byte (fp64) or 8-byte (fp32) record, so an output's B
+// gather is one sector instead of two when B does not stay in L2 (rmat23's B is 1.6 GB).
+template <typename V> struct PackB;
+template <> struct PackB<double> {
+  using T = int4;
+  __device__ static T make(int c, double v) {
+    return make_int4(c, 0, __double2loint(v), __double2hiint(v));
+  }
+  __device__ static int col(const T& t) { return t.x; }
+  __device__ static double val(const T& t) { return __hiloint2double(t.w, t.z); }
+};
+template <> struct PackB<float> {
+  using T = int2;
+  __device__ static T make(int c, float v) { return make_int2(c, __float_as_int(v)); }
+  __device__ static int col(const T& t) { return t.x; }
+  __device__ static float val(const T& t) { return __int_as_float(t.y); }
+};
+
 template <typename V>
+__global__ void __launch_bounds__(256) k_pack_b(const int* __restrict__ colB, const V* __restrict__ valB, long long n,
+                                                typename PackB<V>::T* __restrict__ out) {
+  for (long long x = blockIdx.x * (long long)blockDim.x + threadIdx.x; x < n; x += (long long)gridDim.x * blockDim.x)
+    out[x] = PackB<V>::make(colB[x], valB[x]);
+}
+
+template <typename V, bool PACKED>
 __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
+  using PB = PackB<V>;
+  const typename PB::T* __restrict__ Bp = reinterpret_cast<const typename PB::T*>(P.Bp);
   __shared__ __align__(16) unsigned s_buf[NUM_W][2][NUM_BUFW];
   __shared__ __align__(8) unsigned long long s_bar[NUM_W][2];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -140,8 +167,14 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
       for (int x = 0; x < NUM_U; ++x)
         if (q[x] >= 0) {
           a[x] = __ldg(P.valA + e[x]);
-          col[x] = __ldg(P.colB + q[x]);
-          b[x] = __ldg(P.valB + q[x]);
+          if constexpr (PACKED) {
+            const typename PB::T t = __ldg(Bp + q[x]);
+            col[x] = PB::col(t);
+            b[x] = PB::val(t);
+          } else {
+            col[x] = __ldg(P.colB + q[x]);
+            b[x] = __ldg(P.valB + q[x]);
+          }
         }
 #pragma unroll
       for (int x = 0; x < NUM_U; ++x)
@@ -155,10 +188,14 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
     // ---- repeated products landing in this unit's outputs (R records: B entry, A entry, output) -
     if (cur.d > 0) {
       V* __restrict__ cv0 = cval - (cur.ob & (UNIT_WIDE - 1));
-      if (lane < cur.d) atomicAdd(cv0 + rec.z, __ldg(P.valA + rec.y) * __ldg(P.valB + rec.x));
+      auto bval = [&](int q) -> V {
+        if constexpr (PACKED) return PB::val(__ldg(Bp + q));
+        else return __ldg(P.valB + q);
+      };
+      if (lane < cur.d) atomicAdd(cv0 + rec.z, __ldg(P.valA + rec.y) * bval(rec.x));
       for (int j = 32 + lane; j < cur.d; j += 32) {
         const int4 x = __ldg(P.R + cur.dw + j);
-        atomicAdd(cv0 + x.z, __ldg(P.valA + x.y) * __ldg(P.valB + x.x));
+        atomicAdd(cv0 + x.z, __ldg(P.valA + x.y) * bval(x.x));
       }
     }
     if (!more) break;
@@ -169,22 +206,34 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
 }
 
 template <typename V>
-int numeric_occupancy() {
-  int nb = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_numeric<V>, NUM_NT, 0);
-  return nb < 1 ? 1 : nb;
-}
-
-template <typename V>
-cudaError_t launch_numeric(cudaStream_t st, int grid, const NumProb<V>& P) {
-  if (grid <= 0) return cudaSuccess;
-  k_numeric<V><<<grid, NUM_NT, 0, st>>>(P);
+cudaError_t launch_numeric(cudaStream_t st, int sms, const NumProb<V>& P) {
+  // persistent grid: every block of the variant that fits at once
+  static int occ[2] = {0, 0};
+  const int v = P.Bp ? 1 : 0;
+  if (!occ[v]) {
+    int nb = 1;
+    if (v) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_numeric<V, true>, NUM_NT, 0);
+    else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_numeric<V, false>, NUM_NT, 0);
+    occ[v] = nb < 1 ? 1 : nb;
+  }
+  const int grid = occ[v] * sms;
+  if (v) k_numeric<V, true><<<grid, NUM_NT, 0, st>>>(P);
+  else k_numeric<V, false><<<grid, NUM_NT, 0, st>>>(P);
   return cudaGetLastError();
 }
 
-template int numeric_occupancy<double>();
-template int numeric_occupancy<float>();
+template <typename V>
+cudaError_t launch_pack_b(cudaStream_t st, int sms, const int* colB, const V* valB, long long n, void* out) {
+  if (n <= 0) return cudaSuccess;
+  long long g = (n + 255) / 256;
+  if (g > (long long)sms * 16) g = (long long)sms * 16;
+  k_pack_b<V><<<(int)g, 256, 0, st>>>(colB, valB, n, reinterpret_cast<typename PackB<V>::T*>(out));
+  return cudaGetLastError();
+}
+
 template cudaError_t launch_numeric<double>(cudaStream_t, int, const NumProb<double>&);
 template cudaError_t launch_numeric<float>(cudaStream_t, int, const NumProb<float>&);
+template cudaError_t launch_pack_b<double>(cudaStream_t, int, const int*, const double*, long long, void*);
+template cudaError_t launch_pack_b<float>(cudaStream_t, int, const int*, const float*, long long, void*);
 
 }  // namespace spg

@@ -106,6 +106,7 @@ struct NumProb {
   const int* __restrict__ Tb;           // per A entry: start of its B row
   const int* __restrict__ colB;
   const V* __restrict__ valB;
+  const void* __restrict__ Bp;          // packed {column, value} copy of B (one gather per output) or NULL
   const unsigned* __restrict__ plan;
   const long long* __restrict__ Ro;
   const long long* __restrict__ crow;   // C row offsets (local)
@@ -172,8 +173,8 @@ cudaError_t launch_csrmm(cudaStream_t st, int sms, int M, const int* rpA, const 
 
 // k_numeric.cu — numeric phase.
 template <typename V>
-int numeric_occupancy();
+cudaError_t launch_numeric(cudaStream_t st, int sms, const NumProb<V>& P);
 template <typename V>
-cudaError_t launch_numeric(cudaStream_t st, int grid, const NumProb<V>& P);
+cudaError_t launch_pack_b(cudaStream_t st, int sms, const int* colB, const V* valB, long long n, void* out);
 
 }  // namespace spg

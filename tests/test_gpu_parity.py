@@ -106,6 +106,14 @@ def test_alpha_sweep_pair_variants(alpha):
         compare(A, B, run_gpu(A, B, **opts), ref=ref)
 
 
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_packed_b_numeric(dtype):
+    """SPG_OPT_PACK_B = 1: numeric gathers B through the packed {column, value} copy (automatic
+    only for B > 64 MB, i.e. rmat23) — same C as the oracle, repeats included."""
+    A = W.chung_lu(20000, 20000, 2.1, 80000, 3000, 3000, 6.0, 1.1, 5, dtype)
+    compare(A, A, run_gpu(A, A, pack_b=1))
+
+
 def test_fp32_power_law():
     A = W.chung_lu(20000, 20000, 2.1, 80000, 3000, 3000, 6.0, 1.1, 5, np.float32)
     B = W.chung_lu(20000, 20000, 3.0, 160000, 1000, 1000, -1.0, 1.0, 6, np.float32)

@@ -103,7 +103,7 @@ typedef enum {
   SPG_OPT_LIGHT_MAX_FLOPS = 0,  /* heavy/light threshold t: 0..4096; light rows
                                    above 4096 - TILE_FLOPS are tiles of their own;
                                    default 2048 with tile 2048 (tools/sweep_quick.sh, profiles/);
-                                   when B has > 2^22 columns and neither option was set: 3072
+                                   when B has > 2^22 columns and neither option was set: 4096
                                    with tile 1024.  0 sends every non-SINGLE row to the heavy
                                    path                                                         */
   SPG_OPT_TILE_FLOPS = 1,       /* nominal products per light tile, default 2048               */
@@ -129,10 +129,15 @@ typedef enum {
                                    first in every bin (long lists by log2 class) — with
                                    FORCE_CLASS = HUGE the GPU analogues of the paper's Unsorted-
                                    and Sorted-Workqueue                    */
-  SPG_OPT_PACK_B = 12           /* numeric gathers B through a packed {column, value} copy (one
+  SPG_OPT_PACK_B = 12,          /* numeric gathers B through a packed {column, value} copy (one
                                    sector per output instead of two; the copy is made by every
                                    numeric call, 16 B per B entry for fp64): -1 (default) when
                                    B's columns + values exceed 64 MB (B not L2-resident), 0 never,
+                                   1 always                                                     */
+  SPG_OPT_HEAVY_SORT = 13       /* HEAVY rows (f <= 8192) are sorted like tiles in "big tiles" of
+                                   8192 products (1024 threads) instead of the column bitmap:
+                                   -1 (default) when B has more than 2^20 columns (the bitmap
+                                   would need several column-tile passes per row), 0 never,
                                    1 always                                                     */
 } spg_option;
 

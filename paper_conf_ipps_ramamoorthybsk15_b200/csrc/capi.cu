@@ -84,6 +84,9 @@ struct spg_ctx {
   int csrmm_light = 256;   // SPG_OPT_CSRMM_LIGHT_NNZ
   int heavy_order = 1;     // SPG_OPT_HEAVY_ORDER
   int pack_b = -1;         // SPG_OPT_PACK_B
+  int heavy_sort = -1;     // SPG_OPT_HEAVY_SORT
+  int occ_big = 1;
+  bool use_big = false;    // this symbolic call sorts the cached heavy bins as big tiles
   bool tuned = false;
   SymKey tuned_key{};
   int tuned_light = 0, tuned_tile = 0;
@@ -228,6 +231,16 @@ spg_status fork_heavy(spg_handle h, const spg_csr* A, const spg_csr* B, long lon
     cudaStream_t st = conc ? h->aux[1 + x] : h->stream;
     if (conc) CK(cudaStreamWaitEvent(st, h->ev_fork, 0));
     if (tm && x == 0) CK(cudaEventRecord(h->ev_p[2], st));
+    if (h->use_big && b != BIN_HUGE) {  // both cached bins as big tiles, in one launch
+      if (b == BIN_HEAVY2) {
+        HeavyLists L3;
+        for (int c = 0; c < NUM_BINS; ++c) L3.rows[c] = h->lists.as<int>() + (size_t)c * (size_t)(Mloc > 0 ? Mloc : 1);
+        CK(launch_tile_heavy(st, h->occ_big * h->sms, P, L3, ds->counts, &ds->qhead[BIN_HEAVY]));
+        h->launches++;
+      }
+      if (conc) CK(cudaEventRecord(h->ev_join[1 + x], st));
+      continue;
+    }
     long long grid = (long long)h->occ_heavy[b] * h->sms;
     if (h->huge_slots_opt > 0 && h->huge_slots_opt < grid) grid = h->huge_slots_opt;
     int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
@@ -419,10 +432,12 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     // are kept as given.
     int light_max = h->light_max, tile_cap = h->tile_cap;
     if (!h->thresholds_set && B->ncols > (1 << 22)) {
-      light_max = TILE_PMAX - 1024;
+      light_max = TILE_PMAX;
       tile_cap = 1024;
     }
     ClassParams prm{light_max, h->heavy_max, tile_cap, h->force, h->canonical ? 1 : 0};
+    // cached heavy rows as big tiles when the 1024-thread bitmap needs several column tiles
+    h->use_big = h->heavy_sort > 0 || (h->heavy_sort < 0 && B->ncols > (1 << 20));
     used_light = light_max;
     used_tile = tile_cap;
     HeavyLists L3;
@@ -625,7 +640,8 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
     spg_spgemm_free(h);
     return SPG_ERR_CUDA;
   }
-  h->occ_tile = tile_occupancy();
+  h->occ_tile = tile_occupancy(0);
+  h->occ_big = tile_occupancy(1);
   for (int b = 0; b < NUM_BINS; ++b) h->occ_heavy[b] = heavy_occupancy(b);
   cudaGetLastError();
   *out = h;
@@ -730,6 +746,10 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
       if (v < -1 || v > 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "PACK_B must be -1, 0 or 1");
       h->pack_b = (int)v;
       break;
+    case SPG_OPT_HEAVY_SORT:
+      if (v < -1 || v > 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "HEAVY_SORT must be -1, 0 or 1");
+      h->heavy_sort = (int)v;
+      break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   h->sym_ok = false;
@@ -752,6 +772,7 @@ spg_status spg_get_option(spg_handle h, spg_option opt, int64_t* v) {
     case SPG_OPT_CSRMM_LIGHT_NNZ: *v = h->csrmm_light; break;
     case SPG_OPT_HEAVY_ORDER: *v = h->heavy_order; break;
     case SPG_OPT_PACK_B: *v = h->pack_b; break;
+    case SPG_OPT_HEAVY_SORT: *v = h->heavy_sort; break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   return SPG_OK;

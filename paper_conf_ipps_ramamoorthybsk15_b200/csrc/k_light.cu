@@ -32,13 +32,25 @@
 
 namespace spg {
 
-static_assert(TILE_PMAX / TILE_NT <= 32, "head marks of a thread fit one 32-bit mask");
-constexpr int BATCH_RM = 512;         // rows per batch
-constexpr int BATCH_NI = 16;          // items per queue pop
-constexpr int BATCH_NB = TILE_PMAX / TILE_BK + BATCH_RM;  // buckets per batch (ceil per row)
-constexpr int BATCH_NU = BATCH_NI + TILE_PMAX / NUM_SH;   // numeric units of a batch's tiles
-static_assert(BATCH_RM <= TILE_NT, "one row per thread in the row phases");
-static_assert(TILE_RM <= BATCH_RM, "a tile fits a batch");
+// Two instances of the kernel: tiles (batches of <= 4096 products, 512 threads, two blocks per SM)
+// popped from the item list, and "big tiles" (<= 8192 products, 1024 threads, one block per SM)
+// that sort the register-cached heavy rows (f <= 8192) popped from their bin lists — instead of
+// the column bitmap, whose per-row cost grows with the column count (SPG_OPT_HEAVY_SORT).
+template <int PMAX_, int NT_, bool LIST_>
+struct TileCfg {
+  static constexpr int PMAX = PMAX_;   // products per batch
+  static constexpr int NT = NT_;       // threads
+  static constexpr bool LIST = LIST_;  // pop heavy rows from the bin lists (else items)
+  static constexpr int RM = 512;       // rows per batch
+  static constexpr int NI = 16;        // items per queue pop
+  static constexpr int NB = PMAX / TILE_BK + RM;  // buckets per batch (ceil per row)
+  static constexpr int NU = NI + PMAX / NUM_SH;   // numeric units of a batch's items
+  static_assert(PMAX / NT <= 32, "head marks of a thread fit one 32-bit mask");
+  static_assert(RM <= NT, "one row per thread in the row phases");
+  static_assert(TILE_RM <= RM, "a tile fits a batch");
+};
+using TileSmall = TileCfg<TILE_PMAX, TILE_NT, false>;
+using TileBig = TileCfg<2 * TILE_PMAX, 2 * TILE_NT, true>;
 constexpr int TILE_EU = 4;  // 32-product windows per warp per step (loads in flight)
 
 // Run of product jw + lane for a window starting inside run rb (warp-uniform); advances rb to
@@ -55,104 +67,121 @@ __device__ __forceinline__ int walk_run(const int* seg, int nr, int jw, int& rb)
 }
 
 // Shared-memory layout of one tile block (bytes).
+template <class C>
 struct TileSmem {
   static constexpr int keys = 0;                                    // int[PMAX]   idx -> column (expand), then
                                                                     //             slot -> column (sign: not head)
-  static constexpr int pay = keys + TILE_PMAX * 4;                  // u32[PMAX]   idx -> plan word
-  static constexpr int sidx = pay + TILE_PMAX * 4;                  // u16[PMAX]   slot -> product index
-  static constexpr int sbk = sidx + TILE_PMAX * 2;                  // u16[PMAX]   slot -> bucket (repeats: output)
-  static constexpr int exrow = sbk + TILE_PMAX * 2;                 // u16[PMAX]   idx -> batch row
-  static constexpr int cnt = exrow + TILE_PMAX * 2;                 // int[NB+1]   sizes -> starts -> ends
-  static constexpr int hc = cnt + (BATCH_NB + 1) * 4;               // int[NB+1]   heads -> head prefix
-  static constexpr int ae = (hc + (BATCH_NB + 1) * 4 + 15) & ~15;   // int[RM+1]   A-entry offset of the row
-  static constexpr int pf = ae + (BATCH_RM + 1) * 4;                // int[RM+1]   product offset of the row
-  static constexpr int bb = pf + (BATCH_RM + 1) * 4;                // int[RM+1]   bucket base
-  static constexpr int out = bb + (BATCH_RM + 1) * 4;               // int[RM+1]   output offset in the batch
-  static constexpr int rpa = out + (BATCH_RM + 1) * 4;              // int[RM]     first A entry of the row
-  static constexpr int row = rpa + BATCH_RM * 4;                    // int[RM]     local row index
-  static constexpr int cmin = row + BATCH_RM * 4;                   // int[RM]     column range of the row
-  static constexpr int cmax = cmin + BATCH_RM * 4;                  // int[RM]
-  static constexpr int sh = cmax + BATCH_RM * 4;                    // u8[RM]      bucket width log2
-  static constexpr int kind = sh + BATCH_RM;                        // u8[RM]      class of the row
-  static constexpr int item = kind + BATCH_RM;                      // u8[RM]      tile of the row (in the batch)
-  static constexpr int seg = (item + BATCH_RM + 15) & ~15;          // int[NT+1]   chunk run -> product offset
-  static constexpr int sbs = seg + (TILE_NT + 1) * 4;               // int[NT]     chunk run -> B row start
-  static constexpr int sae = sbs + TILE_NT * 4;                     // int[NT]     chunk run -> tile A entry
-  static constexpr int srw = sae + TILE_NT * 4;                     // u16[NT]     chunk run -> batch row
-  static constexpr int bytes = (srw + TILE_NT * 2 + 15) & ~15;
+  static constexpr int pay = keys + C::PMAX * 4;                  // u32[PMAX]   idx -> plan word
+  static constexpr int sidx = pay + C::PMAX * 4;                  // u16[PMAX]   slot -> product index
+  static constexpr int sbk = sidx + C::PMAX * 2;                  // u16[PMAX]   slot -> bucket (repeats: output)
+  static constexpr int exrow = sbk + C::PMAX * 2;                 // u16[PMAX]   idx -> batch row
+  static constexpr int cnt = exrow + C::PMAX * 2;                 // int[NB+1]   sizes -> starts -> ends
+  static constexpr int hc = cnt + (C::NB + 1) * 4;               // int[NB+1]   heads -> head prefix
+  static constexpr int ae = (hc + (C::NB + 1) * 4 + 15) & ~15;   // int[RM+1]   A-entry offset of the row
+  static constexpr int pf = ae + (C::RM + 1) * 4;                // int[RM+1]   product offset of the row
+  static constexpr int bb = pf + (C::RM + 1) * 4;                // int[RM+1]   bucket base
+  static constexpr int out = bb + (C::RM + 1) * 4;               // int[RM+1]   output offset in the batch
+  static constexpr int rpa = out + (C::RM + 1) * 4;              // int[RM]     first A entry of the row
+  static constexpr int row = rpa + C::RM * 4;                    // int[RM]     local row index
+  static constexpr int cmin = row + C::RM * 4;                   // int[RM]     column range of the row
+  static constexpr int cmax = cmin + C::RM * 4;                  // int[RM]
+  static constexpr int sh = cmax + C::RM * 4;                    // u8[RM]      bucket width log2
+  static constexpr int kind = sh + C::RM;                        // u8[RM]      class of the row
+  static constexpr int item = kind + C::RM;                      // u8[RM]      tile of the row (in the batch)
+  static constexpr int seg = (item + C::RM + 15) & ~15;          // int[NT+1]   chunk run -> product offset
+  static constexpr int sbs = seg + (C::NT + 1) * 4;               // int[NT]     chunk run -> B row start
+  static constexpr int sae = sbs + C::NT * 4;                     // int[NT]     chunk run -> tile A entry
+  static constexpr int srw = sae + C::NT * 4;                     // u16[NT]     chunk run -> batch row
+  static constexpr int bytes = (srw + C::NT * 2 + 15) & ~15;
 };
 
-__global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __restrict__ items,
-                                                       const int* __restrict__ nitems, int* __restrict__ tqhead) {
+template <class C>
+__global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __restrict__ items,
+                                                     const int* __restrict__ nitems, int* __restrict__ tqhead,
+                                                     HeavyLists hl, const int* __restrict__ hcount) {
+  using SM = TileSmem<C>;
   extern __shared__ __align__(16) unsigned char sm[];
-  int* keys = reinterpret_cast<int*>(sm + TileSmem::keys);
-  unsigned* pay = reinterpret_cast<unsigned*>(sm + TileSmem::pay);
-  unsigned short* sidx = reinterpret_cast<unsigned short*>(sm + TileSmem::sidx);
-  unsigned short* sbk = reinterpret_cast<unsigned short*>(sm + TileSmem::sbk);
-  unsigned short* exrow = reinterpret_cast<unsigned short*>(sm + TileSmem::exrow);
-  int* cnt = reinterpret_cast<int*>(sm + TileSmem::cnt);
-  int* hc = reinterpret_cast<int*>(sm + TileSmem::hc);
-  int* s_ae = reinterpret_cast<int*>(sm + TileSmem::ae);
-  int* s_pf = reinterpret_cast<int*>(sm + TileSmem::pf);
-  int* s_bb = reinterpret_cast<int*>(sm + TileSmem::bb);
-  int* s_out = reinterpret_cast<int*>(sm + TileSmem::out);
-  int* s_rpa = reinterpret_cast<int*>(sm + TileSmem::rpa);
-  int* s_row = reinterpret_cast<int*>(sm + TileSmem::row);
-  int* s_cmin = reinterpret_cast<int*>(sm + TileSmem::cmin);
-  int* s_cmax = reinterpret_cast<int*>(sm + TileSmem::cmax);
-  uint8_t* s_sh = reinterpret_cast<uint8_t*>(sm + TileSmem::sh);
-  uint8_t* s_kind = reinterpret_cast<uint8_t*>(sm + TileSmem::kind);
-  uint8_t* s_item = reinterpret_cast<uint8_t*>(sm + TileSmem::item);
-  int* seg = reinterpret_cast<int*>(sm + TileSmem::seg);
-  int* sbs = reinterpret_cast<int*>(sm + TileSmem::sbs);
-  int* sae = reinterpret_cast<int*>(sm + TileSmem::sae);
-  unsigned short* srw = reinterpret_cast<unsigned short*>(sm + TileSmem::srw);
-  __shared__ int2 scratch2[TILE_NT / 32 + 1];
-  __shared__ int scratch[TILE_NT / 32 + 1];
+  int* keys = reinterpret_cast<int*>(sm + SM::keys);
+  unsigned* pay = reinterpret_cast<unsigned*>(sm + SM::pay);
+  unsigned short* sidx = reinterpret_cast<unsigned short*>(sm + SM::sidx);
+  unsigned short* sbk = reinterpret_cast<unsigned short*>(sm + SM::sbk);
+  unsigned short* exrow = reinterpret_cast<unsigned short*>(sm + SM::exrow);
+  int* cnt = reinterpret_cast<int*>(sm + SM::cnt);
+  int* hc = reinterpret_cast<int*>(sm + SM::hc);
+  int* s_ae = reinterpret_cast<int*>(sm + SM::ae);
+  int* s_pf = reinterpret_cast<int*>(sm + SM::pf);
+  int* s_bb = reinterpret_cast<int*>(sm + SM::bb);
+  int* s_out = reinterpret_cast<int*>(sm + SM::out);
+  int* s_rpa = reinterpret_cast<int*>(sm + SM::rpa);
+  int* s_row = reinterpret_cast<int*>(sm + SM::row);
+  int* s_cmin = reinterpret_cast<int*>(sm + SM::cmin);
+  int* s_cmax = reinterpret_cast<int*>(sm + SM::cmax);
+  uint8_t* s_sh = reinterpret_cast<uint8_t*>(sm + SM::sh);
+  uint8_t* s_kind = reinterpret_cast<uint8_t*>(sm + SM::kind);
+  uint8_t* s_item = reinterpret_cast<uint8_t*>(sm + SM::item);
+  int* seg = reinterpret_cast<int*>(sm + SM::seg);
+  int* sbs = reinterpret_cast<int*>(sm + SM::sbs);
+  int* sae = reinterpret_cast<int*>(sm + SM::sae);
+  unsigned short* srw = reinterpret_cast<unsigned short*>(sm + SM::srw);
+  __shared__ int2 scratch2[C::NT / 32 + 1];
+  __shared__ int scratch[C::NT / 32 + 1];
   // the popped items, and the tiles of the current batch
-  __shared__ int s_t0, s_qr0[BATCH_NI + 1], s_qheavy[BATCH_NI], s_qp[BATCH_NI], s_qe0[BATCH_NI];
-  __shared__ long long s_qP0[BATCH_NI + 1];
-  __shared__ int s_nb, s_bi[BATCH_NI], s_irb[BATCH_NI + 1], s_ie0[BATCH_NI], s_iub[BATCH_NI + 1], s_inext;
-  __shared__ long long s_iP0[BATCH_NI], s_idb[BATCH_NI];
-  __shared__ int s_uc[BATCH_NU];
-  constexpr int NT = TILE_NT, NW = NT / 32;
+  __shared__ int s_t0, s_qr0[C::NI], s_qr1[C::NI], s_qskip[C::NI], s_qp[C::NI], s_qe0[C::NI], s_qt[C::NI];
+  __shared__ long long s_qP0[C::NI];
+  __shared__ int s_nb, s_bi[C::NI], s_irb[C::NI + 1], s_ie0[C::NI], s_iub[C::NI + 1], s_inext;
+  __shared__ long long s_iP0[C::NI], s_idb[C::NI];
+  __shared__ int s_uc[C::NU];
+  constexpr int NT = C::NT, NW = NT / 32;
   const Group<NT> g{(int)threadIdx.x, scratch};
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int mloc = P.row_end - P.row_begin;
   if (P.Ro[mloc] > P.r_cap) return;  // plan too small: the host grows it and reruns
-  const int nt = *nitems;
+  // the queue: consecutive items, or (LIST) the HEAVY then HEAVY2 bin lists
+  const int n0 = C::LIST ? hcount[BIN_HEAVY] : 0;
+  const int nt = C::LIST ? n0 + hcount[BIN_HEAVY2] : *nitems;
 
   for (;;) {
-    // ---- pop BATCH_NI consecutive items (their cost varies with their rows' shapes) ----------------
-    if (tid == 0) s_t0 = atomicAdd(tqhead, BATCH_NI);
+    // ---- pop NI consecutive items (their cost varies with their rows' shapes) ---------------------
+    if (tid == 0) s_t0 = atomicAdd(tqhead, C::NI);
     __syncthreads();
     const int t0 = s_t0;
     if (t0 >= nt) break;
-    const int nq = min(BATCH_NI, nt - t0);
-    if (tid <= nq) {
-      const int r = items[t0 + tid];
-      s_qr0[tid] = r;
-      s_qP0[tid] = P.Ro[r];
-      if (tid < nq) {
-        s_qheavy[tid] = (P.cls[r] & CLS_HEAVY_PATH) ? 1 : 0;
-        s_qe0[tid] = P.rpA[P.row_begin + r];
+    const int nq = min(C::NI, nt - t0);
+    if (tid < nq) {
+      int r, r2, t, skip;
+      if constexpr (C::LIST) {  // a heavy row is an item of its own
+        const int x = t0 + tid;
+        r = x < n0 ? hl.rows[BIN_HEAVY][x] : hl.rows[BIN_HEAVY2][x - n0];
+        r2 = r + 1;
+        t = (int)(P.tscan[r] - 1);
+        skip = 0;
+      } else {
+        t = t0 + tid;
+        r = items[t];
+        r2 = items[t + 1];
+        skip = (P.cls[r] & CLS_HEAVY_PATH) ? 1 : 0;  // heavy rows: k_bitmap_rank or the big tiles
       }
+      s_qr0[tid] = r;
+      s_qr1[tid] = r2;
+      s_qt[tid] = t;
+      s_qskip[tid] = skip;
+      s_qP0[tid] = P.Ro[r];
+      s_qp[tid] = (int)(P.Ro[r2] - P.Ro[r]);
+      s_qe0[tid] = P.rpA[P.row_begin + r];
     }
     if (tid == 0) s_inext = 0;
     __syncthreads();
-    if (tid < nq) s_qp[tid] = (int)(s_qP0[tid + 1] - s_qP0[tid]);
-    __syncthreads();
     for (;;) {
-      // ---- the next batch: consecutive tiles of the pop, <= TILE_PMAX products, <= BATCH_RM rows
+      // ---- the next batch: consecutive tiles of the pop, <= C::PMAX products, <= C::RM rows
       if (tid == 0) {
         int k = s_inext, nb = 0, rows = 0;
         long long prod = 0;
         s_irb[0] = 0;
         for (; k < nq; ++k) {
-          if (s_qheavy[k]) continue;
-          const int nr = s_qr0[k + 1] - s_qr0[k];
+          if (s_qskip[k]) continue;
+          const int nr = s_qr1[k] - s_qr0[k];
           const int p = s_qp[k];
-          if (nb > 0 && (rows + nr > BATCH_RM || prod + p > TILE_PMAX)) break;
+          if (nb > 0 && (rows + nr > C::RM || prod + p > C::PMAX)) break;
           s_bi[nb] = k;
           s_iP0[nb] = s_qP0[k];
           s_ie0[nb] = s_qe0[k];
@@ -322,7 +351,7 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
       __syncthreads();
 
       // ---- 4. bucket starts (exclusive scan, contiguous ownership), scatter ------------------------
-      constexpr int BPT = (BATCH_NB + NT - 1) / NT;
+      constexpr int BPT = (C::NB + NT - 1) / NT;
       {
         int c8[BPT], mine = 0;
 #pragma unroll
@@ -343,7 +372,7 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
       __syncthreads();
       //      (the expand pass parked every product's column in keys[idx]; all of them are read into
       //      registers before the first slot is overwritten)
-      constexpr int IPT = TILE_PMAX / TILE_NT;
+      constexpr int IPT = C::PMAX / C::NT;
       {
         int bk[IPT], cl[IPT];
 #pragma unroll
@@ -430,7 +459,7 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
         s_iub[NI] = ub;
         if (dups) atomicAdd(reinterpret_cast<unsigned long long*>(P.dups_all), (unsigned long long)dups);
       }
-      if (tid < BATCH_NU) s_uc[tid] = 0;
+      if (tid < C::NU) s_uc[tid] = 0;
       __syncthreads();
 
       // ---- 7. ranks -> plan: heads in C order; repeats after them, bucketed by numeric unit --------
@@ -471,7 +500,7 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
           long long base = (long long)atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)(F - C));
           if (base + (F - C) > P.r_dcap) base = -1;  // too small: the host grows R and reruns
           s_idb[x] = base;
-          long long* db = P.dub + dub_index(s_iP0[x], t0 + s_bi[x]);
+          long long* db = P.dub + dub_index(s_iP0[x], s_qt[s_bi[x]]);
           const int hs = (C + NUM_SH - 1) / NUM_SH;
           int run = 0;
           for (int k = 0; k < hs; ++k) {
@@ -500,18 +529,31 @@ __global__ void __launch_bounds__(TILE_NT) k_tile_rank(SymProb P, const int* __r
 }
 
 cudaError_t tile_configure() {
-  return cudaFuncSetAttribute(k_tile_rank, cudaFuncAttributeMaxDynamicSharedMemorySize, TileSmem::bytes);
+  cudaError_t e = cudaFuncSetAttribute(k_tile_rank<TileSmall>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       TileSmem<TileSmall>::bytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(k_tile_rank<TileBig>, cudaFuncAttributeMaxDynamicSharedMemorySize, TileSmem<TileBig>::bytes);
+  return e;
 }
 
-int tile_occupancy() {
+int tile_occupancy(int big) {
   int nb = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_tile_rank, TILE_NT, TileSmem::bytes);
+  if (big) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_tile_rank<TileBig>, TileBig::NT, TileSmem<TileBig>::bytes);
+  else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_tile_rank<TileSmall>, TileSmall::NT, TileSmem<TileSmall>::bytes);
   return nb < 1 ? 1 : nb;
 }
 
 cudaError_t launch_tile_rank(cudaStream_t st, int grid, const SymProb& P, const int* items, const int* nitems,
                              int* tqhead) {
-  k_tile_rank<<<grid, TILE_NT, TileSmem::bytes, st>>>(P, items, nitems, tqhead);
+  HeavyLists none{};
+  k_tile_rank<TileSmall><<<grid, TileSmall::NT, TileSmem<TileSmall>::bytes, st>>>(P, items, nitems, tqhead, none,
+                                                                                  nullptr);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tile_heavy(cudaStream_t st, int grid, const SymProb& P, const HeavyLists& lists, const int* counts,
+                              int* qhead) {
+  k_tile_rank<TileBig><<<grid, TileBig::NT, TileSmem<TileBig>::bytes, st>>>(P, nullptr, nullptr, qhead, lists, counts);
   return cudaGetLastError();
 }
 

@@ -155,9 +155,12 @@ cudaError_t launch_narrow(cudaStream_t st, const long long* in, int* out, long l
 
 // k_light.cu — symbolic sort of the tiles, one tile per block iteration.
 cudaError_t tile_configure();
-int tile_occupancy();
+int tile_occupancy(int big);
 cudaError_t launch_tile_rank(cudaStream_t st, int grid, const SymProb& P, const int* items, const int* nitems,
                              int* tqhead);
+// big tiles: the HEAVY and HEAVY2 bins' rows (f <= 8192) sorted like tiles (SPG_OPT_HEAVY_SORT)
+cudaError_t launch_tile_heavy(cudaStream_t st, int grid, const SymProb& P, const HeavyLists& lists, const int* counts,
+                              int* qhead);
 
 // k_heavy.cu — symbolic sort of the heavy rows (column bitmap), one row per block iteration.
 cudaError_t heavy_configure();

@@ -106,6 +106,17 @@ def test_alpha_sweep_pair_variants(alpha):
         compare(A, B, run_gpu(A, B, **opts), ref=ref)
 
 
+@pytest.mark.parametrize("light", [0, 1024, 2048])
+def test_heavy_rows_as_big_tiles(light):
+    """SPG_OPT_HEAVY_SORT = 1: the register-cached heavy bins sorted in big tiles (8192
+    products, 1024 threads) instead of the column bitmap — same C as the oracle."""
+    A, B = W.make("cl10k")
+    ref = oracle.spgemm(A, B, nthreads=8)
+    compare(A, B, run_gpu(A, B, heavy_sort=1, light_max_flops=light), ref=ref)
+    A2 = W.chung_lu(30000, 30000, 2.1, 150000, 4000, 4000, 5.0, 1.1, 17)
+    compare(A2, A2, run_gpu(A2, A2, heavy_sort=1, light_max_flops=light))
+
+
 @pytest.mark.parametrize("dtype", [np.float64, np.float32])
 def test_packed_b_numeric(dtype):
     """SPG_OPT_PACK_B = 1: numeric gathers B through the packed {column, value} copy (automatic

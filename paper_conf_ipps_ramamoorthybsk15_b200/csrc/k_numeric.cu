@@ -141,48 +141,64 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
       mbar_wait(&s_bar[w][cb], (phases >> cb) & 1u);
       phases ^= 1u << cb;
     }
-    for (int o00 = lane; o00 < n; o00 += 32 * NUM_U) {
-      int e[NUM_U], q[NUM_U];
+    // one output: its A entry and B entry from the plan word(s), then the gathers
+    auto gather = [&](unsigned er, unsigned qo, int& col, V& prod) {
+      const int e = e0 + (int)er;
+      const int q = __ldg(P.Tb + e) + (int)qo;
+      const V a = __ldg(P.valA + e);
+      V b;
+      if constexpr (PACKED) {
+        const typename PB::T t = __ldg(Bp + q);
+        col = PB::col(t);
+        b = PB::val(t);
+      } else {
+        col = __ldg(P.colB + q);
+        b = __ldg(P.valB + q);
+      }
+      prod = a * b;
+    };
+    if (!wide) {
+      // full iterations without predicates, then the ragged tail
+      int o00 = lane;
+      for (; o00 + 32 * (NUM_U - 1) < n; o00 += 32 * NUM_U) {
+        unsigned wd[NUM_U];
 #pragma unroll
-      for (int x = 0; x < NUM_U; ++x) {
-        const int o = o00 + 32 * x;
-        q[x] = -1;
-        if (o < n) {
-          unsigned er, qo;
-          if (!wide) {
-            const unsigned wd = pb[o];
-            er = wd & 0xffffu;
-            qo = wd >> 16;
-          } else {
-            er = __ldcs(P.plan + cur.pw + 2 * (long long)o);
-            qo = __ldcs(P.plan + cur.pw + 2 * (long long)o + 1);
-          }
-          e[x] = e0 + (int)er;
-          q[x] = __ldg(P.Tb + e[x]) + (int)qo;
+        for (int x = 0; x < NUM_U; ++x) wd[x] = pb[o00 + 32 * x];
+        int col[NUM_U];
+        V prod[NUM_U];
+#pragma unroll
+        for (int x = 0; x < NUM_U; ++x) gather(wd[x] & 0xffffu, wd[x] >> 16, col[x], prod[x]);
+#pragma unroll
+        for (int x = 0; x < NUM_U; ++x) {
+          st_cs(ccol + o00 + 32 * x, col[x]);
+          st_cs(cval + o00 + 32 * x, prod[x]);
         }
       }
-      int col[NUM_U];
-      V a[NUM_U], b[NUM_U];
+      if (o00 < n) {  // fewer than 32 NUM_U outputs left: one predicated pass
+        int col[NUM_U];
+        V prod[NUM_U];
 #pragma unroll
-      for (int x = 0; x < NUM_U; ++x)
-        if (q[x] >= 0) {
-          a[x] = __ldg(P.valA + e[x]);
-          if constexpr (PACKED) {
-            const typename PB::T t = __ldg(Bp + q[x]);
-            col[x] = PB::col(t);
-            b[x] = PB::val(t);
-          } else {
-            col[x] = __ldg(P.colB + q[x]);
-            b[x] = __ldg(P.valB + q[x]);
+        for (int x = 0; x < NUM_U; ++x)
+          if (o00 + 32 * x < n) {
+            const unsigned wd = pb[o00 + 32 * x];
+            gather(wd & 0xffffu, wd >> 16, col[x], prod[x]);
           }
-        }
 #pragma unroll
-      for (int x = 0; x < NUM_U; ++x)
-        if (q[x] >= 0) {
-          const int o = o00 + 32 * x;
-          st_cs(ccol + o, col[x]);
-          st_cs(cval + o, a[x] * b[x]);
-        }
+        for (int x = 0; x < NUM_U; ++x)
+          if (o00 + 32 * x < n) {
+            st_cs(ccol + o00 + 32 * x, col[x]);
+            st_cs(cval + o00 + 32 * x, prod[x]);
+          }
+      }
+    } else {
+      const unsigned* __restrict__ pw = P.plan + cur.pw;
+      for (int o = lane; o < n; o += 32) {
+        int col;
+        V prod;
+        gather(__ldcs(pw + 2 * o), __ldcs(pw + 2 * o + 1), col, prod);
+        st_cs(ccol + o, col);
+        st_cs(cval + o, prod);
+      }
     }
     __syncwarp();  // every lane is done with buffer cb, and its stores precede the adds below
     // ---- repeated products landing in this unit's outputs (R records: B entry, A entry, output) -

@@ -266,98 +266,6 @@ __global__ void __launch_bounds__(256) k_unit_fill(const int* __restrict__ ucnt,
   if (blockIdx.x == 0 && threadIdx.x == 0) sm->nunits = n > 0 ? uscan[n - 1] : 0;
 }
 
-// Repeats of a HUGE (uncached bitmap) row, left unsorted at the end of its plan region with their
-// outputs in D, become R records bucketed by numeric unit (counting sort on o / NUM_SH): one block
-// per row; dub[dub_index(P0, t) + k] = first R record of unit k, k <= hs.
-constexpr int DS_NT = 1024;
-__global__ void __launch_bounds__(DS_NT) k_dup_sort(HeavyLists lists, int c0, int c1, int c2, SymProb P) {
-  extern __shared__ int s_cnt[];  // [hs + 1]
-  __shared__ int scratch_s[DS_NT / 32 + 1];
-  __shared__ long long s_base;
-  const Group<DS_NT> g{(int)threadIdx.x, scratch_s};
-  const int tid = threadIdx.x;
-  int b = blockIdx.x, bin = 0;
-  const int cnts[3] = {c0, c1, c2};
-  while (b >= cnts[bin]) b -= cnts[bin++];
-  const int li = lists.rows[bin][b];
-  const long long t = P.tscan[li] - 1;
-  const long long o0 = P.crow[li], c = P.crow[li + 1] - o0, P0 = P.Ro[li];
-  const bool wide = P.cls[li] & CLS_WIDE;
-  const int sw = wide ? 2 : 1;
-  const long long f = (P.Ro[li + 1] - P0) / sw;
-  const long long d = f - c;
-  const long long hs = (c + NUM_SH - 1) / NUM_SH;
-  if (d <= 0) return;
-  if (hs > DUP_SORT_UNITS) {
-    if (tid == 0) atomicOr(P.err, 4);
-    return;
-  }
-  long long* db = P.dub + dub_index(P0, t);
-  const int e0 = P.rpA[P.row_begin + li];
-  for (long long k = tid; k <= hs; k += DS_NT) s_cnt[k] = 0;
-  __syncthreads();
-  const long long w0 = P0 + c * sw;  // first repeat's entry
-  for (long long j = tid; j < d; j += DS_NT) atomicAdd(&s_cnt[P.D[w0 + j * sw] / NUM_SH], 1);
-  if (tid == 0) {
-    long long base = (long long)atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)d);
-    if (base + d > P.r_dcap) base = -1;  // too small: the host grows R and reruns
-    s_base = base;
-  }
-  __syncthreads();
-  const long long base = s_base;
-  {  // exclusive scan of the bucket sizes (contiguous ownership)
-    const int per = (int)((hs + DS_NT) / DS_NT);
-    int mine = 0;
-    for (int x = 0; x < per; ++x) {
-      const long long k = (long long)tid * per + x;
-      if (k < hs) mine += s_cnt[k];
-    }
-    int tot;
-    int run = g.excl_scan(mine, tot);
-    for (int x = 0; x < per; ++x) {
-      const long long k = (long long)tid * per + x;
-      if (k < hs) {
-        const int v = s_cnt[k];
-        s_cnt[k] = run;
-        db[k] = base + run;
-        run += v;
-      }
-    }
-    if (tid == 0) db[hs] = base + tot;
-  }
-  __syncthreads();
-  if (base < 0) return;
-  for (long long j = tid; j < d; j += DS_NT) {
-    const long long x = w0 + j * sw;
-    const unsigned o = P.D[x];
-    unsigned er, qo;
-    if (wide) {
-      er = P.plan[x];
-      qo = P.plan[x + 1];
-    } else {
-      const unsigned w = P.plan[x];
-      er = w & 0xffffu;
-      qo = w >> 16;
-    }
-    const int e = e0 + (int)er;
-    const int pos = atomicAdd(&s_cnt[o / NUM_SH], 1);
-    P.R[base + pos] = make_int4(P.Tb[e] + (int)qo, e, (int)o, 0);
-  }
-}
-
-cudaError_t dup_sort_configure() {
-  return cudaFuncSetAttribute(k_dup_sort, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              (DUP_SORT_UNITS + 1) * (int)sizeof(int));
-}
-
-cudaError_t launch_dup_sort(cudaStream_t st, const HeavyLists& lists, const int* counts_host, const SymProb& P) {
-  const long long n = (long long)counts_host[0] + counts_host[1] + counts_host[2];
-  if (n <= 0) return cudaSuccess;
-  k_dup_sort<<<(unsigned)n, DS_NT, (DUP_SORT_UNITS + 1) * sizeof(int), st>>>(lists, counts_host[0], counts_host[1],
-                                                                             counts_host[2], P);
-  return cudaGetLastError();
-}
-
 // ---- inclusive scan to int64 (three passes: tile scan, tile-sum scan, add) -------------------
 constexpr int SCAN_NT = 256, SCAN_IPT = 8, SCAN_TILE = SCAN_NT * SCAN_IPT;
 

@@ -491,16 +491,7 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
                 (long long)NUM_SH * DUP_SORT_UNITS);
   h->nnzC = h->hr->nnz;
   h->nitems = hs.nitems;
-  {  // repeats of HUGE rows as R records bucketed by numeric unit, then the numeric work units
-     // (structure only: built once, reused by every numeric call)
-    HeavyLists HL;
-    int hc[NUM_BINS];
-    for (int b = 0; b < NUM_BINS; ++b) {  // (register-cached bins bucket their repeats themselves)
-      HL.rows[b] = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
-      hc[b] = b == BIN_HUGE ? hs.counts[b] : 0;
-    }
-    CK(launch_dup_sort(h->stream, HL, hc, make_sym(h, A, B, crow)));
-    h->launches += 1;
+  {  // the numeric work units (structure only: built once, reused by every numeric call)
     const long long ucap = (long long)hs.nitems + h->nnzC / NUM_SH + 2;
     CK(h->units.ensure((size_t)ucap * sizeof(NumUnit)));
     const int n = hs.nitems;
@@ -624,7 +615,6 @@ spg_status create_common(spg_handle* out, int device, void* stream, spg_dtype dt
   cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, device);
   e = tile_configure();
   if (e == cudaSuccess) e = heavy_configure();
-  if (e == cudaSuccess) e = dup_sort_configure();
   if (e == cudaSuccess) e = cudaHostAlloc((void**)&h->hr, sizeof(HostRead), cudaHostAllocDefault);
   for (int c = 0; c < 6 && e == cudaSuccess; ++c) {
     e = cudaStreamCreateWithFlags(&h->aux[c], cudaStreamNonBlocking);

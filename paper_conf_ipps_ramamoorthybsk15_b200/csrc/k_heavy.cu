@@ -18,8 +18,8 @@
 // the passes and their head flags in a shared bit array, and write their repeats as R records
 // {B entry, A entry, output} bucketed by numeric unit at the end of the row; HUGE rows re-gather
 // columns per pass, keep the flag in a global byte per product (fl8) between pass 1 and pass 2,
-// and leave their repeats unsorted at the end of the plan region with the outputs in D
-// (k_dup_sort turns them into R records after symbolic).  Products are
+// and park their repeats at the end of the plan region with the outputs in D, then turn them into
+// R records bucketed by numeric unit at the end of the row.  Products are
 // visited in 32-product warp windows (coalesced within a B row); the run of each lane comes from
 // a REDUX.OR mask of run starts.  SINGLE rows (one non-empty B row) only copy their run.
 #include "kernels.cuh"
@@ -62,6 +62,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
   unsigned short* ctab = reinterpret_cast<unsigned short*>(sm + 3 * al16((RCAP + 1) * 4));  // window -> run
   unsigned char* region = sm + bmp_fixed_bytes<NT>();
   constexpr int REGION = SMEM - bmp_fixed_bytes<NT>();
+  static_assert(CACHED || (DUP_SORT_UNITS + 1) * 4 <= REGION, "HUGE rows' unit counters fit the region");
   __shared__ int scratch[NT / 32 + 1];
   const Group<NT> g{(int)threadIdx.x, scratch};
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -440,6 +441,71 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
               P.R[rbase + pos] = make_int4(sbs[r] + qo, sae[r], oo[s], 0);
             }
           }
+        }
+      }
+    }
+    if constexpr (!CACHED) {
+      // HUGE rows: the repeats parked at the end of the plan region (outputs in D) become R
+      // records bucketed by numeric unit — a counting sort on o / NUM_SH with the counters in the
+      // (now zero) region, while the row's plan words and D are still in L2
+      if (f > out) {
+        const int d = f - out;
+        const int hs = (out + NUM_SH - 1) / NUM_SH;
+        const int sw = wide ? 2 : 1;
+        int* ucnt = reinterpret_cast<int*>(region);
+        const unsigned* Drow = P.D + ro;
+        if (hs <= DUP_SORT_UNITS) {
+          for (int j = tid; j < d; j += NT) atomicAdd(&ucnt[Drow[(long long)(out + j) * sw] / NUM_SH], 1);
+          if (tid == 0) {
+            long long base = (long long)atomicAdd(reinterpret_cast<unsigned long long*>(P.dups), (unsigned long long)d);
+            if (base + d > P.r_dcap) base = -1;  // too small: the host grows R and reruns
+            s_rbase = base;
+          }
+          __syncthreads();
+          const long long rbase = s_rbase;
+          long long* db = P.dub + dub_index(ro, P.tscan[li] - 1);
+          {  // exclusive scan of the unit counters (contiguous ownership); db[k] = first record of unit k
+            const int per = (hs + NT) / NT;
+            int mine = 0;
+            for (int x = 0; x < per; ++x) {
+              const int k = tid * per + x;
+              if (k < hs) mine += ucnt[k];
+            }
+            int tot;
+            int run = g.excl_scan(mine, tot);
+            for (int x = 0; x < per; ++x) {
+              const int k = tid * per + x;
+              if (k < hs) {
+                const int v = ucnt[k];
+                ucnt[k] = run;
+                db[k] = rbase + run;
+                run += v;
+              }
+            }
+            if (tid == 0) db[hs] = rbase + tot;
+          }
+          __syncthreads();
+          if (rbase >= 0)
+            for (int j = tid; j < d; j += NT) {
+              const long long x = (long long)(out + j) * sw;
+              const unsigned o = Drow[x];
+              unsigned er, qo;
+              if (wide) {
+                er = prow[x];
+                qo = prow[x + 1];
+              } else {
+                const unsigned w = prow[x];
+                er = w & 0xffffu;
+                qo = w >> 16;
+              }
+              const int e = pa0 + (int)er;
+              const int pos = atomicAdd(&ucnt[o / NUM_SH], 1);
+              P.R[rbase + pos] = make_int4(P.Tb[e] + (int)qo, e, (int)o, 0);
+            }
+          __syncthreads();
+          for (int k = tid; k <= hs; k += NT) ucnt[k] = 0;  // the zero invariant (next row's barrier orders it)
+        } else if (tid == 0) {
+          atomicOr(P.err, 4);  // more numeric units than counters: the host reports NOT_SUPPORTED
         }
       }
     }

@@ -82,10 +82,10 @@ struct SymProb {
 // the item's repeated products (d_t = f_t - c_t) that land in its own outputs: a warp only ever
 // adds into outputs it stored itself, so no unit waits for another.  The repeats are 16-byte
 // records {B entry, A entry, item-relative output} in R, bucketed by unit (tiles: k_tile_rank;
-// register-cached heavy rows: k_bitmap_rank; HUGE rows: k_dup_sort after symbolic); unit k's
+// heavy rows: k_bitmap_rank at the end of the row); unit k's
 // records start at R[dub[dub_index(P0, t) + k]].
 constexpr int NUM_SH = 512;
-constexpr int DUP_SORT_UNITS = 48 * 1024;   // k_dup_sort's shared counters (rows up to 24M outputs)
+constexpr int DUP_SORT_UNITS = 48 * 1024;   // HUGE rows' unit counters in k_bitmap_rank (rows up to 24M outputs)
 __host__ __device__ __forceinline__ long long dub_index(long long P0, long long t) { return P0 / NUM_SH + 2 * t; }
 struct NumUnit {
   long long pw;   // plan word of the unit's first output
@@ -128,8 +128,6 @@ cudaError_t launch_unit_count(cudaStream_t st, int sms, const int* items, const 
 cudaError_t launch_unit_fill(cudaStream_t st, int sms, const int* ucnt, const long long* uscan, int n,
                              NumUnit* units, Small* small, const int* items, const long long* crow,
                              const long long* Ro, const uint8_t* cls, const int* rpA, int rb, const long long* dub);
-cudaError_t dup_sort_configure();
-cudaError_t launch_dup_sort(cudaStream_t st, const HeavyLists& lists, const int* counts_host, const SymProb& P);
 cudaError_t launch_classify(cudaStream_t st, int sms, const int* f, const uint8_t* nz, int rb, int re,
                             const ClassParams& prm, uint8_t* cls, int* pw, const HeavyLists& lists, Small* small);
 cudaError_t launch_tile_flags(cudaStream_t st, int sms, const int* f, const int* rpA, int rb, int re, int tile_cap,

@@ -125,8 +125,8 @@ typedef enum {
                                    per row), the rest light (a warp per row); default 256      */
   SPG_OPT_HEAVY_ORDER = 11,     /* order in which heavy-row blocks take rows from their queues:
                                    0 natural (row order), 1 (default) largest rows first in the
-                                   HUGE / HEAVY2 bins when they hold <= 2048 rows, 2 largest
-                                   first in every bin (long lists by log2 class) — with
+                                   HUGE / HEAVY2 bins, 2 largest first in every bin (rows ordered
+                                   by f_i in 8 classes per octave) — with
                                    FORCE_CLASS = HUGE the GPU analogues of the paper's Unsorted-
                                    and Sorted-Workqueue                    */
   SPG_OPT_PACK_B = 12,          /* numeric gathers B through a packed {column, value} copy (one

@@ -266,74 +266,80 @@ __global__ void __launch_bounds__(256) k_unit_fill(const int* __restrict__ ucnt,
   if (blockIdx.x == 0 && threadIdx.x == 0) sm->nunits = n > 0 ? uscan[n - 1] : 0;
 }
 
-// ---- inclusive scan to int64 (three passes: tile scan, tile-sum scan, add) -------------------
+// ---- inclusive scan to int64: one pass with decoupled look-back ----------------------------------
+// Tiles of SCAN_TILE elements take their index from a counter in launch order; a tile publishes
+// its aggregate (flag A), then — once its predecessors' prefix is known — its inclusive prefix
+// (flag P), each as one 64-bit word {flag:2, value:62}.  Warp 0 of a tile looks back over the
+// 32 preceding words at a time: it stops at the nearest P, summing the A values in between.  A
+// tile only waits on tiles with smaller indices, which were started before it, so the scan
+// cannot deadlock.  In place is allowed (a tile reads its whole input before writing).
 constexpr int SCAN_NT = 256, SCAN_IPT = 8, SCAN_TILE = SCAN_NT * SCAN_IPT;
+constexpr unsigned long long SCAN_FA = 1ull << 62, SCAN_FP = 2ull << 62, SCAN_VAL = SCAN_FA - 1;
 
 template <typename Tin>
-__global__ void __launch_bounds__(SCAN_NT) k_scan_tiles(const Tin* __restrict__ in, long long* __restrict__ out,
-                                                        long long n, long long* __restrict__ tile_sums) {
+__global__ void __launch_bounds__(SCAN_NT) k_scan_lb(const Tin* __restrict__ in, long long* __restrict__ out,
+                                                     long long n, unsigned long long* __restrict__ st,
+                                                     int* __restrict__ ctr) {
   __shared__ long long s_w[SCAN_NT / 32];
-  const long long base = (long long)blockIdx.x * SCAN_TILE + (long long)threadIdx.x * SCAN_IPT;
+  __shared__ long long s_pre;
+  __shared__ int s_tile;
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) s_tile = atomicAdd(ctr, 1);
+  __syncthreads();
+  const int tile = s_tile;
+  const long long base = (long long)tile * SCAN_TILE + (long long)threadIdx.x * SCAN_IPT;
   long long v[SCAN_IPT];
   long long run = 0;
 #pragma unroll
   for (int k = 0; k < SCAN_IPT; ++k) {
-    long long x = base + k < n ? (long long)in[base + k] : 0;
+    const long long x = base + k < n ? (long long)in[base + k] : 0;
     run += x;
     v[k] = run;
   }
-  // block exclusive scan of per-thread totals
-  long long incl = warp_incl_scan(run);
-  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const long long incl = warp_incl_scan(run);
   if (lane == 31) s_w[w] = incl;
   __syncthreads();
   if (w == 0) {
-    long long x = lane < SCAN_NT / 32 ? s_w[lane] : 0;
-    long long xi = warp_incl_scan(x);
+    const long long x = lane < SCAN_NT / 32 ? s_w[lane] : 0;
+    const long long xi = warp_incl_scan(x);
     if (lane < SCAN_NT / 32) s_w[lane] = xi - x;
-    if (lane == SCAN_NT / 32 - 1) tile_sums[blockIdx.x] = xi;
+    const long long agg = __shfl_sync(FULL, xi, SCAN_NT / 32 - 1);
+    volatile unsigned long long* vst = st;
+    if (tile == 0) {
+      if (lane == 0) {
+        vst[0] = SCAN_FP | (unsigned long long)agg;
+        s_pre = 0;
+      }
+    } else {
+      if (lane == 0) vst[tile] = SCAN_FA | (unsigned long long)agg;
+      long long pre = 0;
+      int p = tile - 1;  // lane k inspects tile p - k
+      for (;;) {
+        unsigned long long wd = SCAN_FP;  // below tile 0: a zero prefix
+        if (p - lane >= 0) {
+          do { wd = vst[p - lane]; } while ((wd >> 62) == 0);
+        }
+        const unsigned pm = __ballot_sync(FULL, (wd & SCAN_FP) != 0);
+        // the nearest P (lowest lane) ends the look-back; 64-bit sum of the lanes up to it
+        const int stop = pm ? __ffs(pm) - 1 : 31;
+        long long val = lane <= stop ? (long long)(wd & SCAN_VAL) : 0;
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) val += __shfl_xor_sync(FULL, val, d);
+        pre += val;
+        if (pm) break;
+        p -= 32;
+      }
+      if (lane == 0) {
+        vst[tile] = SCAN_FP | (unsigned long long)(pre + agg);
+        s_pre = pre;
+      }
+    }
   }
   __syncthreads();
-  const long long off = incl - run + s_w[w];
+  const long long off = incl - run + s_w[w] + s_pre;
 #pragma unroll
   for (int k = 0; k < SCAN_IPT; ++k)
     if (base + k < n) out[base + k] = v[k] + off;
-}
-
-// Exclusive scan of tile sums in place (one block, sequential over chunks).
-__global__ void __launch_bounds__(1024) k_scan_tile_sums(long long* __restrict__ s, int ntiles) {
-  __shared__ long long s_w[32];
-  __shared__ long long s_carry;
-  if (threadIdx.x == 0) s_carry = 0;
-  __syncthreads();
-  for (int c0 = 0; c0 < ntiles; c0 += 1024) {
-    const int i = c0 + threadIdx.x;
-    long long x = i < ntiles ? s[i] : 0;
-    long long incl = warp_incl_scan(x);
-    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    if (lane == 31) s_w[w] = incl;
-    __syncthreads();
-    if (w == 0) {
-      long long y = s_w[lane];
-      long long yi = warp_incl_scan(y);
-      s_w[lane] = yi - y;
-    }
-    __syncthreads();
-    long long excl = incl - x + s_w[w] + s_carry;
-    __syncthreads();
-    if (i < ntiles) s[i] = excl;
-    if (threadIdx.x == 1023) s_carry = excl + x;
-    __syncthreads();
-  }
-}
-
-__global__ void __launch_bounds__(SCAN_NT) k_scan_add(long long* __restrict__ out, long long n,
-                                                      const long long* __restrict__ tile_off) {
-  const long long base = (long long)blockIdx.x * SCAN_TILE;
-  const long long add = tile_off[blockIdx.x];
-  if (add == 0) return;
-  for (int k = threadIdx.x; k < SCAN_TILE; k += SCAN_NT)
-    if (base + k < n) out[base + k] += add;
 }
 
 // s_0 = 0, s_P = M, s_r = min{ i : Pf[i]*P >= r*F }.  Pf = int64[M+1].
@@ -467,97 +473,80 @@ cudaError_t launch_items(cudaStream_t st, int sms, const int* tflag, const long 
   return cudaGetLastError();
 }
 
-// Largest rows first: a bitmap bin's row list is sorted by descending f_i (one block, bitonic sort
-// of up to LPT_MAX (f, row) pairs in shared memory; longer lists keep their order).  Launched on
-// the bin's own stream, just before its kernel.
-// The bins' blocks take rows from a dynamic queue, so this is longest-processing-time-first
-// scheduling: the biggest HUGE rows (up to ~9x the bin average on webbase1m) start first instead
-// of forming the kernel's tail.
-constexpr int LPT_MAX = 2048;
-__global__ void __launch_bounds__(1024) k_sort_lists(HeavyLists lists, int b, const int* __restrict__ f, int rb,
-                                                     const Small* __restrict__ sm) {
-  __shared__ unsigned long long key[LPT_MAX];
+// Largest rows first: a bitmap bin's row list is put in descending f_i order (approximately: 8
+// classes per octave, order inside a class arbitrary — a one-block counting sort, the rows held
+// in shared memory when they fit, else through a scratch copy).  Launched on the bin's own
+// stream, just before its kernel.  The bins' blocks take rows from a dynamic queue, so this is
+// longest-processing-time-first scheduling: the biggest HUGE rows (up to ~9x the bin average on
+// webbase1m) start first instead of forming the kernel's tail.
+constexpr int ORD_NT = 1024, ORD_CAP = 4096, ORD_KEYS = 256;
+__global__ void __launch_bounds__(ORD_NT) k_order_list(HeavyLists lists, int b, const int* __restrict__ f, int rb,
+                                                      const Small* __restrict__ sm, int* __restrict__ tmp) {
+  __shared__ int hist[ORD_KEYS];
+  __shared__ int s_li[ORD_CAP];
   const int n = sm->counts[b];
-  if (n <= 1 || n > LPT_MAX) return;
+  if (n <= 1) return;
   int* list = lists.rows[b];
-  int np = 1;
-  while (np < n) np <<= 1;
-  for (int x = threadIdx.x; x < np; x += blockDim.x) {
-    unsigned long long k = 0;  // padding sorts last
-    if (x < n) {
-      const int li = list[x];
-      k = ((unsigned long long)(unsigned)f[rb + li] << 32) | (unsigned)li;
+  const bool insm = n <= ORD_CAP;
+  const int tid = threadIdx.x;
+  if (tid < ORD_KEYS) hist[tid] = 0;
+  __syncthreads();
+  auto key = [&](int li) {  // ascending key = descending f: exponent and 3 bits below the leading one
+    const unsigned v = (unsigned)max(f[rb + li], 1);
+    const int ex = 31 - __clz(v);
+    const unsigned m = ex >= 3 ? (v >> (ex - 3)) & 7u : (v << (3 - ex)) & 7u;
+    return ORD_KEYS - 1 - (ex * 8 + (int)m);
+  };
+  for (int x = tid; x < n; x += ORD_NT) {
+    const int li = list[x];
+    if (insm) s_li[x] = li;
+    atomicAdd(&hist[key(li)], 1);
+  }
+  __syncthreads();
+  if (tid < 32) {  // exclusive scan of the counters: 8 per lane
+    int c[ORD_KEYS / 32], sum = 0;
+#pragma unroll
+    for (int k = 0; k < ORD_KEYS / 32; ++k) {
+      c[k] = hist[tid * (ORD_KEYS / 32) + k];
+      sum += c[k];
     }
-    key[x] = k;
-  }
-  __syncthreads();
-  for (int size = 2; size <= np; size <<= 1)
-    for (int j = size >> 1; j > 0; j >>= 1) {
-      for (int x = threadIdx.x; x < np; x += blockDim.x) {
-        const int y = x ^ j;
-        if (y > x) {
-          const bool desc = (x & size) == 0;
-          const unsigned long long a = key[x], c = key[y];
-          if (desc ? a < c : a > c) { key[x] = c; key[y] = a; }
-        }
-      }
-      __syncthreads();
+    int run = warp_incl_scan(sum) - sum;
+#pragma unroll
+    for (int k = 0; k < ORD_KEYS / 32; ++k) {
+      hist[tid * (ORD_KEYS / 32) + k] = run;
+      run += c[k];
     }
-  for (int x = threadIdx.x; x < n; x += blockDim.x) list[x] = (int)(unsigned)(key[x] & 0xffffffffu);
-}
-
-// Lists longer than LPT_MAX (SPG_OPT_HEAVY_ORDER = 2): descending log2(f) classes — a one-block
-// counting sort through a scratch copy (order inside a class is arbitrary).
-__global__ void __launch_bounds__(1024) k_sort_lists_bins(HeavyLists lists, int b, const int* __restrict__ f, int rb,
-                                                          const Small* __restrict__ sm, int* __restrict__ tmp) {
-  __shared__ int hist[33];
-  const int n = sm->counts[b];
-  if (n <= LPT_MAX) return;
-  int* list = lists.rows[b];
-  if (threadIdx.x < 33) hist[threadIdx.x] = 0;
-  __syncthreads();
-  for (int x = threadIdx.x; x < n; x += blockDim.x) {
-    const int v = f[rb + list[x]];
-    atomicAdd(&hist[v > 0 ? 31 - __clz(v) : 32], 1);
   }
   __syncthreads();
-  if (threadIdx.x == 0) {  // exclusive prefix in descending class order
-    int run = 0;
-    for (int c = 31; c >= 0; --c) {
-      const int v = hist[c];
-      hist[c] = run;
-      run += v;
-    }
-    hist[32] = run;
+  for (int x = tid; x < n; x += ORD_NT) {
+    const int li = insm ? s_li[x] : list[x];
+    const int pos = atomicAdd(&hist[key(li)], 1);
+    if (insm) list[pos] = li;
+    else tmp[pos] = li;
   }
+  if (insm) return;
   __syncthreads();
-  for (int x = threadIdx.x; x < n; x += blockDim.x) {
-    const int li = list[x], v = f[rb + li];
-    tmp[atomicAdd(&hist[v > 0 ? 31 - __clz(v) : 32], 1)] = li;
-  }
-  __syncthreads();
-  for (int x = threadIdx.x; x < n; x += blockDim.x) list[x] = tmp[x];
+  for (int x = tid; x < n; x += ORD_NT) list[x] = tmp[x];
 }
 
 cudaError_t launch_sort_list(cudaStream_t st, const HeavyLists& lists, int bin, const int* f, int rb,
                              const Small* small, int* tmp) {
-  k_sort_lists<<<1, 1024, 0, st>>>(lists, bin, f, rb, small);
-  if (tmp) k_sort_lists_bins<<<1, 1024, 0, st>>>(lists, bin, f, rb, small, tmp);
+  k_order_list<<<1, ORD_NT, 0, st>>>(lists, bin, f, rb, small, tmp);
   return cudaGetLastError();
 }
 
-size_t scan_tmp_elems(long long n) { return (size_t)((n + SCAN_TILE - 1) / SCAN_TILE) + 1; }
-int scan_launches(long long n) { return n <= 0 ? 0 : (n > SCAN_TILE ? 3 : 1); }
+size_t scan_tmp_elems(long long n) { return (size_t)((n + SCAN_TILE - 1) / SCAN_TILE) + 2; }
+int scan_launches(long long n) { return n <= 0 ? 0 : 1; }
 
+// tmp: scan_tmp_elems(n) words — the tiles' status words, then the tile counter
 template <typename Tin>
 cudaError_t launch_incl_scan(cudaStream_t st, const Tin* in, long long* out, long long n, long long* tmp) {
   if (n <= 0) return cudaSuccess;
   const int ntiles = (int)((n + SCAN_TILE - 1) / SCAN_TILE);
-  k_scan_tiles<Tin><<<ntiles, SCAN_NT, 0, st>>>(in, out, n, tmp);
-  if (ntiles > 1) {
-    k_scan_tile_sums<<<1, 1024, 0, st>>>(tmp, ntiles);
-    k_scan_add<<<ntiles, SCAN_NT, 0, st>>>(out, n, tmp);
-  }
+  cudaError_t e = cudaMemsetAsync(tmp, 0, (size_t)(ntiles + 1) * sizeof(long long), st);
+  if (e != cudaSuccess) return e;
+  k_scan_lb<Tin><<<ntiles, SCAN_NT, 0, st>>>(in, out, n, reinterpret_cast<unsigned long long*>(tmp),
+                                            reinterpret_cast<int*>(tmp + ntiles));
   return cudaGetLastError();
 }
 template cudaError_t launch_incl_scan<int>(cudaStream_t, const int*, long long*, long long, long long*);

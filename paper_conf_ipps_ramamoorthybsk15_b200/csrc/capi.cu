@@ -244,18 +244,13 @@ spg_status fork_heavy(spg_handle h, const spg_csr* A, const spg_csr* B, long lon
     long long grid = (long long)h->occ_heavy[b] * h->sms;
     if (h->huge_slots_opt > 0 && h->huge_slots_opt < grid) grid = h->huge_slots_opt;
     int* list = h->lists.as<int>() + (size_t)b * (size_t)(Mloc > 0 ? Mloc : 1);
-    // largest rows first (HEAVY_ORDER 1: the HUGE and HEAVY2 lists when they hold <= 2048 rows;
-    // 2: every list, long ones by log2 class; 0: natural order)
+    // largest rows first (HEAVY_ORDER 1: the HUGE and HEAVY2 lists; 2: every list; 0: natural order)
     if (Mloc > 0 && (h->heavy_order == 2 || (h->heavy_order == 1 && b != BIN_HEAVY))) {
       HeavyLists L3;
       for (int c = 0; c < NUM_BINS; ++c) L3.rows[c] = h->lists.as<int>() + (size_t)c * (size_t)Mloc;
-      int* tmp = nullptr;
-      if (h->heavy_order == 2) {
-        CK(h->lsort.ensure((size_t)NUM_BINS * (size_t)Mloc * sizeof(int)));
-        tmp = h->lsort.as<int>() + (size_t)b * (size_t)Mloc;
-      }
-      CK(launch_sort_list(st, L3, b, h->f.as<int>(), h->rb, ds, tmp));
-      h->launches += tmp ? 2 : 1;
+      CK(h->lsort.ensure((size_t)NUM_BINS * (size_t)Mloc * sizeof(int)));
+      CK(launch_sort_list(st, L3, b, h->f.as<int>(), h->rb, ds, h->lsort.as<int>() + (size_t)b * (size_t)Mloc));
+      h->launches += 1;
     }
     CK(launch_heavy_rank(b, st, (int)grid, P, list, ds->counts + b, B->ncols));
     h->launches++;

@@ -41,7 +41,7 @@ struct TileCfg {
   static constexpr int PMAX = PMAX_;   // products per batch
   static constexpr int NT = NT_;       // threads
   static constexpr bool LIST = LIST_;  // pop heavy rows from the bin lists (else items)
-  static constexpr int RM = 512;       // rows per batch
+  static constexpr int RM = NT_ < 512 ? NT_ : 512;  // rows per batch
   static constexpr int NI = 16;        // items per queue pop
   static constexpr int NB = PMAX / TILE_BK + RM;  // buckets per batch (ceil per row)
   static constexpr int NU = NI + PMAX / NUM_SH;   // numeric units of a batch's items
@@ -50,7 +50,7 @@ struct TileCfg {
   static_assert(TILE_RM <= RM, "a tile fits a batch");
 };
 using TileSmall = TileCfg<TILE_PMAX, TILE_NT, false>;
-using TileBig = TileCfg<2 * TILE_PMAX, 2 * TILE_NT, true>;
+using TileBig = TileCfg<HEAVY_CAP, 1024, true>;
 constexpr int TILE_EU = 4;  // 32-product windows per warp per step (loads in flight)
 
 // Run of product jw + lane for a window starting inside run rb (warp-uniform); advances rb to

@@ -220,6 +220,29 @@ def test_split_points_exact():
         spg.spg_spgemm_free(h)
 
 
+def test_split_points_flop_prefix_beyond_2_32():
+    """The flop prefix (one-pass look-back scan over ~60 tiles) passes 2^32: 120000 rows of one
+    entry each, most pointing at a 65535-long B row (4.4e9 products), some at a 1000-long row,
+    every seventh empty.  Only the analysis and the scan run (no symbolic)."""
+    M = 120000
+    i = np.arange(M)
+    has = (i % 7) != 0
+    col = np.where(i % 3 == 0, 1, 0).astype(np.int32)[has]
+    rp = np.concatenate([[0], np.cumsum(has)]).astype(np.int32)
+    A = W.CSR(M, 2, rp, col, np.ones(col.shape[0]))
+    bcol = np.concatenate([np.arange(65535), np.arange(1000)]).astype(np.int32)
+    B = W.CSR(2, 65535, np.array([0, 65535, 66535], np.int32), bcol, np.ones(bcol.shape[0]))
+    f = oracle.row_flops(A, B)
+    assert int(f.sum()) > 2**32
+    h = spg.spg_create(0, None, torch.float64)
+    try:
+        dA, dB = to_dev(A), to_dev(B)
+        for P in (1, 2, 3, 8, 13):
+            np.testing.assert_array_equal(spg.spg_split_points(h, dA, dB, P), oracle.split_points(f, P))
+    finally:
+        spg.spg_spgemm_free(h)
+
+
 def test_error_paths():
     A = W.random_csr(10, 8, 0.3, 1)
     B = W.random_csr(9, 8, 0.3, 2)

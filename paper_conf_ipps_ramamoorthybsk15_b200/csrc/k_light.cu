@@ -344,9 +344,22 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
         const int j = exrow[idx];
         return s_kind[j] >= CLS_TINY ? s_bb[j] + ((keys[idx] - s_cmin[j]) >> s_sh[j]) : -1;
       };
-      for (int idx = tid; idx < PT; idx += NT) {
-        const int b = bucket_of(idx);
-        if (b >= 0) atomicAdd(&cnt[b], 1);
+      // every product's bucket and column in registers (thread tid owns products tid + u NT);
+      // single: bit u set for a product of a SINGLE row (placed in order, no sort)
+      constexpr int IPT = C::PMAX / C::NT;
+      int bk[IPT], cl[IPT];
+      unsigned single = 0;
+#pragma unroll
+      for (int u = 0; u < IPT; ++u) {
+        const int idx = tid + u * NT;
+        bk[u] = -1;
+        cl[u] = 0;
+        if (idx < PT) {
+          bk[u] = bucket_of(idx);
+          cl[u] = keys[idx];
+          if (bk[u] >= 0) atomicAdd(&cnt[bk[u]], 1);
+          else if (s_kind[exrow[idx]] == CLS_SINGLE) single |= 1u << u;
+        }
       }
       __syncthreads();
 
@@ -372,16 +385,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
       __syncthreads();
       //      (the expand pass parked every product's column in keys[idx]; all of them are read into
       //      registers before the first slot is overwritten)
-      constexpr int IPT = C::PMAX / C::NT;
       {
-        int bk[IPT], cl[IPT];
-#pragma unroll
-        for (int u = 0; u < IPT; ++u) {
-          const int idx = tid + u * NT;
-          bk[u] = idx < PT ? bucket_of(idx) : -1;
-          cl[u] = idx < PT ? keys[idx] : 0;
-        }
-        __syncthreads();
 #pragma unroll
         for (int u = 0; u < IPT; ++u) {
           const int b = bk[u];
@@ -484,8 +488,10 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
           atomicAdd(&s_uc[s_iub[it] + o / NUM_SH], 1);
         }
       }
-      for (int idx = tid; idx < PT; idx += NT)  // SINGLE rows: products already in column order
-        if (s_kind[exrow[idx]] == CLS_SINGLE) {
+#pragma unroll
+      for (int u = 0; u < IPT; ++u)  // SINGLE rows: products already in column order
+        if (single >> u & 1u) {
+          const int idx = tid + u * NT;
           const int j = exrow[idx];
           const int it = s_item[j];
           P.plan[s_iP0[it] + s_out[j] - s_out[s_irb[it]] + idx - s_pf[j]] = pay[idx];

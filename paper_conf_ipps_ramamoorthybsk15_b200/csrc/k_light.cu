@@ -76,14 +76,14 @@ struct TileSmem {
   static constexpr int sbk = sidx + C::PMAX * 2;                  // u16[PMAX]   slot -> bucket (repeats: output)
   static constexpr int exrow = sbk + C::PMAX * 2;                 // u16[PMAX]   idx -> batch row
   static constexpr int cnt = exrow + C::PMAX * 2;                 // int[NB+1]   sizes -> starts -> ends
-  static constexpr int hc = cnt + (C::NB + 1) * 4;               // int[NB+1]   heads -> head prefix
-  static constexpr int ae = (hc + (C::NB + 1) * 4 + 15) & ~15;   // int[RM+1]   A-entry offset of the row
+  static constexpr int ae = (cnt + (C::NB + 1) * 4 + 15) & ~15;  // int[RM+1]   A-entry offset of the row
   static constexpr int pf = ae + (C::RM + 1) * 4;                // int[RM+1]   product offset of the row
   static constexpr int bb = pf + (C::RM + 1) * 4;                // int[RM+1]   bucket base
   static constexpr int out = bb + (C::RM + 1) * 4;               // int[RM+1]   output offset in the batch
   static constexpr int rpa = out + (C::RM + 1) * 4;              // int[RM]     first A entry of the row
   static constexpr int row = rpa + C::RM * 4;                    // int[RM]     local row index
-  static constexpr int cmin = row + C::RM * 4;                   // int[RM]     column range of the row
+  static constexpr int cmin = row + C::RM * 4;                   // int[RM]     column range of the row (later:
+                                                                  //             heads before the row)
   static constexpr int cmax = cmin + C::RM * 4;                  // int[RM]
   static constexpr int sh = cmax + C::RM * 4;                    // u8[RM]      bucket width log2
   static constexpr int kind = sh + C::RM;                        // u8[RM]      class of the row
@@ -107,7 +107,6 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
   unsigned short* sbk = reinterpret_cast<unsigned short*>(sm + SM::sbk);
   unsigned short* exrow = reinterpret_cast<unsigned short*>(sm + SM::exrow);
   int* cnt = reinterpret_cast<int*>(sm + SM::cnt);
-  int* hc = reinterpret_cast<int*>(sm + SM::hc);
   int* s_ae = reinterpret_cast<int*>(sm + SM::ae);
   int* s_pf = reinterpret_cast<int*>(sm + SM::pf);
   int* s_bb = reinterpret_cast<int*>(sm + SM::bb);
@@ -131,6 +130,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
   __shared__ int s_nb, s_bi[C::NI], s_irb[C::NI + 1], s_ie0[C::NI], s_iub[C::NI + 1], s_inext;
   __shared__ long long s_iP0[C::NI], s_idb[C::NI];
   __shared__ int s_uc[C::NU];
+  __shared__ int s_htot;
   constexpr int NT = C::NT, NW = NT / 32;
   const Group<NT> g{(int)threadIdx.x, scratch};
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -334,10 +334,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
       }
       __syncthreads();
       const int NBt = s_bb[NR];
-      for (int b = tid; b <= NBt; b += NT) {
-        cnt[b] = 0;
-        hc[b] = 0;
-      }
+      for (int b = tid; b <= NBt; b += NT) cnt[b] = 0;
       __syncthreads();
       // bucket of product idx (light rows; -1: SINGLE row, no sort)
       auto bucket_of = [&](int idx) -> int {
@@ -399,50 +396,90 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
       __syncthreads();
       const int Pg = NBt > 0 ? cnt[NBt - 1] : 0;
 
-      // ---- 5. heads: first slot of its column within the bucket -----------------------------------
-      //      (non-head marks are applied after a barrier, so no thread reads a key while another
-      //      marks it)
-      unsigned nonhead = 0;  // bit u: slot tid + u·NT is not a head
-      for (int x = tid, u = 0; x < Pg; x += NT, ++u) {
-        const int b = sbk[x];
-        const int s0 = b ? cnt[b - 1] : 0;
-        const int kx = keys[x];
-        bool head = true;
-        for (int y = s0; y < x; ++y)
-          if (keys[y] == kx) { head = false; break; }
-        if (head) atomicAdd(&hc[b], 1);
-        else nonhead |= 1u << u;
-      }
-      __syncthreads();
-      for (int x = tid, u = 0; x < Pg; x += NT, ++u)
-        if (nonhead >> u & 1u) keys[x] |= int(0x80000000);
-      {  // head prefix per bucket; hc[NBt] = total
-        int c8[BPT], mine = 0;
+      // ---- 5. sort every bucket in place: slot x moves to s0 + #{y : (key, slot) of y < that of x}
+      //         (buckets hold ~TILE_BK products; the permutation goes through registers)
+      {
+        static_assert(C::PMAX <= 65536, "slot and product index in 16 bits each");
+        unsigned nps[IPT];  // new slot | product index << 16; ~0u: none
+        int nkey[IPT];
 #pragma unroll
-        for (int k = 0; k < BPT; ++k) {
-          const int b = tid * BPT + k;
-          c8[k] = b < NBt ? hc[b] : 0;
-          mine += c8[k];
+        for (int u = 0; u < IPT; ++u) {
+          const int x = tid + u * NT;
+          nps[u] = ~0u;
+          if (x < Pg) {
+            const int bb = sbk[x];
+            const int s0 = bb ? cnt[bb - 1] : 0, s1 = cnt[bb];
+            const int kx = keys[x];
+            int pos = x;
+            if (s1 - s0 > 1) {
+              pos = s0;
+              for (int y = s0; y < s1; ++y) {
+                const int ky = keys[y];
+                pos += (ky < kx) || (ky == kx && y < x);
+              }
+            }
+            nps[u] = (unsigned)pos | ((unsigned)sidx[x] << 16);
+            nkey[u] = kx;
+          }
         }
-        int tot;
-        int run = g.excl_scan(mine, tot);  // (its barriers also order the marks above)
+        __syncthreads();
 #pragma unroll
-        for (int k = 0; k < BPT; ++k) {
-          const int b = tid * BPT + k;
-          if (b < NBt) hc[b] = run;
-          run += c8[k];
+        for (int u = 0; u < IPT; ++u) {
+          const int pos = (int)(nps[u] & 0xffffu);
+          if (nps[u] != ~0u && pos != tid + u * NT) {
+            keys[pos] = nkey[u];
+            sidx[pos] = (unsigned short)(nps[u] >> 16);
+          }
         }
-        if (tid == 0) hc[NBt] = tot;
       }
       __syncthreads();
 
-      // ---- 6. c_j and output offsets of the rows (in the batch; a tile's outputs start at the
-      //         offset of its first row) ----------------------------------------------------------
+      // ---- 6. heads: the first slot of its bucket or a column unlike the previous slot's; a block
+      //         scan of the head flags (slots are in (row, column) order) numbers the outputs:
+      //         keys[x] = index of the column's head among the batch's heads, sign bit = repeat
+      {
+        unsigned hf = 0;
+        int nh = 0;
+#pragma unroll
+        for (int k = 0; k < IPT; ++k) {
+          const int x = tid * IPT + k;
+          if (x < Pg) {
+            const bool h = x == 0 || sbk[x] != sbk[x - 1] || keys[x] != keys[x - 1];
+            hf |= (unsigned)h << k;
+            nh += h;
+          }
+        }
+        int tot;
+        int run = g.excl_scan(nh, tot);  // (its barriers order the reads above before the writes below)
+#pragma unroll
+        for (int k = 0; k < IPT; ++k) {
+          const int x = tid * IPT + k;
+          if (x < Pg) {
+            const bool h = hf >> k & 1u;
+            run += h;
+            keys[x] = (run - 1) | (h ? 0 : int(0x80000000));
+          }
+        }
+        if (tid == 0) s_htot = tot;
+      }
+      __syncthreads();
+
+      // ---- 7. c_j and output offsets of the rows (in the batch; a tile's outputs start at the
+      //         offset of its first row); s_cmin[j] = heads before row j's first slot -------------
       {
         int cj = 0;
         if (tid < NR) {
           const int k = s_kind[tid];
-          cj = k >= CLS_TINY ? hc[s_bb[tid + 1]] - hc[s_bb[tid]] : (k == CLS_SINGLE ? s_pf[tid + 1] - s_pf[tid] : 0);
+          if (k >= CLS_TINY) {
+            const int b0 = s_bb[tid], b1 = s_bb[tid + 1];
+            const int x0 = b0 ? cnt[b0 - 1] : 0, x1 = b1 ? cnt[b1 - 1] : 0;
+            const int h0 = x0 < Pg ? keys[x0] & 0x7fffffff : s_htot;  // (a row's first slot is a head)
+            const int h1 = x1 < Pg ? keys[x1] & 0x7fffffff : s_htot;
+            cj = h1 - h0;
+            s_cmin[tid] = h0;
+          } else if (k == CLS_SINGLE) {
+            cj = s_pf[tid + 1] - s_pf[tid];
+          }
           P.crow[s_row[tid] + 1] = cj;
         }
         int tot;
@@ -466,24 +503,16 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
       if (tid < C::NU) s_uc[tid] = 0;
       __syncthreads();
 
-      // ---- 7. ranks -> plan: heads in C order; repeats after them, bucketed by numeric unit --------
+      // ---- 8. plan: heads in C order; repeats after them, bucketed by numeric unit ----------------
       for (int x = tid; x < Pg; x += NT) {
-        const int b = sbk[x];
-        const int s0 = b ? cnt[b - 1] : 0, s1 = cnt[b];
         const int kx = keys[x];
-        const int k = kx & 0x7fffffff;
-        int u = 0;
-        for (int y = s0; y < s1; ++y) {
-          const int ky = keys[y];
-          u += (ky >= 0 && ky < k);
-        }
         const int jr = exrow[sidx[x]];
         const int it = s_item[jr];
         // output of the product's column, relative to its tile
-        const int o = s_out[jr] - s_out[s_irb[it]] + hc[b] - hc[s_bb[jr]] + u;
+        const int o = s_out[jr] - s_out[s_irb[it]] + (kx & 0x7fffffff) - s_cmin[jr];
         if (kx >= 0) {
           P.plan[s_iP0[it] + o] = pay[sidx[x]];
-        } else {  // a repeat: its output parked in sbk (read above, own slot only)
+        } else {  // a repeat: its output parked in sbk (own slot only)
           sbk[x] = (unsigned short)o;
           atomicAdd(&s_uc[s_iub[it] + o / NUM_SH], 1);
         }

@@ -13,9 +13,11 @@ namespace spg {
 
 // f_i = sum over stored A(i,k) of len_B(k); nz_i = #entries with len_B(k) > 0 (capped at 2), plus
 // the NZ_* size flags (A row longer than 512 / 1024 / 65535 entries, a B row longer than 65535).  One block owns ROWS
-// consecutive rows; its threads stride over the rows' A entries (coalesced), find the owning row
-// by binary search in the cached row_ptr tile, pre-reduce per warp and row, and add into shared
-// 32-bit accumulators.
+// consecutive rows; its threads stride over the rows' A entries (coalesced) and find the owning row
+// by binary search in the cached row_ptr tile; rows are non-decreasing across a warp's lanes, so
+// a segmented warp scan (5 shuffles of one 64-bit word: products in
+// the low 40 bits, non-empty runs above) leaves each row's sums in its last lane, which adds
+// them into 32-bit shared accumulators.
 template <int ROWS>
 __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict__ rpA, const int* __restrict__ colA,
                                                     int K, const int* __restrict__ rpB, int* __restrict__ f_out,
@@ -43,7 +45,7 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
   int bad = 0;
   for (int base = e0; base < e1; base += ROWS) {  // uniform trip count: warp collectives below
     const int e = base + t;
-    bool act = e < e1;
+    const bool act = e < e1;
     int L = 0, r = -1;
     if (act) {
       const int k = colA[e];
@@ -55,22 +57,26 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
       Tl[e] = L;
       if (L > 65535) atomicOr(&s_lb[r], 1);
     }
-    act = r >= 0;
-    const unsigned nzb = __ballot_sync(FULL, act && L > 0);
-    const unsigned grp = __match_any_sync(FULL, r);
-    if (act) {
-      const unsigned lo = __reduce_add_sync(grp, (unsigned)L & 0xffffu);
-      const unsigned hi = __reduce_add_sync(grp, (unsigned)L >> 16);
-      if (lane == __ffs(grp) - 1) {
-        const unsigned long long tot = ((unsigned long long)hi << 16) + lo;
-        if (tot > (unsigned long long)INT_MAX) {
-          bad |= 2;
-        } else {
-          const unsigned old = atomicAdd(&s_f[r], (unsigned)tot);
-          if ((unsigned long long)old + tot > (unsigned long long)INT_MAX) bad |= 2;
-        }
-        atomicAdd(&s_nz[r], __popc(grp & nzb));
+    // segmented inclusive scan over the lanes of each row (inactive lanes, r = -1, come last)
+    const int rprev = __shfl_up_sync(FULL, r, 1);
+    const unsigned heads = __ballot_sync(FULL, lane == 0 || r != rprev);
+    const int sstart = 31 - __clz(heads & ((2u << lane) - 1u));
+    unsigned long long v = act ? (unsigned long long)(unsigned)L + (L > 0 ? (1ull << 40) : 0ull) : 0ull;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const unsigned long long o = __shfl_up_sync(FULL, v, d);
+      if (lane - d >= sstart) v += o;
+    }
+    const bool last = lane == 31 || ((heads >> (lane + 1)) & 1u);
+    if (act && last) {
+      const unsigned long long tot = v & ((1ull << 40) - 1);
+      if (tot > (unsigned long long)INT_MAX) {
+        bad |= 2;
+      } else {
+        const unsigned old = atomicAdd(&s_f[r], (unsigned)tot);
+        if ((unsigned long long)old + tot > (unsigned long long)INT_MAX) bad |= 2;
       }
+      atomicAdd(&s_nz[r], (int)(v >> 40));
     }
   }
   __syncthreads();

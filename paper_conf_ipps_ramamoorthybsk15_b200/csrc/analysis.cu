@@ -5,8 +5,8 @@
 //
 // No 64-bit shared-memory atomics anywhere: on sm_100a they compile to ATOMS.CAST.SPIN.64
 // CAS loops that serialise under contention (hub rows, 7-way class counters).  Sums are
-// pre-reduced per warp with MATCH.ANY + REDUX (split in 16-bit halves so they cannot wrap)
-// and accumulated with native 32-bit ATOMS.
+// pre-reduced per warp — per-row sums by a segmented warp scan (k_row_flops), class counters by
+// MATCH.ANY + REDUX in 16-bit halves (k_classify) — and accumulated with native 32-bit ATOMS.
 #include "kernels.cuh"
 
 namespace spg {

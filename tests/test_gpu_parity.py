@@ -559,6 +559,35 @@ def test_fallback_clustered_columns():
     compare(A, B, run_gpu(A, B), exact_values=True)
 
 
+def test_columns_up_to_2_31():
+    """B with 2^31 - 1 columns (the int32 limit), its first and last column used: light rows whose
+    column range spans everything (bucket widths up to 2^31), heavy rows as big tiles (B wider
+    than 2^20 columns) and HUGE rows making 2048 bitmap column-tile passes."""
+    rng = np.random.default_rng(41)
+    N = 2**31 - 1
+    K = 3000
+    rows = []
+    for k in range(K):
+        c = rng.choice(N - 2, 30, replace=False) + 1
+        if k % 97 == 0:
+            c[0] = 0
+        if k % 89 == 0:
+            c[1] = N - 1
+        rows.append(np.unique(c))
+    rp = np.concatenate([[0], np.cumsum([len(r) for r in rows])]).astype(np.int32)
+    B = W.CSR(K, N, rp, np.concatenate(rows).astype(np.int32),
+              rng.integers(-4, 5, int(rp[-1])).astype(np.float64))
+    lens = np.concatenate([rng.integers(0, 6, 480), np.full(14, 200), np.full(6, 400)])
+    rng.shuffle(lens)
+    arp = np.concatenate([[0], np.cumsum(lens)]).astype(np.int32)
+    acol = np.concatenate([np.sort(rng.choice(K, n, replace=False)) for n in lens]).astype(np.int32)
+    A = W.CSR(len(lens), K, arp, acol, rng.integers(-4, 5, int(arp[-1])).astype(np.float64))
+    got = run_gpu(A, B)
+    st = got[3]
+    assert st["heavy_rows"] >= 20 and st["class_rows"][6] >= 6  # HUGE rows were exercised
+    compare(A, B, got, exact_values=True)
+
+
 # ---- sparse x dense (csrmm, PAPER.md L289) ---------------------------------------------------
 def _csrmm_gpu(A, D, **opts):
     dA = to_dev(A)

@@ -38,6 +38,8 @@
  *   - Every function returns a status and never throws, exits or aborts across the ABI.
  *   - CUDA / NCCL failures map to SPG_ERR_CUDA / SPG_ERR_NCCL; spg_last_error(h) gives
  *     the detail.  Asynchronous kernel faults surface at the next synchronising call.
+ *   - nnz of an input is at most SPG_MAX_NNZ = 2^31 - 4097 (kernels form entry indices a block
+ *     stride past a row range in 32-bit arithmetic); larger inputs give SPG_ERR_INDEX_OVERFLOW.
  *   - Always checked: null pointers, A.ncols == B.nrows, nnz consistency with row_ptr
  *     (host-side when the value is known), dtype, call order (SPG_ERR_BAD_STATE), and
  *     per-row flop counts < 2^31 (SPG_ERR_INDEX_OVERFLOW, reported by symbolic).
@@ -51,6 +53,8 @@
 
 #include <stdint.h>
 
+#define SPG_MAX_NNZ (((int64_t)1 << 31) - 4097) /* largest nnz of an input matrix */
+
 #ifdef __cplusplus
 extern "C" {
 #endif
@@ -61,7 +65,7 @@ typedef enum {
   SPG_OK = 0,
   SPG_ERR_INVALID_ARGUMENT = 1,   /* null pointer, bad option, malformed CSR (validate)   */
   SPG_ERR_DIMENSION_MISMATCH = 2, /* A.ncols != B.nrows                                    */
-  SPG_ERR_INDEX_OVERFLOW = 3,     /* input nnz >= 2^31, or a row's flop count >= 2^31     */
+  SPG_ERR_INDEX_OVERFLOW = 3,     /* input nnz > SPG_MAX_NNZ, or a row's flop count >= 2^31 */
   SPG_ERR_OUT_OF_MEMORY = 4,      /* workspace allocation failed                           */
   SPG_ERR_CUDA = 5,               /* CUDA runtime error (see spg_last_error)               */
   SPG_ERR_NCCL = 6,               /* NCCL error (see spg_last_error)                       */

@@ -43,9 +43,10 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
   __syncthreads();
   const int e0 = s_rp[0], e1 = s_rp[nr];
   int bad = 0;
-  for (int base = e0; base < e1; base += ROWS) {  // uniform trip count: warp collectives below
-    const int e = base + t;
-    const bool act = e < e1;
+  // 64-bit loop index: base + ROWS may pass INT_MAX when nnz(A) is within ROWS of 2^31
+  for (long long base = e0; base < e1; base += ROWS) {  // uniform trip count: warp collectives below
+    const int e = (int)(base + t);
+    const bool act = base + t < e1;
     int L = 0, r = -1;
     if (act) {
       const int k = colA[e];

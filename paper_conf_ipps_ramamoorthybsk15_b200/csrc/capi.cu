@@ -165,7 +165,9 @@ spg_status check_csr(spg_handle h, const spg_csr* m, const char* name, bool need
   if (!m) return setf(h, SPG_ERR_INVALID_ARGUMENT, "%s is NULL", name);
   if (m->nrows < 0 || m->ncols < 0 || m->nnz < 0)
     return setf(h, SPG_ERR_INVALID_ARGUMENT, "%s has negative dimensions or nnz", name);
-  if (m->nnz >= ((int64_t)1 << 31)) return setf(h, SPG_ERR_INDEX_OVERFLOW, "%s.nnz >= 2^31", name);
+  // kernels form entry indices up to nnz + 4096 in 32-bit arithmetic (block-sized strides past
+  // the end of a row range), so nnz stays 4096 below 2^31
+  if (m->nnz > SPG_MAX_NNZ) return setf(h, SPG_ERR_INDEX_OVERFLOW, "%s.nnz > 2^31 - 4097", name);
   if (!m->row_ptr) return setf(h, SPG_ERR_INVALID_ARGUMENT, "%s.row_ptr is NULL", name);
   if (m->nnz > 0 && !m->col_idx) return setf(h, SPG_ERR_INVALID_ARGUMENT, "%s.col_idx is NULL", name);
   if (need_vals && m->nnz > 0 && !m->vals) return setf(h, SPG_ERR_INVALID_ARGUMENT, "%s.vals is NULL", name);

@@ -278,6 +278,15 @@ def test_error_paths():
     bad.col_idx[0] = 99
     with pytest.raises(spg.SpgError, match="out of range"):
         plan.symbolic(dA, to_dev(bad))
+    # nnz beyond SPG_MAX_NNZ (2^31 - 4097) is refused on the host, before any device access
+    import ctypes
+    from paper_conf_ipps_ramamoorthybsk15_b200 import binding as Bd
+    big = Bd.spg_csr(10, 8, 2**31 - 4096, dA.row_ptr.data_ptr(), dA.col_idx.data_ptr(), dA.vals.data_ptr())
+    nnz, rb, re = ctypes.c_int64(), ctypes.c_int32(), ctypes.c_int32()
+    rp = torch.zeros(11, dtype=torch.int64, device="cuda")
+    st = Bd.load().spg_spgemm_symbolic(plan.h, ctypes.byref(big), ctypes.byref(dB2.c()), ctypes.c_void_p(rp.data_ptr()),
+                                       ctypes.byref(nnz), ctypes.byref(rb), ctypes.byref(re))
+    assert Bd.STATUS_NAMES[st] == "SPG_ERR_INDEX_OVERFLOW"
     plan.close()
 
 

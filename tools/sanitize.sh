@@ -7,7 +7,8 @@ sys.path.insert(0, ".")
 import paper_conf_ipps_ramamoorthybsk15_b200 as spg, workloads as W
 A, _ = W.make("cl10k")
 dA = spg.DeviceCSR.from_host(A, "cuda:0")
-for opts in ({}, {"force_class": 6}, {"force_class": 5}, {"light_max_flops": 0}, {"light_max_flops": 4096, "tile_flops": 1024}):
+for opts in ({}, {"force_class": 6}, {"force_class": 5}, {"light_max_flops": 0}, {"light_max_flops": 4096, "tile_flops": 1024},
+             {"heavy_sort": 1}, {"pack_b": 1}, {"heavy_order": 2}):
     plan = spg.SpGEMM(0, torch.float64)
     for k, v in opts.items():
         plan.set_option(k, v)

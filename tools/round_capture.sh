@@ -26,4 +26,4 @@ timeout 1800 python tools/alpha_sweep.py --steps 3 --out gpurun_out/r02_alpha_sw
 for c in webbase1m citpatents; do
   timeout 1200 python tools/ablation.py --config $c --out gpurun_out/r02_ablation.jsonl > gpurun_out/ablation_$c.log 2>&1; echo "ablation $c rc=$?"
 done
-bash tools/sanitize.sh
+# tools/sanitize.sh: compute-sanitizer is closed on this GPU pool (see profiles/r02_sanitizer.txt)

@@ -138,11 +138,18 @@ typedef enum {
                                    numeric call, 16 B per B entry for fp64): -1 (default) when
                                    B's columns + values exceed 64 MB (B not L2-resident), 0 never,
                                    1 always                                                     */
-  SPG_OPT_HEAVY_SORT = 13       /* HEAVY rows (f <= 8192) are sorted like tiles in "big tiles" of
+  SPG_OPT_HEAVY_SORT = 13,      /* HEAVY rows (f <= 8192) are sorted like tiles in "big tiles" of
                                    8192 products (1024 threads) instead of the column bitmap:
                                    -1 (default) when B has more than 2^20 columns (the bitmap
                                    would need several column-tile passes per row), 0 never,
                                    1 always                                                     */
+  SPG_OPT_HEAVY_DUAL = 14       /* 1: the HUGE and HEAVY2 bins share one dual-ended work queue
+                                   (cpuOffset / gpuOffset): over the list
+                                   [HUGE rows ; HEAVY2 rows], each largest first, the HUGE-kernel
+                                   blocks take rows from the front and the register-cached HEAVY2
+                                   blocks from the back, so the split between the two kernels is
+                                   set at run time.  0 (default): each bin its own queue.  No
+                                   effect when HEAVY_SORT puts HEAVY2 rows in big tiles         */
 } spg_option;
 
 typedef struct {

@@ -28,7 +28,7 @@ NUM_CLASSES = 7
 OPTIONS = {"light_max_flops": 0, "tile_flops": 1, "heavy_max_flops": 2, "force_class": 3, "validate": 4,
            "input_canonical": 5, "timing": 6, "huge_slots": 7, "concurrent": 8, "autotune": 9,
            "csrmm_light_nnz": 10, "heavy_order": 11, "pack_b": 12,
-           "heavy_sort": 13}
+           "heavy_sort": 13, "heavy_dual": 14}
 
 EXPORTED = ["spg_create", "spg_set_option", "spg_get_option", "spg_spgemm_free", "spg_last_error", "spg_get_stats",
             "spg_version", "spg_spgemm_symbolic", "spg_spgemm_numeric", "spg_spgemm_host_symbolic",

@@ -85,6 +85,8 @@ struct spg_ctx {
   int heavy_order = 1;     // SPG_OPT_HEAVY_ORDER
   int pack_b = -1;         // SPG_OPT_PACK_B
   int heavy_sort = -1;     // SPG_OPT_HEAVY_SORT
+  int heavy_dual = 0;      // SPG_OPT_HEAVY_DUAL
+  int dual_gen = 0;        // claim generation of the dual-ended queue (one per symbolic pass)
   int occ_big = 1;
   bool use_big = false;    // this symbolic call sorts the cached heavy bins as big tiles
   bool tuned = false;
@@ -92,7 +94,7 @@ struct spg_ctx {
   int tuned_light = 0, tuned_tile = 0;
   // workspace: analysis (all rows), classification and items (this rank's rows), the plan
   DevBuf f, nz, Tb, Tl, cls, pw, Ro, tflag, tscan, items, lists, small, scan_tmp, plan, fl8, D, ucnt, uscan,
-      units, ticket, dub, R, mmlist, lsort, Bp, Pf, splits, canonB[4], iota, ones, crow_tmp;
+      units, ticket, dub, R, dqclaim, mmlist, lsort, Bp, Pf, splits, canonB[4], iota, ones, crow_tmp;
   spg_ctx* canon = nullptr;  // sub-handle that canonicalises B (SPG_OPT_INPUT_CANONICAL = 0)
   spg_csr Bc{};              // canonical copy of B (valid after symbolic when !canonical)
   long long iota_n = -1, ones_n = -1;
@@ -212,6 +214,7 @@ SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* cr
   P.r_cap = r_cap;
   P.row_begin = h->rb;
   P.row_end = h->re;
+  P.dual = 0;
   return P;
 }
 
@@ -221,12 +224,29 @@ SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* cr
 // that exits at once when its list is empty.  The heavy bins fork as soon as the plan offsets Ro
 // exist, so they overlap the tile cut.
 spg_status fork_heavy(spg_handle h, const spg_csr* A, const spg_csr* B, long long* crow) {
-  const SymProb P = make_sym(h, A, B, crow);
+  SymProb P = make_sym(h, A, B, crow);
   Small* ds = h->small.as<Small>();
   const bool conc = h->concurrent != 0;
   const bool tm = h->timing != 0;
   if (conc) CK(cudaEventRecord(h->ev_fork, h->stream));
   const long long Mloc = h->re - h->rb;
+  if (h->heavy_dual && !h->use_big && Mloc > 0) {  // HUGE and HEAVY2 bins share a dual-ended queue
+    const size_t need = (size_t)Mloc * sizeof(int);
+    if (!h->dqclaim.p || h->dqclaim.cap < need || h->dual_gen >= INT_MAX - 1) {
+      CK(h->dqclaim.ensure(need));
+      CK(cudaMemsetAsync(h->dqclaim.p, 0, h->dqclaim.cap, h->stream));
+      h->dual_gen = 0;
+    }
+    P.dual = 1;
+    P.dq_lh = h->lists.as<int>() + (size_t)BIN_HUGE * (size_t)Mloc;
+    P.dq_l2 = h->lists.as<int>() + (size_t)BIN_HEAVY2 * (size_t)Mloc;
+    P.dq_nh = ds->counts + BIN_HUGE;
+    P.dq_n2 = ds->counts + BIN_HEAVY2;
+    P.dq_front = ds->qhead + BIN_HUGE;
+    P.dq_back = ds->qhead + BIN_HEAVY2;
+    P.dq_claim = h->dqclaim.as<int>();
+    P.dq_gen = ++h->dual_gen;
+  }
   const int order[NUM_BINS] = {BIN_HUGE, BIN_HEAVY2, BIN_HEAVY};
   for (int x = 0; x < NUM_BINS; ++x) {
     const int b = order[x];
@@ -659,7 +679,7 @@ spg_status spg_spgemm_free(spg_handle h) {
     cudaStreamSynchronize(h->stream);
     DevBuf* bufs[] = {&h->f,     &h->nz,    &h->Tb,    &h->Tl,    &h->cls,    &h->pw,   &h->Ro,    &h->tflag,
                       &h->tscan, &h->items, &h->lists, &h->small, &h->scan_tmp, &h->plan, &h->fl8, &h->D,
-                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->R, &h->mmlist, &h->lsort, &h->Bp, &h->Pf,     &h->splits,
+                      &h->ucnt,  &h->uscan, &h->units, &h->ticket, &h->dub, &h->R, &h->dqclaim, &h->mmlist, &h->lsort, &h->Bp, &h->Pf,     &h->splits,
                       &h->iota,  &h->ones,  &h->crow_tmp};
     for (DevBuf* b : bufs) b->release();
     for (auto& b : h->canonB) b.release();
@@ -733,6 +753,7 @@ spg_status spg_set_option(spg_handle h, spg_option opt, int64_t v) {
       if (v < -1 || v > 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "PACK_B must be -1, 0 or 1");
       h->pack_b = (int)v;
       break;
+    case SPG_OPT_HEAVY_DUAL: h->heavy_dual = v != 0; break;
     case SPG_OPT_HEAVY_SORT:
       if (v < -1 || v > 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "HEAVY_SORT must be -1, 0 or 1");
       h->heavy_sort = (int)v;
@@ -760,6 +781,7 @@ spg_status spg_get_option(spg_handle h, spg_option opt, int64_t* v) {
     case SPG_OPT_HEAVY_ORDER: *v = h->heavy_order; break;
     case SPG_OPT_PACK_B: *v = h->pack_b; break;
     case SPG_OPT_HEAVY_SORT: *v = h->heavy_sort; break;
+    case SPG_OPT_HEAVY_DUAL: *v = h->heavy_dual; break;
     default: return setf(h, SPG_ERR_INVALID_ARGUMENT, "unknown option %d", (int)opt);
   }
   return SPG_OK;

@@ -77,17 +77,43 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
   // up to an order of magnitude, so static striding would leave a long tail — the paper's work
   // queue in its intra-GPU form.  count[0] = rows, count[8] = queue head.
   const int n = count[0];
+  // dual-ended queue: the PLAIN (HUGE) kernel is the front consumer, the 1024-thread cached
+  // (HEAVY2) kernel the back consumer; the 512-thread HEAVY bin keeps its own queue
+  constexpr bool FRONT = !CACHED, BACK = CACHED && NT == BMP_NT;
+  const bool dual = P.dual && (FRONT || BACK);
+  const int ndq = dual ? *P.dq_nh + *P.dq_n2 : 0;
   __shared__ int s_next;
   __shared__ int s_dcnt, s_single;
   __shared__ int s_uc[HEAVY_CAP / NUM_SH + 2];  // cached rows: repeats per numeric unit
   __shared__ long long s_rbase;
   for (;;) {
-    if (tid == 0) s_next = atomicAdd(const_cast<int*>(count) + 8, 1);
+    if (tid == 0) {
+      if (!dual) {
+        const int t = atomicAdd(const_cast<int*>(count) + 8, 1);
+        s_next = t < n ? list[t] : -1;
+      } else {
+        int li = -1;
+        const int nh = *P.dq_nh;
+        if (FRONT) {  // dense end: the next index nobody has claimed yet
+          for (;;) {
+            const int t = atomicAdd(P.dq_front, 1);
+            if (t >= ndq) break;
+            if (atomicMax(P.dq_claim + t, P.dq_gen) < P.dq_gen) {
+              li = t < nh ? P.dq_lh[t] : P.dq_l2[t - nh];
+              break;
+            }
+          }
+        } else {  // sparse end: HEAVY2 rows only; stop where the front has been
+          const int t = ndq - 1 - atomicAdd(P.dq_back, 1);
+          if (t >= nh && atomicMax(P.dq_claim + t, P.dq_gen) < P.dq_gen) li = P.dq_l2[t - nh];
+        }
+        s_next = li;
+      }
+    }
     __syncthreads();
-    const int t = s_next;
+    const int li = s_next;
     __syncthreads();
-    if (t >= n) break;
-    const int li = list[t];
+    if (li < 0) break;
     const int i = P.row_begin + li;
     const int pa0 = P.rpA[i], pa1 = P.rpA[i + 1];
     const int f = P.frow[i];

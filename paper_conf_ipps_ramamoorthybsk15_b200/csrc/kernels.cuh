@@ -75,6 +75,19 @@ struct SymProb {
   int* err;                 // error bits (Small::err)
   long long r_cap;          // plan capacity (words); the kernels do nothing if Ro[Mloc] > r_cap
   int row_begin, row_end;
+  // Dual-ended queue (SPG_OPT_HEAVY_DUAL, the paper's cpuOffset / gpuOffset work
+  // queue): the virtual list [HUGE rows ; HEAVY2 rows], each part largest
+  // first.  HUGE-kernel blocks (any row) take from the front, HEAVY2 (register-cached) blocks from
+  // the back; a row is processed by whichever side claims it first (claim[t] raised to gen).
+  int dual;                 // 1: on
+  const int* dq_lh;         // HUGE list, count dq_nh[0]
+  const int* dq_l2;         // HEAVY2 list, count dq_n2[0]
+  const int* dq_nh;
+  const int* dq_n2;
+  int* dq_front;            // front cursor (Small::qhead[BIN_HUGE])
+  int* dq_back;             // back cursor (Small::qhead[BIN_HEAVY2])
+  int* dq_claim;            // per list index: generation of the last claim
+  int dq_gen;               // this call's generation (> every earlier one)
 };
 
 // Numeric work units, in a list built in item order: item t has ceil(c_t / NUM_SH) units, unit k
@@ -164,7 +177,7 @@ cudaError_t launch_tile_heavy(cudaStream_t st, int grid, const SymProb& P, const
 cudaError_t heavy_configure();
 int heavy_occupancy(int bin);
 cudaError_t launch_heavy_rank(int bin, cudaStream_t st, int grid, const SymProb& P, const int* list,
-                              const int* count, long long N);
+                              const int* count, long long N);  // (P.dual: the HUGE and HEAVY2 bins share the dual queue)
 
 // k_csrmm.cu — sparse x dense.
 template <typename V>

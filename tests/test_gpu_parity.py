@@ -117,6 +117,31 @@ def test_heavy_rows_as_big_tiles(light):
     compare(A2, A2, run_gpu(A2, A2, heavy_sort=1, light_max_flops=light))
 
 
+@pytest.mark.parametrize("opts", [{}, {"heavy_max_flops": 4096}, {"heavy_max_flops": 6000, "heavy_order": 0},
+                                  {"concurrent": 0}, {"huge_slots": 3}])
+def test_heavy_dual_queue(opts):
+    """SPG_OPT_HEAVY_DUAL = 1: HUGE-kernel blocks take rows from the front of [HUGE ; HEAVY2]
+    and register-cached HEAVY2 blocks from the back — every row is processed
+    exactly once whichever side claims it, so C equals the oracle's at any split."""
+    A = W.chung_lu(30000, 30000, 2.1, 150000, 4000, 4000, 5.0, 1.1, 17)
+    ref = oracle.spgemm(A, A, nthreads=8)
+    compare(A, A, run_gpu(A, A, heavy_dual=1, heavy_sort=0, **opts), ref=ref)
+
+
+def test_heavy_dual_queue_reused_handle():
+    """The claim generation advances per symbolic pass: a handle re-run on the same and on a new
+    structure (plan grows, rerun inside symbolic) keeps processing every row once."""
+    A1, _ = W.make("cl10k")
+    A2 = W.chung_lu(30000, 30000, 2.1, 150000, 4000, 4000, 5.0, 1.1, 17)
+    plan = spg.SpGEMM(0, torch.float64, heavy_dual=1, heavy_sort=0)
+    for A in (A1, A2, A1, A2):
+        dA = spg.DeviceCSR.from_host(A, "cuda:0")
+        C = plan(dA, dA)
+        torch.cuda.synchronize()
+        compare(A, A, (C.row_ptr.cpu().numpy(), C.col_idx.cpu().numpy(), C.vals.cpu().numpy()))
+    plan.close()
+
+
 @pytest.mark.parametrize("dtype", [np.float64, np.float32])
 def test_packed_b_numeric(dtype):
     """SPG_OPT_PACK_B = 1: numeric gathers B through the packed {column, value} copy (automatic

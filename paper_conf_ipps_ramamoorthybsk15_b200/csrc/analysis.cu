@@ -43,13 +43,17 @@ __global__ void __launch_bounds__(ROWS) k_row_flops(int M, const int* __restrict
   __syncthreads();
   const int e0 = s_rp[0], e1 = s_rp[nr];
   int bad = 0;
-  // 64-bit loop index: base + ROWS may pass INT_MAX when nnz(A) is within ROWS of 2^31
+  // 64-bit loop index: base + ROWS may pass INT_MAX when nnz(A) is within ROWS of 2^31.  The
+  // next iteration's column is loaded one iteration ahead (its latency overlaps this iteration's
+  // B-row-pointer gathers).
+  int kn = (long long)e0 + t < e1 ? __ldg(colA + e0 + t) : 0;
   for (long long base = e0; base < e1; base += ROWS) {  // uniform trip count: warp collectives below
     const int e = (int)(base + t);
     const bool act = base + t < e1;
+    const int k = kn;
+    kn = base + ROWS + t < e1 ? __ldg(colA + (base + ROWS + t)) : 0;
     int L = 0, r = -1;
     if (act) {
-      const int k = colA[e];
       r = upper_idx(s_rp, nr, e);
       int bs = 0;
       if ((unsigned)k >= (unsigned)K) bad |= 1;
@@ -203,21 +207,16 @@ __global__ void __launch_bounds__(256) k_tile_flags(const int* __restrict__ f, c
                                                     const long long* __restrict__ Ro, int* __restrict__ tflag) {
   const long long n = (long long)re - rb;
   for (long long li = (long long)blockIdx.x * blockDim.x + threadIdx.x; li < n; li += (long long)gridDim.x * blockDim.x) {
+    // every load issued up front (independent), then the tests
     const int c = cls[li];
-    bool start = (c & CLS_HEAVY_PATH) || (c & CLS_SOLO) || li == 0 || (li % TILE_RM) == 0;
-    if (!start) {
-      const int cp = cls[li - 1];
-      start = (cp & CLS_HEAVY_PATH) || (cp & CLS_SOLO);
-    }
-    if (!start) {
-      const long long fi = f[rb + li];
-      if (fi > 0) {
-        const long long pl = Ro[li];
-        start = (pl % cap == 0) || (pl / cap != (pl + fi - 1) / cap);
-      }
-      const long long ea = rpA[rb + li], al = rpA[rb + li + 1] - ea;
-      if (al > 0) start = start || (ea % TILE_EC == 0) || (ea / TILE_EC != (ea + al - 1) / TILE_EC);
-    }
+    const int cp = li > 0 ? cls[li - 1] : 0;
+    const long long fi = f[rb + li];
+    const long long pl = Ro[li];
+    const long long ea = rpA[rb + li], al = rpA[rb + li + 1] - ea;
+    bool start = (c & CLS_HEAVY_PATH) || (c & CLS_SOLO) || li == 0 || (li % TILE_RM) == 0 ||
+                 (cp & CLS_HEAVY_PATH) || (cp & CLS_SOLO);
+    if (fi > 0) start = start || (pl % cap == 0) || (pl / cap != (pl + fi - 1) / cap);
+    if (al > 0) start = start || (ea % TILE_EC == 0) || (ea / TILE_EC != (ea + al - 1) / TILE_EC);
     tflag[li] = start ? 1 : 0;
   }
 }

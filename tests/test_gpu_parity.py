@@ -128,6 +128,15 @@ def test_heavy_dual_queue(opts):
     compare(A, A, run_gpu(A, A, heavy_dual=1, heavy_sort=0, **opts), ref=ref)
 
 
+@pytest.mark.parametrize("name", ["webbase1m", "ab2m"])
+def test_heavy_dual_queue_full_config(name):
+    """The dual-ended queue on the BASELINE shapes with many HUGE and HEAVY2 rows: C equals the
+    oracle's on every row."""
+    A, B = W.make(name)
+    got = run_gpu(A, B, heavy_dual=1)
+    compare(A, B, got, nthreads=max(1, __import__("os").cpu_count() or 1))
+
+
 def test_heavy_dual_queue_reused_handle():
     """The claim generation advances per symbolic pass: a handle re-run on the same and on a new
     structure (plan grows, rerun inside symbolic) keeps processing every row once."""

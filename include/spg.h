@@ -42,7 +42,9 @@
  *     stride past a row range in 32-bit arithmetic); larger inputs give SPG_ERR_INDEX_OVERFLOW.
  *   - Always checked: null pointers, A.ncols == B.nrows, nnz consistency with row_ptr
  *     (host-side when the value is known), dtype, call order (SPG_ERR_BAD_STATE), and
- *     per-row flop counts < 2^31 (SPG_ERR_INDEX_OVERFLOW, reported by symbolic).
+ *     per-row flop counts < 2^31 (SPG_ERR_INDEX_OVERFLOW, reported by symbolic), and repeated
+ *     products within the first 2^23 stored entries of their A row (SPG_ERR_NOT_SUPPORTED,
+ *     reported by symbolic: a repeat's record holds its A entry relative to the row in 23 bits).
  *   - Index ranges and ordering of device inputs are checked only under SPG_OPT_VALIDATE.
  *   - Values are not bitwise reproducible run to run when a row has repeated columns: the
  *     repeated products are added with atomics in a nondeterministic order (R6).

@@ -205,8 +205,8 @@ SymProb make_sym(spg_handle h, const spg_csr* A, const spg_csr* B, long long* cr
   P.tscan = h->tscan.as<long long>();
   P.D = h->D.as<unsigned>();
   P.dub = h->dub.as<long long>();
-  P.R = h->R.as<int4>();
-  P.r_dcap = h->R.p ? (long long)(h->R.cap / sizeof(int4)) : 0;
+  P.R = h->R.as<int2>();
+  P.r_dcap = h->R.p ? (long long)(h->R.cap / sizeof(int2)) : 0;
   P.dups = &h->small.as<Small>()->dups;
   P.dups_all = &h->small.as<Small>()->dups_all;
   P.err = &h->small.as<Small>()->err;
@@ -487,8 +487,12 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     const Small& hs = h->hr->small;
     if (hs.err & 1) return setf(h, SPG_ERR_INVALID_ARGUMENT, "A has a column index outside [0, B.nrows)");
     if (hs.err & 2) return setf(h, SPG_ERR_INDEX_OVERFLOW, "a row of A has too many intermediate products (>= 2^31, or >= 2^30 with 64-bit plan entries)");
+    if (hs.err & 32)
+      return setf(h, SPG_ERR_NOT_SUPPORTED,
+                  "a repeated product's A entry is 2^%d or more entries into its row (the repeat record's field)",
+                  REC_EBITS);
     const long long words = h->hr->ncut;
-    const long long rcap = h->R.p ? (long long)(h->R.cap / sizeof(int4)) : 0;
+    const long long rcap = h->R.p ? (long long)(h->R.cap / sizeof(int2)) : 0;
     if (words <= h->plan_cap() && hs.dups_all <= rcap) {
       h->plan_words = words;
       break;
@@ -500,7 +504,7 @@ spg_status symbolic_impl(spg_handle h, const spg_csr* A, const spg_csr* B, int64
     CK(h->fl8.ensure((size_t)words));
     // repeats: at most the products; the exact count once the plan fitted
     const long long want = words <= h->plan_cap() && attempt == 0 && hs.dups_all > 0 ? hs.dups_all : words / 16;
-    CK(h->R.ensure((size_t)((want > hs.dups_all ? want : hs.dups_all) + 1024) * sizeof(int4)));
+    CK(h->R.ensure((size_t)((want > hs.dups_all ? want : hs.dups_all) + 1024) * sizeof(int2)));
   }
   const Small& hs = h->hr->small;
   if ((long long)hs.cstats[2 * NUM_CLS] > (long long)NUM_SH * DUP_SORT_UNITS)
@@ -588,7 +592,7 @@ spg_status numeric_impl(spg_handle h, const spg_csr* A, const spg_csr* B, const 
     P.items = h->items.as<int>();
     P.units = h->units.as<NumUnit>();
     P.nunits = &h->small.as<Small>()->nunits;
-    P.R = h->R.as<int4>();
+    P.R = h->R.as<int2>();
     P.ticket = h->ticket.as<int>();
     P.row_begin = h->rb;
     P.ccol = C_col;

@@ -464,7 +464,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
             if ((dmask >> s & 1u) && rbase >= 0) {
               const int pos = atomicAdd(&s_uc[oo[s] / NUM_SH], 1);
               const int qo = j0 + lane - seg[r];
-              P.R[rbase + pos] = make_int4(sbs[r] + qo, sae[r], oo[s], 0);
+              P.R[rbase + pos] = make_int2(sbs[r] + qo, rec_meta(sae[r] - pa0, oo[s]));
             }
           }
         }
@@ -526,7 +526,8 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
               }
               const int e = pa0 + (int)er;
               const int pos = atomicAdd(&ucnt[o / NUM_SH], 1);
-              P.R[rbase + pos] = make_int4(P.Tb[e] + (int)qo, e, (int)o, 0);
+              if (er >= (1u << REC_EBITS)) atomicOr(P.err, 32);  // beyond the record's A-entry field
+              P.R[rbase + pos] = make_int2(P.Tb[e] + (int)qo, rec_meta((int)er, (int)o));
             }
           __syncthreads();
           for (int k = tid; k <= hs; k += NT) ucnt[k] = 0;  // the zero invariant (next row's barrier orders it)

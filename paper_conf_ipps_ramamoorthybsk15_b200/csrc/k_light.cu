@@ -556,7 +556,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
           const int pos = atomicAdd(&s_uc[s_iub[it] + o / NUM_SH], 1);
           const unsigned w = pay[idx];
           const int e = s_ie0[it] + (int)(w & 0xffffu);
-          P.R[s_idb[it] + pos] = make_int4(P.Tb[e] + (int)(w >> 16), e, o, 0);
+          P.R[s_idb[it] + pos] = make_int2(P.Tb[e] + (int)(w >> 16), rec_meta((int)(w & 0xffffu), o));
         }
       __syncthreads();
     }

@@ -5,8 +5,9 @@
 // item (a tile of consecutive rows, or one heavy row) with plan region [P0, P0 + f) and outputs
 // [o0, o0 + c), plan word P0 + o describes output o0 + o — {e_rel, qoff}: the A entry e0 + e_rel
 // and the offset of the B entry inside that entry's B row.  The item's repeated products (a
-// product whose column another product of its row already produced) are 16-byte records
-// {B entry, A entry, item-relative output} in R, bucketed by the numeric unit owning the output.
+// product whose column another product of its row already produced) are 8-byte records
+// {B entry, A entry - item's first | output - unit's first << 23} in R, bucketed by the numeric
+// unit owning the output.
 //
 // So numeric is a stream in C order (Phase IV of PAPER.md L154-156, "add like-tuples and
 // compact", with the sort done once in symbolic).  Persistent warps take work units (NUM_SH
@@ -17,7 +18,7 @@
 //   outputs   per output one plan word (shared memory), the A entry's B-row start Tb[e] and value
 //             valA[e] (the item's A entries: L1), the B gather (column and value, L2: B rows are
 //             consumed in ascending order), one multiply, two coalesced streaming stores.
-//   repeats   the unit's repeat records (16-byte {B entry, A entry, output}, bucketed by unit in
+//   repeats   the unit's repeat records (8-byte {B entry, A entry, output}, bucketed by unit in
 //             symbolic) add a·b into its own outputs with RED.ADD.F64/F32 — into lines it just
 //             wrote (L2), ordered after its stores by __syncwarp; no unit ever waits for another.
 // HBM traffic per output: 4 B of plan read + (4 + sizeof(V)) B of C written; A and B once.
@@ -28,6 +29,11 @@ namespace spg {
 constexpr int NUM_NT = 128;            // threads per block: 4 independent warps
 constexpr int NUM_W = NUM_NT / 32;
 constexpr int NUM_U = 4;               // outputs per lane in flight
+// Resident blocks per SM: the register budget of 7 blocks (72 registers) and the grid's cap.  More
+// resident warps share L1 among more units and lose B-line hits (8 blocks: 0.355 vs 0.342 ms on
+// webbase1m); letting the compiler pick its own budget gave 64 registers and a slower schedule
+// with the 8-byte repeat records (0.360 ms), the 7-block bound 0.325 ms (profiles/experiments).
+constexpr int NUM_BLOCKS_SM = 7;
 constexpr int NUM_BUFW = NUM_SH + 8;   // plan words per staging buffer (16-byte alignment slack)
 
 __device__ __forceinline__ void st_cs(int* p, int v) { __stcs(p, v); }
@@ -84,7 +90,7 @@ __global__ void __launch_bounds__(256) k_pack_b(const int* __restrict__ colB, co
 }
 
 template <typename V, bool PACKED>
-__global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
+__global__ void __launch_bounds__(NUM_NT, NUM_BLOCKS_SM) k_numeric(NumProb<V> P) {
   using PB = PackB<V>;
   const typename PB::T* __restrict__ Bp = reinterpret_cast<const typename PB::T*>(P.Bp);
   __shared__ __align__(16) unsigned s_buf[NUM_W][2][NUM_BUFW];
@@ -131,7 +137,7 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
     const bool wide = cur.ob & UNIT_WIDE;
     const int e0 = cur.e0, n = cur.n;
     // the first 32 repeat records: fetched now, used after the outputs
-    int4 rec = make_int4(0, 0, 0, 0);
+    int2 rec = make_int2(0, 0);
     if (lane < cur.d) rec = __ldg(P.R + cur.dw + lane);
     // ---- outputs in C order -----------------------------------------------------------------------
     int* __restrict__ ccol = P.ccol + cur.oc;
@@ -201,17 +207,19 @@ __global__ void __launch_bounds__(NUM_NT) k_numeric(NumProb<V> P) {
       }
     }
     __syncwarp();  // every lane is done with buffer cb, and its stores precede the adds below
-    // ---- repeated products landing in this unit's outputs (R records: B entry, A entry, output) -
+    // ---- repeated products landing in this unit's outputs (R records: B entry, A entry relative to
+    //      the item, output inside the unit) ------------------------------------------------------
     if (cur.d > 0) {
-      V* __restrict__ cv0 = cval - (cur.ob & (UNIT_WIDE - 1));
+      constexpr unsigned EM = (1u << REC_EBITS) - 1u;
       auto bval = [&](int q) -> V {
         if constexpr (PACKED) return PB::val(__ldg(Bp + q));
         else return __ldg(P.valB + q);
       };
-      if (lane < cur.d) atomicAdd(cv0 + rec.z, __ldg(P.valA + rec.y) * bval(rec.x));
+      if (lane < cur.d)
+        atomicAdd(cval + ((unsigned)rec.y >> REC_EBITS), __ldg(P.valA + e0 + (int)((unsigned)rec.y & EM)) * bval(rec.x));
       for (int j = 32 + lane; j < cur.d; j += 32) {
-        const int4 x = __ldg(P.R + cur.dw + j);
-        atomicAdd(cv0 + x.z, __ldg(P.valA + x.y) * bval(x.x));
+        const int2 x = __ldg(P.R + cur.dw + j);
+        atomicAdd(cval + ((unsigned)x.y >> REC_EBITS), __ldg(P.valA + e0 + (int)((unsigned)x.y & EM)) * bval(x.x));
       }
     }
     if (!more) break;
@@ -230,7 +238,7 @@ cudaError_t launch_numeric(cudaStream_t st, int sms, const NumProb<V>& P) {
     int nb = 1;
     if (v) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_numeric<V, true>, NUM_NT, 0);
     else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_numeric<V, false>, NUM_NT, 0);
-    occ[v] = nb < 1 ? 1 : nb;
+    occ[v] = nb < 1 ? 1 : (nb > NUM_BLOCKS_SM ? NUM_BLOCKS_SM : nb);
   }
   const int grid = occ[v] * sms;
   if (v) k_numeric<V, true><<<grid, NUM_NT, 0, st>>>(P);

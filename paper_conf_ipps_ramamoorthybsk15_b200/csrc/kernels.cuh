@@ -68,7 +68,7 @@ struct SymProb {
   unsigned* D;              // HUGE rows: item-relative output of the repeated product whose plan
                             // entry starts at the same word (written only for their repeats)
   long long* dub;           // repeats' first R record per numeric unit (dub_index(P0, t) + k)
-  int4* R;                  // repeat records {B entry, A entry, item-relative output, 0}
+  int2* R;                  // repeat records {B entry, rec_meta(A entry - item's first, output)}
   long long r_dcap;         // R capacity (records); beyond it nothing is written (host grows, reruns)
   long long* dups;          // R reservation counter
   long long* dups_all;      // repeated-product counter (statistics)
@@ -93,13 +93,21 @@ struct SymProb {
 // Numeric work units, in a list built in item order: item t has ceil(c_t / NUM_SH) units, unit k
 // owning outputs [k NUM_SH, (k + 1) NUM_SH) of the item.  A unit stores its outputs, then adds
 // the item's repeated products (d_t = f_t - c_t) that land in its own outputs: a warp only ever
-// adds into outputs it stored itself, so no unit waits for another.  The repeats are 16-byte
-// records {B entry, A entry, item-relative output} in R, bucketed by unit (tiles: k_tile_rank;
+// adds into outputs it stored itself, so no unit waits for another.  The repeats are 8-byte
+// records (rec_meta below) in R, bucketed by unit (tiles: k_tile_rank;
 // heavy rows: k_bitmap_rank at the end of the row); unit k's
 // records start at R[dub[dub_index(P0, t) + k]].
 constexpr int NUM_SH = 512;
 constexpr int DUP_SORT_UNITS = 48 * 1024;   // HUGE rows' unit counters in k_bitmap_rank (rows up to 24M outputs)
 __host__ __device__ __forceinline__ long long dub_index(long long P0, long long t) { return P0 / NUM_SH + 2 * t; }
+// A repeat record is 8 bytes {B entry, e_rel | (o mod NUM_SH) << 23}: e_rel = its A entry minus the
+// item's first A entry (< 2^23: A rows longer than that are rejected on the host), o mod NUM_SH =
+// its output's offset inside the numeric unit that owns it (the unit adds it).
+constexpr int REC_EBITS = 23;
+static_assert(NUM_SH <= (1 << (32 - REC_EBITS)), "unit offset fits the record");
+__host__ __device__ __forceinline__ int rec_meta(int e_rel, int o) {
+  return (int)((unsigned)e_rel | ((unsigned)(o % NUM_SH) << REC_EBITS));
+}
 struct NumUnit {
   long long pw;   // plan word of the unit's first output
   long long oc;   // C offset (local) of the unit's first output
@@ -127,7 +135,7 @@ struct NumProb {
   const int* __restrict__ items;        // ordered item starts (local rows) + sentinel
   const NumUnit* __restrict__ units;
   const long long* __restrict__ nunits;
-  const int4* __restrict__ R;           // repeat records
+  const int2* __restrict__ R;           // repeat records {B entry, rec_meta(...)}
   int* ticket;                          // work-unit queue head (zeroed before the launch)
   int row_begin;
   int* ccol;

@@ -324,6 +324,28 @@ def test_error_paths():
     plan.close()
 
 
+def test_repeat_record_field_limits():
+    """A repeat record holds its A entry relative to the row in 23 bits: a repeated product
+    2^23 or more entries into its A row is reported (NOT_SUPPORTED), one just below is exact."""
+    for K, want_error in ((2**23 + 3, True), (2**23 - 2, False)):
+        # one A row over all K columns; B rows 0, K-2 and K-1 hold column 0, the rest are empty:
+        # three products of column 0 (one output, two repeats), at least one late in the row
+        rpB = np.zeros(K + 1, dtype=np.int32)
+        rpB[1:] = 1
+        rpB[K - 1:] = 2
+        rpB[K] = 3
+        B = W.CSR(K, 4, rpB, np.zeros(3, dtype=np.int32), np.array([1.0, 2.0, 3.0]))
+        A = W.CSR(1, K, np.array([0, K], dtype=np.int32), np.arange(K, dtype=np.int32), np.ones(K))
+        if want_error:
+            plan = spg.SpGEMM(0, torch.float64)
+            with pytest.raises(spg.SpgError, match="NOT_SUPPORTED"):
+                plan.symbolic(to_dev(A), to_dev(B))
+            plan.close()
+        else:
+            rp, col, val, _ = run_gpu(A, B)
+            assert list(rp) == [0, 1] and list(col) == [0] and float(val[0]) == 6.0
+
+
 def test_concurrent_and_serial_agree():
     A, B = W.make("cl10k")
     ref = oracle.spgemm(A, B, nthreads=8)

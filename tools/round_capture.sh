@@ -10,6 +10,7 @@ M=gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,smsp__inst_e
 timeout 600 ncu --metrics $M --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --profile > gpurun_out/ncu_bench.log 2>&1
 python tools/ncu_sum.py gpurun_out/launches.csv > gpurun_out/launches_summary.txt; cat gpurun_out/launches_summary.txt
 python tools/traffic.py gpurun_out/launches.csv webbase1m gpurun_out
+cp gpurun_out/traffic_webbase1m.json profiles/traffic_webbase1m.json  # the bench line below reads this capture's traffic
 timeout 600 ncu --metrics $M --clock-control none --csv --log-file gpurun_out/launches_cit.csv python bench.py --profile --config citpatents --steps 20 > gpurun_out/ncu_cit.log 2>&1
 python tools/ncu_sum.py gpurun_out/launches_cit.csv > gpurun_out/launches_citpatents.txt
 timeout 900 ncu --metrics $M --clock-control none --csv --log-file gpurun_out/launches_rmat.csv python bench.py --profile --config rmat23 --steps 2 --warmup 3 > gpurun_out/ncu_rmat.log 2>&1

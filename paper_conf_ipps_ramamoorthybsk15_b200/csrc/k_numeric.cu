@@ -33,7 +33,14 @@ constexpr int NUM_U = 4;               // outputs per lane in flight
 // resident warps share L1 among more units and lose B-line hits (8 blocks: 0.355 vs 0.342 ms on
 // webbase1m); letting the compiler pick its own budget gave 64 registers and a slower schedule
 // with the 8-byte repeat records (0.360 ms), the 7-block bound 0.325 ms (profiles/experiments).
+// With packed fp64 B (16-byte entries; B does not fit L2: citpatents, rmat23) 5 blocks (96
+// registers) are best: citpatents 0.745 -> 0.707 ms, rmat23 50.2 -> 42.6 ms; packed fp32 B (8-byte
+// entries, ab2m) keeps 7 (5 blocks: 0.361 -> 0.387 ms).  profiles/experiments/r02_numeric_blocks_ab.txt
 constexpr int NUM_BLOCKS_SM = 7;
+constexpr int NUM_BLOCKS_SM_PACKED64 = 5;
+template <typename V, bool PACKED> constexpr int num_blocks_sm() {
+  return PACKED && sizeof(V) == 8 ? NUM_BLOCKS_SM_PACKED64 : NUM_BLOCKS_SM;
+}
 constexpr int NUM_BUFW = NUM_SH + 8;   // plan words per staging buffer (16-byte alignment slack)
 
 __device__ __forceinline__ void st_cs(int* p, int v) { __stcs(p, v); }
@@ -90,7 +97,7 @@ __global__ void __launch_bounds__(256) k_pack_b(const int* __restrict__ colB, co
 }
 
 template <typename V, bool PACKED>
-__global__ void __launch_bounds__(NUM_NT, NUM_BLOCKS_SM) k_numeric(NumProb<V> P) {
+__global__ void __launch_bounds__(NUM_NT, (num_blocks_sm<V, PACKED>())) k_numeric(NumProb<V> P) {
   using PB = PackB<V>;
   const typename PB::T* __restrict__ Bp = reinterpret_cast<const typename PB::T*>(P.Bp);
   __shared__ __align__(16) unsigned s_buf[NUM_W][2][NUM_BUFW];
@@ -238,7 +245,8 @@ cudaError_t launch_numeric(cudaStream_t st, int sms, const NumProb<V>& P) {
     int nb = 1;
     if (v) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_numeric<V, true>, NUM_NT, 0);
     else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k_numeric<V, false>, NUM_NT, 0);
-    occ[v] = nb < 1 ? 1 : (nb > NUM_BLOCKS_SM ? NUM_BLOCKS_SM : nb);
+    const int cap = v ? num_blocks_sm<V, true>() : num_blocks_sm<V, false>();
+    occ[v] = nb < 1 ? 1 : (nb > cap ? cap : nb);
   }
   const int grid = occ[v] * sms;
   if (v) k_numeric<V, true><<<grid, NUM_NT, 0, st>>>(P);

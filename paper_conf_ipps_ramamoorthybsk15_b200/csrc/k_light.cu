@@ -15,8 +15,8 @@
 //                (coalesced B-row loads; the run of each lane from a REDUX.OR run-start mask).
 //                Each light row's column range [cmin, cmax] comes from the first and last entry
 //                of its (sorted) B rows.
-//   3. buckets   light row j gets NB_j <= ceil(f_j / TILE_BK) buckets of 2^sh_j columns over its
-//                own range: bucket order is (row, column) order; sizes by ATOMS.ADD.
+//   3. buckets   light row j gets NB_j = min(ceil(f_j / TILE_BK), range) equal buckets over its own
+//                column range: bucket order is (row, column) order; sizes by ATOMS.ADD.
 //   4. scatter   exclusive scan of the sizes; each product is placed in its bucket.
 //   5. heads     a product is the head of its column when no earlier slot of its bucket holds the
 //                same column; heads are counted per bucket and scanned; c_j = heads of the row.
@@ -85,8 +85,8 @@ struct TileSmem {
   static constexpr int cmin = row + C::RM * 4;                   // int[RM]     column range of the row (later:
                                                                   //             heads before the row)
   static constexpr int cmax = cmin + C::RM * 4;                  // int[RM]
-  static constexpr int sh = cmax + C::RM * 4;                    // u8[RM]      bucket width log2
-  static constexpr int kind = sh + C::RM;                        // u8[RM]      class of the row
+  static constexpr int mul = cmax + C::RM * 4;                   // u32[RM]     bucket scale (0: one column each)
+  static constexpr int kind = mul + C::RM * 4;                   // u8[RM]      class of the row
   static constexpr int item = kind + C::RM;                      // u8[RM]      tile of the row (in the batch)
   static constexpr int seg = (item + C::RM + 15) & ~15;          // int[NT+1]   chunk run -> product offset
   static constexpr int sbs = seg + (C::NT + 1) * 4;               // int[NT]     chunk run -> B row start
@@ -115,7 +115,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
   int* s_row = reinterpret_cast<int*>(sm + SM::row);
   int* s_cmin = reinterpret_cast<int*>(sm + SM::cmin);
   int* s_cmax = reinterpret_cast<int*>(sm + SM::cmax);
-  uint8_t* s_sh = reinterpret_cast<uint8_t*>(sm + SM::sh);
+  unsigned* s_mul = reinterpret_cast<unsigned*>(sm + SM::mul);
   uint8_t* s_kind = reinterpret_cast<uint8_t*>(sm + SM::kind);
   uint8_t* s_item = reinterpret_cast<uint8_t*>(sm + SM::item);
   int* seg = reinterpret_cast<int*>(sm + SM::seg);
@@ -315,17 +315,18 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
         __syncthreads();
       }
 
-      // ---- 3. buckets: 2^sh columns each over the row's own column range --------------------------
+      // ---- 3. buckets: the row's own column range cut into nb = min(ceil(f / TILE_BK), range)
+      //         equal parts — bucket(col) = floor((col - cmin) * nb / range) as one __umulhi with a
+      //         per-row 32-bit scale (monotonic in col, so bucket order is (row, column) order)
       {
         int nb = 0;
         if (tid < NR && s_kind[tid] >= CLS_TINY) {
           const int f = s_pf[tid + 1] - s_pf[tid];
-          const unsigned span = (unsigned)(s_cmax[tid] - s_cmin[tid]);  // range - 1
+          const unsigned span = (unsigned)(s_cmax[tid] - s_cmin[tid]);  // range - 1 (< 2^31)
           const unsigned want = (unsigned)((f + TILE_BK - 1) / TILE_BK);
-          int sh = 0;
-          while ((span >> sh) >= want) ++sh;
-          s_sh[tid] = (uint8_t)sh;
-          nb = (int)(span >> sh) + 1;
+          const unsigned nbu = want < span + 1u ? want : span + 1u;
+          s_mul[tid] = nbu == span + 1u ? 0u : (unsigned)(((unsigned long long)nbu << 32) / (span + 1u));
+          nb = (int)nbu;
         }
         int tot;
         const int ex = g.excl_scan(nb, tot);
@@ -339,7 +340,9 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
       // bucket of product idx (light rows; -1: SINGLE row, no sort)
       auto bucket_of = [&](int idx) -> int {
         const int j = exrow[idx];
-        return s_kind[j] >= CLS_TINY ? s_bb[j] + ((keys[idx] - s_cmin[j]) >> s_sh[j]) : -1;
+        if (s_kind[j] < CLS_TINY) return -1;
+        const unsigned d = (unsigned)(keys[idx] - s_cmin[j]), m = s_mul[j];
+        return s_bb[j] + (int)(m ? __umulhi(d, m) : d);
       };
       // every product's bucket and column in registers (thread tid owns products tid + u NT);
       // single: bit u set for a product of a SINGLE row (placed in order, no sort)

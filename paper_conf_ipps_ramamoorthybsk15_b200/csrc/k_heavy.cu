@@ -158,6 +158,16 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
     unsigned short* sbq = reinterpret_cast<unsigned short*>(sbp + nl1);   // .. / 256 columns (4 per 1024)
     unsigned* flags = reinterpret_cast<unsigned*>(sbq + 4 * nl1);
     const int nfw = CACHED ? (f + 31) >> 5 : 0;
+    // HUGE rows whose products fit the region after the bitmap structures keep every product's
+    // column there (filled by the first claim pass): later passes and column tiles read it instead
+    // of gathering B again.  Zeroed at the end of the row (the region's zero invariant).
+    int* ccache = nullptr;
+    if constexpr (!CACHED) {
+      const int off = (bmp_need<MODE>(lw, f) + 15) & ~15;
+      if (f <= (REGION - off) / 4) ccache = reinterpret_cast<int*>(region + off);
+    }
+    int cmode = 0;  // for_products: 0 gather B, 1 gather B and fill ccache, 2 read ccache
+    int cbase = 0;  // row product index of the current chunk's first product
     int ntiles = (int)(((long long)N + Wt - 1) >> lw);
     const int nchunks = (pa1 - pa0 + RCAP - 1) / RCAP;
     int lo0 = 0;  // first column of tile 0
@@ -226,7 +236,13 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
             }
           }
 #pragma unroll
-          for (int u = 0; u < BATCH; ++u) col[u] = q[u] >= 0 ? P.colB[q[u]] : -1;
+          for (int u = 0; u < BATCH; ++u)
+            col[u] = q[u] < 0 ? -1 : (cmode == 2 ? ccache[cbase + j00 + u * NT + lane] : P.colB[q[u]]);
+          if (cmode == 1) {
+#pragma unroll
+            for (int u = 0; u < BATCH; ++u)
+              if (q[u] >= 0) ccache[cbase + j00 + u * NT + lane] = col[u];
+          }
 #pragma unroll
           for (int u = 0; u < BATCH; ++u)
             if (q[u] >= 0) fn(j00 + u * NT + lane, col[u]);
@@ -267,7 +283,8 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
     for (int tile = 0; tile < ntiles; ++tile) {
       const int lo = lo0 + (tile << lw);
       // ---- pass 1: claim bits; first claimers flagged -----------------------------------------
-      int cbase = 0;
+      cbase = 0;
+      cmode = ccache ? (tile == 0 ? 1 : 2) : 0;
       for (int c = 0; c < nchunks; ++c) {
         if (nchunks > 1 || tile == 0) {
           gather(c);
@@ -395,7 +412,7 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
             uint8_t fb[BATCH];
 #pragma unroll
             for (int u = 0; u < BATCH; ++u) {
-              col[u] = q[u] >= 0 ? P.colB[sbs[rr[u]] + q[u]] : -1;
+              col[u] = q[u] < 0 ? -1 : (ccache ? ccache[cbase + j00 + u * NT + lane] : P.colB[sbs[rr[u]] + q[u]]);
               fb[u] = q[u] >= 0 ? frow8[cbase + j00 + u * NT + lane] : 0;
             }
 #pragma unroll
@@ -429,6 +446,10 @@ __global__ void __launch_bounds__(NT, SMEM > 120 * 1024 ? 1 : 2) k_bitmap_rank(S
       }
       if (CACHED)
         for (int x = tid; x < nfw; x += NT) flags[x] = 0;
+      __syncthreads();
+    }
+    if (ccache) {  // the zero invariant of the region
+      for (int x = tid; x < f; x += NT) ccache[x] = 0;
       __syncthreads();
     }
     if constexpr (CACHED) {

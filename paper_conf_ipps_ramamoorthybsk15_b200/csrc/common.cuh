@@ -88,7 +88,10 @@ struct Group {
   __device__ __forceinline__ void sync() const {
     if constexpr (G == 32) __syncwarp(); else __syncthreads();
   }
-  // Exclusive scan of v over the group; *total = group sum.  All G threads must call.
+  // Exclusive scan of v over the group; *total = group sum.  All G threads must call.  TRAIL =
+  // false drops the closing barrier that protects the scratch words from the next scan: only for
+  // call sites followed by a barrier of their own before the group scans again.
+  template <bool TRAIL = true>
   __device__ __forceinline__ int excl_scan(int v, int& total) const {
     int incl = warp_incl_scan(v);
     if constexpr (G == 32) {
@@ -108,7 +111,7 @@ struct Group {
       __syncthreads();
       int r = incl - v + scratch[w];
       total = scratch[NW];
-      __syncthreads();
+      if constexpr (TRAIL) __syncthreads();
       return r;
     }
   }

@@ -27,7 +27,8 @@
 //                bucketed by the numeric unit that owns that output.  SINGLE rows (one non-empty
 //                B row, already sorted) write their products in order.
 // This is Phase IV's "sort, mark like-tuples, scan, compact", done per batch
-// in shared memory.
+// in shared memory.  Every block scan here is followed by a barrier of its own before the next
+// one, so the scans skip their closing barrier (excl_scan<false>).
 #include "kernels.cuh"
 
 namespace spg {
@@ -273,7 +274,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
           }
         }
         int tot;
-        const int ex = g.excl_scan((L << 16) | (L > 0 ? 1 : 0), tot);  // L <= PT <= 2^12, runs <= NT
+        const int ex = g.template excl_scan<false>((L << 16) | (L > 0 ? 1 : 0), tot);  // L <= PT <= 2^12, runs <= NT
         const int slot = ex & 0xffff, nrun = tot & 0xffff, Lt = tot >> 16;
         if (L > 0) {
           seg[slot] = ex >> 16;
@@ -329,7 +330,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
           nb = (int)nbu;
         }
         int tot;
-        const int ex = g.excl_scan(nb, tot);
+        const int ex = g.template excl_scan<false>(nb, tot);
         if (tid < NR) s_bb[tid] = ex;
         if (tid == 0) s_bb[NR] = tot;
       }
@@ -374,7 +375,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
           mine += c8[k];
         }
         int tot;
-        int run = g.excl_scan(mine, tot);
+        int run = g.template excl_scan<false>(mine, tot);
 #pragma unroll
         for (int k = 0; k < BPT; ++k) {
           const int b = tid * BPT + k;
@@ -453,7 +454,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
           }
         }
         int tot;
-        int run = g.excl_scan(nh, tot);  // (its barriers order the reads above before the writes below)
+        int run = g.template excl_scan<false>(nh, tot);  // (its barriers order the reads above before the writes below)
 #pragma unroll
         for (int k = 0; k < IPT; ++k) {
           const int x = tid * IPT + k;
@@ -486,7 +487,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
           P.crow[s_row[tid] + 1] = cj;
         }
         int tot;
-        const int ex = g.excl_scan(cj, tot);
+        const int ex = g.template excl_scan<false>(cj, tot);
         if (tid < NR) s_out[tid] = ex;
         if (tid == 0) s_out[NR] = tot;
       }

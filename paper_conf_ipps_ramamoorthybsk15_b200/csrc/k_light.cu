@@ -197,6 +197,8 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
       const int NI = s_nb;
       if (NI == 0) break;
       const int NR = s_irb[NI];
+      // the bucket counters of step 3, zeroed here (the barriers of steps 1-2 order it)
+      for (int b = tid; b <= C::NB; b += NT) cnt[b] = 0;
 
       // ---- 1. rows: tile, first A entry, A entries and products (block scans) ------------------------
       int ii = 0, j_al = 0, j_f = 0;
@@ -336,8 +338,6 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
       }
       __syncthreads();
       const int NBt = s_bb[NR];
-      for (int b = tid; b <= NBt; b += NT) cnt[b] = 0;
-      __syncthreads();
       // bucket of product idx (light rows; -1: SINGLE row, no sort)
       auto bucket_of = [&](int idx) -> int {
         const int j = exrow[idx];

@@ -530,6 +530,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
           P.plan[s_iP0[it] + s_out[j] - s_out[s_irb[it]] + idx - s_pf[j]] = pay[idx];
         }
       __syncthreads();
+      if (PT == s_out[NR]) continue;  // no repeated product in the batch (block-uniform): no R records
       if (tid < NI) {  // R records of the tile's repeats, bucketed by numeric unit (dub: first record)
         const int x = tid;
         const int C = s_out[s_irb[x + 1]] - s_out[s_irb[x]];

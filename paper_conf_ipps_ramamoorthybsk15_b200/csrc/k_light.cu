@@ -492,20 +492,23 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
         if (tid == 0) s_out[NR] = tot;
       }
       __syncthreads();
-      if (tid == 0) {  // per tile: repeats (statistics), numeric-unit bases of the repeat counters
-        long long dups = 0;
-        int ub = 0;
-        for (int x = 0; x < NI; ++x) {
-          const int C = s_out[s_irb[x + 1]] - s_out[s_irb[x]];
-          dups += (s_pf[s_irb[x + 1]] - s_pf[s_irb[x]]) - C;
-          s_iub[x] = ub;
-          ub += (C + NUM_SH - 1) / NUM_SH;
+      const bool reps = PT != s_out[NR];  // the batch has repeated products (block-uniform)
+      if (reps) {
+        if (tid == 0) {  // per tile: repeats (statistics), numeric-unit bases of the repeat counters
+          long long dups = 0;
+          int ub = 0;
+          for (int x = 0; x < NI; ++x) {
+            const int C = s_out[s_irb[x + 1]] - s_out[s_irb[x]];
+            dups += (s_pf[s_irb[x + 1]] - s_pf[s_irb[x]]) - C;
+            s_iub[x] = ub;
+            ub += (C + NUM_SH - 1) / NUM_SH;
+          }
+          s_iub[NI] = ub;
+          if (dups) atomicAdd(reinterpret_cast<unsigned long long*>(P.dups_all), (unsigned long long)dups);
         }
-        s_iub[NI] = ub;
-        if (dups) atomicAdd(reinterpret_cast<unsigned long long*>(P.dups_all), (unsigned long long)dups);
+        if (tid < C::NU) s_uc[tid] = 0;
+        __syncthreads();
       }
-      if (tid < C::NU) s_uc[tid] = 0;
-      __syncthreads();
 
       // ---- 8. plan: heads in C order; repeats after them, bucketed by numeric unit ----------------
       for (int x = tid; x < Pg; x += NT) {
@@ -530,7 +533,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
           P.plan[s_iP0[it] + s_out[j] - s_out[s_irb[it]] + idx - s_pf[j]] = pay[idx];
         }
       __syncthreads();
-      if (PT == s_out[NR]) continue;  // no repeated product in the batch (block-uniform): no R records
+      if (!reps) continue;  // no repeated product in the batch: no R records
       if (tid < NI) {  // R records of the tile's repeats, bucketed by numeric unit (dub: first record)
         const int x = tid;
         const int C = s_out[s_irb[x + 1]] - s_out[s_irb[x]];

@@ -81,7 +81,8 @@ struct TileSmem {
   static constexpr int pf = ae + (C::RM + 1) * 4;                // int[RM+1]   product offset of the row
   static constexpr int bb = pf + (C::RM + 1) * 4;                // int[RM+1]   bucket base
   static constexpr int out = bb + (C::RM + 1) * 4;               // int[RM+1]   output offset in the batch
-  static constexpr int rpa = out + (C::RM + 1) * 4;              // int[RM]     first A entry of the row
+  static constexpr int sf = out + (C::RM + 1) * 4;               // int[RM+1]   SINGLE-row products before the row
+  static constexpr int rpa = sf + (C::RM + 1) * 4;               // int[RM]     first A entry of the row
   static constexpr int row = rpa + C::RM * 4;                    // int[RM]     local row index
   static constexpr int cmin = row + C::RM * 4;                   // int[RM]     column range of the row (later:
                                                                   //             heads before the row)
@@ -112,6 +113,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
   int* s_pf = reinterpret_cast<int*>(sm + SM::pf);
   int* s_bb = reinterpret_cast<int*>(sm + SM::bb);
   int* s_out = reinterpret_cast<int*>(sm + SM::out);
+  int* s_sf = reinterpret_cast<int*>(sm + SM::sf);
   int* s_rpa = reinterpret_cast<int*>(sm + SM::rpa);
   int* s_row = reinterpret_cast<int*>(sm + SM::row);
   int* s_cmin = reinterpret_cast<int*>(sm + SM::cmin);
@@ -201,7 +203,7 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
       for (int b = tid; b <= C::NB; b += NT) cnt[b] = 0;
 
       // ---- 1. rows: tile, first A entry, A entries and products (block scans) ------------------------
-      int ii = 0, j_al = 0, j_f = 0;
+      int ii = 0, j_al = 0, j_f = 0, j_s = 0;
       if (tid < NR) {
         ii = upper_idx(s_irb, NI, tid);
         const int li = s_qr0[s_bi[ii]] + (tid - s_irb[ii]);
@@ -212,15 +214,18 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
         s_row[tid] = li;
         s_rpa[tid] = pa;
         s_item[tid] = (uint8_t)ii;
-        s_kind[tid] = P.cls[li] & 7;
+        const int k1 = P.cls[li] & 7;
+        s_kind[tid] = (uint8_t)k1;
+        j_s = k1 == CLS_SINGLE ? j_f : 0;
         s_cmin[tid] = INT_MAX;
         s_cmax[tid] = -1;
       }
       {
         int2 tot;
         const int lane_ = tid & 31, w_ = tid >> 5;
-        // exclusive scans of (A entries, products) over the batch rows
-        int ia = j_al, ib = j_f;
+        // exclusive scans of (A entries, products | SINGLE-row products << 16) over the batch rows
+        // (both halves sum to <= PMAX < 2^16)
+        int ia = j_al, ib = j_f | (j_s << 16);
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
           const int oa = __shfl_up_sync(FULL, ia, d), ob = __shfl_up_sync(FULL, ib, d);
@@ -243,12 +248,15 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
         const int2 base = scratch2[w_];
         tot = scratch2[NW];
         if (tid < NR) {
+          const int ex = base.y + ib - (j_f | (j_s << 16));
           s_ae[tid] = base.x + ia - j_al;
-          s_pf[tid] = base.y + ib - j_f;
+          s_pf[tid] = ex & 0xffff;
+          s_sf[tid] = ex >> 16;
         }
         if (tid == 0) {
           s_ae[NR] = tot.x;
-          s_pf[NR] = tot.y;
+          s_pf[NR] = tot.y & 0xffff;
+          s_sf[NR] = tot.y >> 16;
         }
       }
       __syncthreads();
@@ -468,30 +476,20 @@ __global__ void __launch_bounds__(C::NT) k_tile_rank(SymProb P, const int* __res
       }
       __syncthreads();
 
-      // ---- 7. c_j and output offsets of the rows (in the batch; a tile's outputs start at the
-      //         offset of its first row); s_cmin[j] = heads before row j's first slot -------------
-      {
-        int cj = 0;
-        if (tid < NR) {
-          const int k = s_kind[tid];
-          if (k >= CLS_TINY) {
-            const int b0 = s_bb[tid], b1 = s_bb[tid + 1];
-            const int x0 = b0 ? cnt[b0 - 1] : 0, x1 = b1 ? cnt[b1 - 1] : 0;
-            const int h0 = x0 < Pg ? keys[x0] & 0x7fffffff : s_htot;  // (a row's first slot is a head)
-            const int h1 = x1 < Pg ? keys[x1] & 0x7fffffff : s_htot;
-            cj = h1 - h0;
-            s_cmin[tid] = h0;
-          } else if (k == CLS_SINGLE) {
-            cj = s_pf[tid + 1] - s_pf[tid];
-          }
-          P.crow[s_row[tid] + 1] = cj;
-        }
-        int tot;
-        const int ex = g.template excl_scan<false>(cj, tot);
-        if (tid < NR) s_out[tid] = ex;
-        if (tid == 0) s_out[NR] = tot;
+      // ---- 7. output offsets of the rows (in the batch; a tile's outputs start at the offset of its
+      //         first row) without a scan: heads before the row's first slot (that slot is a head;
+      //         for a row without buckets, the next light row's) + SINGLE-row products before it;
+      //         s_cmin[j] = the heads before row j -----------------------------------------------------
+      if (tid < NR) {
+        const int b0 = s_bb[tid];
+        const int x0 = b0 ? cnt[b0 - 1] : 0;
+        const int h = x0 < Pg ? keys[x0] & 0x7fffffff : s_htot;
+        s_out[tid] = h + s_sf[tid];
+        s_cmin[tid] = h;
       }
+      if (tid == 0) s_out[NR] = s_htot + s_sf[NR];
       __syncthreads();
+      if (tid < NR) P.crow[s_row[tid] + 1] = s_out[tid + 1] - s_out[tid];  // c_j
       const bool reps = PT != s_out[NR];  // the batch has repeated products (block-uniform)
       if (reps) {
         if (tid == 0) {  // per tile: repeats (statistics), numeric-unit bases of the repeat counters
